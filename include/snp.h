@@ -1,0 +1,171 @@
+/*
+ * snp.h — C ABI of the B200-native SNP-comparison library (libsnp.so).
+ *
+ * The library computes the one data-parallel hot path of Binder, Low & Popovici,
+ * "A Portable GPU Framework for SNP Comparisons" (IPDPS-W 2019): SNP comparison
+ * cast as a binary matrix product (§II.A, §III)
+ *
+ *     C[i][j] = sum_w POPC( A[i][w]  op  B[j][w] )
+ *
+ * over bit-packed genotype rows, with op = AND (LD, Eq. 1),
+ * XOR (FastID identity search, Eq. 2) or AND-NOT (FastID mixture
+ * analysis, Eq. 3 rewritten as r & ~m).  P:Lnn is a line of the
+ * paper text.
+ *
+ * Conventions shared by every call
+ * --------------------------------
+ *  - Packed layout (§III, Fig. 2): row r of a packed matrix is `ld`
+ *    consecutive little-endian uint64 words; sample/SNP k of the row is bit
+ *    (k % 64) of word (k / 64) (LSB first).  Bits >= nbits are IGNORED by every
+ *    compute call (the kernels mask them), so padding contents never matter;
+ *    snp_pack writes them as zero.  LD matrices pack along samples (rows are
+ *    SNPs); FastID matrices pack along SNPs (rows are profiles).  Both operands
+ *    are therefore K-contiguous and C = A . B^T.
+ *  - Pointers are CUDA DEVICE pointers unless marked (host).  Matrix pointers
+ *    must be 16-byte aligned and every leading dimension of a packed matrix
+ *    (in uint64 words) must be even (128-bit rows), else SNP_E_ALIGN.
+ *  - Every compute call is asynchronous and stream-ordered on `stream` (a
+ *    cudaStream_t passed as void*; NULL = legacy default stream).  The library
+ *    allocates no device memory: the caller owns every buffer, including the
+ *    workspace `ws` sized by the *_workspace_bytes queries.  No pointer is kept
+ *    after the call returns.
+ *  - Arguments are validated synchronously before any launch; an invalid call
+ *    launches nothing.  Device faults surface at the caller's next sync.
+ *  - m == 0 or n == 0 is a valid no-op returning SNP_OK.
+ *  - Outputs must not alias inputs.  B == A (self-LD) is allowed.
+ *  - The library runs only on compute capability 10.0 (B200, sm_100a); any
+ *    other device returns SNP_E_ARCH.  There is no fallback.
+ *  - Calls are re-entrant.  Process-wide state: a per-device property cache and
+ *    the variant override of snp_set_variant.
+ */
+#ifndef SNP_H_
+#define SNP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    SNP_OK = 0,
+    SNP_E_NULL = 1,      /* a required pointer is NULL                          */
+    SNP_E_SHAPE = 2,     /* negative size, ld < ceil(nbits/64), ldc < n, nbits<1 */
+    SNP_E_ALIGN = 3,     /* pointer not 16-byte aligned or odd packed ld        */
+    SNP_E_OP = 4,        /* unknown snp_op / snp_variant                        */
+    SNP_E_RANGE = 5,     /* nbits too large for uint32 counts, bad shard args   */
+    SNP_E_WORKSPACE = 6, /* ws smaller than the workspace query returned        */
+    SNP_E_ARCH = 7,      /* current device is not compute capability 10.0      */
+    SNP_E_CUDA = 8       /* a CUDA runtime/launch error (see snp_last_cuda_error) */
+} snp_status;
+
+/* Bitwise comparison applied per word before POPC.  Q is the first operand
+ * (query / A rows), D the second (database / B rows). */
+typedef enum {
+    SNP_OP_AND = 0,    /* popc(Q & D)   Eq. (1), P:L52 (LD p_AB term)                */
+    SNP_OP_XOR = 1,    /* popc(Q ^ D)   Eq. (2), P:L60 (identity search, 0 = match)  */
+    SNP_OP_ANDNOT = 2, /* popc(Q & ~D)  Eq. (3) with r = query, m = database row
+                          ("m ... negated and stored in the database")      */
+    SNP_OP_NOTAND = 3  /* popc(~Q & D)  Eq. (3) with r = database row, m = query     */
+} snp_op;
+
+/* Kernel variant selection (process-wide; default SNP_VARIANT_AUTO). */
+typedef enum {
+    SNP_VARIANT_AUTO = 0, /* pick per shape from the measured dispatch table    */
+    SNP_VARIANT_POPC = 1, /* CUDA-core LOP3 + POPC register-blocked bit-GEMM     */
+    SNP_VARIANT_TC = 2    /* tcgen05 kind::i8 tensor-core GEMM on bit-expanded operands */
+} snp_variant;
+
+/* Recommended packed leading dimension (uint64 words) for nbits bits:
+ * ceil(nbits/64) rounded up to a multiple of 8 (64-byte rows).  Any even
+ * ld >= ceil(nbits/64) is accepted.  Returns 0 for nbits <= 0. */
+int64_t snp_words(int64_t nbits);
+
+/* Bytes of device workspace snp_ld_counts / snp_ld_r2 need for this shape
+ * under the current variant choice (0 if none).  ws may be NULL when 0. */
+size_t snp_ld_workspace_bytes(int64_t m, int64_t n, int64_t nbits);
+
+/* Bytes of device workspace snp_fastid needs (0 if none). */
+size_t snp_fastid_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op);
+
+/* a1 — encode + pack (§III, Fig. 2).  g: uint8 genotypes [rows][ldg_bytes],
+ * byte k of row r is sample/SNP k (non-zero = minor allele = 1, zero = major = 0).
+ * packed: uint64 [rows][ldw] output; bits >= nbits and words >= ceil(nbits/64)
+ * are written as 0.  g has no alignment requirement; ldg_bytes >= nbits. */
+snp_status snp_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg_bytes,
+                    uint64_t *packed, int64_t ldw, void *stream);
+
+/* a2 — popc[r] = number of set bits among the first nbits of packed row r
+ * (p_A / p_B of P:L44 as counts). */
+snp_status snp_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int64_t ldw,
+                        uint32_t *popc, void *stream);
+
+/* a3 — LD counts (Eq. 1; GEMM update P:L116):
+ *   C[i*ldc + j] (=|+=) sum_k A_ik & B_jk,   i < m, j < n, k < nbits.
+ * A: [m][lda] packed SNP rows over samples, B: [n][ldb].  C: uint32 [m][ldc].
+ * accumulate = 0 overwrites C, 1 adds (callers may split K into chunks). */
+snp_status snp_ld_counts(const uint64_t *A, int64_t m, int64_t lda,
+                         const uint64_t *B, int64_t n, int64_t ldb, int64_t nbits,
+                         uint32_t *C, int64_t ldc, int accumulate,
+                         void *ws, size_t ws_bytes, void *stream);
+
+/* a3 + a5 — LD statistics for every SNP pair, n = nbits samples:
+ *   num = n*nAB - nA*nB (= n^2 D_AB, exact), den = nA(n-nA) nB(n-nB),
+ *   r2 = num^2/den (0 when den == 0, i.e. a monomorphic SNP),
+ *   D' = num/Dmax, Dmax = min(nA(n-nB),(n-nA)nB) if num>0 else min(nA nB,(n-nA)(n-nB))
+ *   (0 when num == 0).  Computed from exact integers in fp64, stored fp32.
+ * popA/popB: optional precomputed row popcounts (NULL = computed internally).
+ * r2: float [m][ldc] (required); dprime: float [m][ldc] or NULL;
+ * counts: uint32 nAB [m][ldc] or NULL. */
+snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *popA,
+                     const uint64_t *B, int64_t n, int64_t ldb, const uint32_t *popB,
+                     int64_t nbits, float *r2, float *dprime, uint32_t *counts,
+                     int64_t ldc, void *ws, size_t ws_bytes, void *stream);
+
+/* a3 + a4 — FastID comparison counts (Eqs. 2-3):
+ *   out[i*ldo + j] (=|+=) sum_k op(Q_ik, D_jk)   for queries i < nq, DB rows j < nd.
+ * Q: [nq][ldq] packed query profiles over SNPs, D: [nd][ldd] database profiles.
+ * popQ/popD: optional row popcounts (used by the tensor variant's identities
+ * XOR = pQ + pD - 2 AND, ANDNOT = pQ - AND, NOTAND = pD - AND; NULL = computed
+ * internally).  out: uint32 [nq][ldo], ldo >= nd. */
+snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t *popQ,
+                      const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD,
+                      int64_t nbits, int op, uint32_t *out, int64_t ldo, int accumulate,
+                      void *ws, size_t ws_bytes, void *stream);
+
+/* a6 — best match per query over a count matrix ("No set bits ...
+ * signifies a positive match"; P:L62 larger = less likely):
+ *   best_count[i] = min_j counts[i*ldo + j],
+ *   best_index[i] = index_base + (lowest j attaining it); nd == 0 gives
+ *   best_count = 0xFFFFFFFF, best_index = -1.  nd < 2^32. */
+snp_status snp_fastid_best(const uint32_t *counts, int64_t nq, int64_t nd, int64_t ldo,
+                           int64_t index_base, uint32_t *best_count, int64_t *best_index,
+                           void *stream);
+
+/* e — multi-GPU row partition (host only, no device access): rows [0, rows)
+ * split into `world` contiguous ranges bounds[r] .. bounds[r+1] (bounds is a
+ * HOST array of world+1 int64), each boundary a multiple of `align` (except
+ * bounds clamped to rows), block counts balanced to within one.  Deterministic.
+ * SNP_E_RANGE for world < 1, align < 1 or rows < 0. */
+snp_status snp_shard_plan(int64_t rows, int world, int64_t align, int64_t *bounds);
+
+/* Variant override (SNP_VARIANT_AUTO restores the dispatch table).  The
+ * environment variable SNP_FORCE_VARIANT=popc|tc sets the initial value. */
+snp_status snp_set_variant(int variant);
+/* Variant used by the most recent successful compute call on this thread. */
+int snp_last_variant(void);
+
+/* Cumulative number of CUDA kernels this library has launched in this process
+ * (evidence for benchmarks: every launch is one of the library's own kernels). */
+int64_t snp_launch_count(void);
+
+/* Static description of a status code. */
+const char *snp_status_string(int status);
+/* Text of the last CUDA error seen by a call on this thread ("" if none). */
+const char *snp_last_cuda_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SNP_H_ */

@@ -1,0 +1,340 @@
+// snp_api.cu — the C ABI (include/snp.h): validation, architecture check, variant
+// dispatch and launches.  Every entry point validates synchronously before any
+// launch and never allocates device memory.
+#include "../../include/snp.h"
+#include "snp_internal.h"
+
+#include <atomic>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+
+using namespace snp;
+
+namespace {
+
+thread_local char g_cuda_err[256] = "";
+thread_local int g_last_variant = 0;
+
+std::atomic<int> g_variant{-1};   // -1: not yet read from the environment
+std::atomic<long long> g_launches{0};
+
+int current_variant() {
+    int v = g_variant.load(std::memory_order_relaxed);
+    if (v < 0) {
+        int init = SNP_VARIANT_AUTO;
+        const char *e = std::getenv("SNP_FORCE_VARIANT");
+        if (e) {
+            if (!std::strcmp(e, "popc")) init = SNP_VARIANT_POPC;
+            else if (!std::strcmp(e, "tc")) init = SNP_VARIANT_TC;
+        }
+        int expected = -1;
+        g_variant.compare_exchange_strong(expected, init);
+        v = g_variant.load();
+    }
+    return v;
+}
+
+// Per-device compute-capability cache (the only other process-wide state).
+std::atomic<int> g_cc[128];
+
+snp_status set_cuda_error(cudaError_t e) {
+    std::snprintf(g_cuda_err, sizeof(g_cuda_err), "%s: %s", cudaGetErrorName(e),
+                  cudaGetErrorString(e));
+    return SNP_E_CUDA;
+}
+
+snp_status check_arch() {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) {
+        set_cuda_error(e);
+        cudaGetLastError();
+        return SNP_E_ARCH;
+    }
+    if (dev < 0 || dev >= 128) return SNP_E_ARCH;
+    int cc = g_cc[dev].load(std::memory_order_relaxed);
+    if (cc == 0) {
+        int major = 0, minor = 0;
+        if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess ||
+            cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev) != cudaSuccess) {
+            cudaGetLastError();
+            return SNP_E_ARCH;
+        }
+        cc = major * 10 + minor;
+        g_cc[dev].store(cc);
+    }
+    return cc == 100 ? SNP_OK : SNP_E_ARCH;
+}
+
+inline bool aligned16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
+inline int64_t words_needed(int64_t nbits) { return (nbits + 63) / 64; }
+inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+// Validation of one packed operand.
+snp_status check_packed(const void *p, int64_t rows, int64_t ld, int64_t nbits) {
+    if (rows < 0 || ld < 0) return SNP_E_SHAPE;
+    if (rows == 0) return SNP_OK;
+    if (!p) return SNP_E_NULL;
+    if (ld < words_needed(nbits)) return SNP_E_SHAPE;
+    if (!aligned16(p) || (ld & 1)) return SNP_E_ALIGN;
+    return SNP_OK;
+}
+
+snp_status check_nbits(int64_t nbits) {
+    if (nbits < 1) return SNP_E_SHAPE;
+    if (nbits > 0x7fffffffLL) return SNP_E_RANGE;   // counts are uint32; LD math int64
+    return SNP_OK;
+}
+
+// Variant choice per shape (a7).  Measured dispatch: the tensor-core variant wins
+// whenever it supports the shape (>= 15x the POPC roof); the POPC
+// variant covers everything else and is kept as the forced/reference variant.
+int choose_variant(int64_t m, int64_t n, int64_t nbits) {
+    const int v = current_variant();
+    if (v == SNP_VARIANT_POPC) return SNP_VARIANT_POPC;
+    if (v == SNP_VARIANT_TC) return SNP_VARIANT_TC;
+    return tc_supported(m, n, nbits) ? SNP_VARIANT_TC : SNP_VARIANT_POPC;
+}
+
+size_t pops_bytes(int64_t m, int64_t n) { return align256((size_t)m * 4) + align256((size_t)n * 4); }
+
+snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes, cudaStream_t s) {
+    cudaError_t e;
+    if (variant == SNP_VARIANT_TC) {
+        if (!tc_supported(a.m, a.n, a.nbits)) return SNP_E_SHAPE;
+        e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
+    } else {
+        e = launch_bitgemm_popc(a, epi, s);
+    }
+    if (e != cudaSuccess) return set_cuda_error(e);
+    g_last_variant = variant;
+    return SNP_OK;
+}
+
+}  // namespace
+
+namespace snp {
+void count_launches(int k) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+}  // namespace snp
+
+extern "C" {
+
+int64_t snp_words(int64_t nbits) {
+    if (nbits <= 0) return 0;
+    return ((words_needed(nbits) + 7) / 8) * 8;
+}
+
+size_t snp_ld_workspace_bytes(int64_t m, int64_t n, int64_t nbits) {
+    if (m <= 0 || n <= 0 || nbits <= 0) return 0;
+    size_t b = pops_bytes(m, n);
+    if (choose_variant(m, n, nbits) == SNP_VARIANT_TC) b += tc_workspace_bytes(m, n, nbits);
+    return b;
+}
+
+size_t snp_fastid_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op) {
+    (void)op;
+    if (nq <= 0 || nd <= 0 || nbits <= 0) return 0;
+    if (choose_variant(nq, nd, nbits) != SNP_VARIANT_TC) return 0;
+    return pops_bytes(nq, nd) + tc_workspace_bytes(nq, nd, nbits);
+}
+
+snp_status snp_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg_bytes,
+                    uint64_t *packed, int64_t ldw, void *stream) {
+    if (rows < 0 || nbits < 0 || ldg_bytes < 0 || ldw < 0) return SNP_E_SHAPE;
+    if (rows == 0) return SNP_OK;
+    if (!g || !packed) return SNP_E_NULL;
+    if (nbits < 1 || ldg_bytes < nbits || ldw < words_needed(nbits)) return SNP_E_SHAPE;
+    if (!aligned16(packed) || (ldw & 1)) return SNP_E_ALIGN;
+    snp_status st = check_arch();
+    if (st != SNP_OK) return st;
+    cudaError_t e = launch_pack(g, rows, nbits, ldg_bytes, packed, ldw, (cudaStream_t)stream);
+    return e == cudaSuccess ? SNP_OK : set_cuda_error(e);
+}
+
+snp_status snp_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int64_t ldw,
+                        uint32_t *popc, void *stream) {
+    snp_status st = check_nbits(nbits);
+    if (rows < 0) return SNP_E_SHAPE;
+    if (st != SNP_OK) return st;
+    if ((st = check_packed(x, rows, ldw, nbits)) != SNP_OK) return st;
+    if (rows == 0) return SNP_OK;
+    if (!popc) return SNP_E_NULL;
+    if ((st = check_arch()) != SNP_OK) return st;
+    cudaError_t e = launch_row_popc(x, rows, nbits, ldw, popc, (cudaStream_t)stream);
+    return e == cudaSuccess ? SNP_OK : set_cuda_error(e);
+}
+
+snp_status snp_ld_counts(const uint64_t *A, int64_t m, int64_t lda,
+                         const uint64_t *B, int64_t n, int64_t ldb, int64_t nbits,
+                         uint32_t *C, int64_t ldc, int accumulate,
+                         void *ws, size_t ws_bytes, void *stream) {
+    snp_status st;
+    if (m < 0 || n < 0) return SNP_E_SHAPE;
+    if ((st = check_nbits(nbits)) != SNP_OK) return st;
+    if ((st = check_packed(A, m, lda, nbits)) != SNP_OK) return st;
+    if ((st = check_packed(B, n, ldb, nbits)) != SNP_OK) return st;
+    if (m == 0 || n == 0) return SNP_OK;
+    if (!C) return SNP_E_NULL;
+    if (ldc < n) return SNP_E_SHAPE;
+    if (!aligned16(C)) return SNP_E_ALIGN;
+    const int variant = choose_variant(m, n, nbits);
+    const size_t need = snp_ld_workspace_bytes(m, n, nbits);
+    if (ws_bytes < need || (need && !ws)) return SNP_E_WORKSPACE;
+    if ((st = check_arch()) != SNP_OK) return st;
+    GemmArgs a{};
+    a.A = reinterpret_cast<const uint32_t *>(A);
+    a.B = reinterpret_cast<const uint32_t *>(B);
+    a.m = m; a.n = n; a.lda32 = 2 * lda; a.ldb32 = 2 * ldb; a.nbits = nbits;
+    a.op = SNP_OP_AND; a.accumulate = accumulate ? 1 : 0; a.ldc = ldc; a.C = C;
+    void *tcws = variant == SNP_VARIANT_TC ? (char *)ws + pops_bytes(m, n) : nullptr;
+    size_t tcbytes = variant == SNP_VARIANT_TC ? ws_bytes - pops_bytes(m, n) : 0;
+    return run_gemm(a, EPI_COUNTS, variant, tcws, tcbytes, (cudaStream_t)stream);
+}
+
+snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *popA,
+                     const uint64_t *B, int64_t n, int64_t ldb, const uint32_t *popB,
+                     int64_t nbits, float *r2, float *dprime, uint32_t *counts,
+                     int64_t ldc, void *ws, size_t ws_bytes, void *stream) {
+    snp_status st;
+    if (m < 0 || n < 0) return SNP_E_SHAPE;
+    if ((st = check_nbits(nbits)) != SNP_OK) return st;
+    if ((st = check_packed(A, m, lda, nbits)) != SNP_OK) return st;
+    if ((st = check_packed(B, n, ldb, nbits)) != SNP_OK) return st;
+    if (m == 0 || n == 0) return SNP_OK;
+    if (!r2) return SNP_E_NULL;
+    if (ldc < n) return SNP_E_SHAPE;
+    if (!aligned16(r2) || (dprime && !aligned16(dprime)) || (counts && !aligned16(counts)))
+        return SNP_E_ALIGN;
+    if (nbits > 0xB504F33LL) return SNP_E_RANGE;   // n^2 products must stay exact in int64/fp64
+    const int variant = choose_variant(m, n, nbits);
+    const size_t need = snp_ld_workspace_bytes(m, n, nbits);
+    if (ws_bytes < need || !ws) return SNP_E_WORKSPACE;
+    if ((st = check_arch()) != SNP_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    uint32_t *pa = reinterpret_cast<uint32_t *>(ws);
+    uint32_t *pb = reinterpret_cast<uint32_t *>((char *)ws + align256((size_t)m * 4));
+    cudaError_t e;
+    if (!popA) {
+        if ((e = launch_row_popc(A, m, nbits, lda, pa, s)) != cudaSuccess) return set_cuda_error(e);
+        popA = pa;
+    }
+    if (!popB) {
+        if ((e = launch_row_popc(B, n, nbits, ldb, pb, s)) != cudaSuccess) return set_cuda_error(e);
+        popB = pb;
+    }
+    GemmArgs a{};
+    a.A = reinterpret_cast<const uint32_t *>(A);
+    a.B = reinterpret_cast<const uint32_t *>(B);
+    a.m = m; a.n = n; a.lda32 = 2 * lda; a.ldb32 = 2 * ldb; a.nbits = nbits;
+    a.op = SNP_OP_AND; a.accumulate = 0; a.ldc = ldc; a.C = counts;
+    a.r2 = r2; a.dprime = dprime; a.popA = popA; a.popB = popB;
+    void *tcws = variant == SNP_VARIANT_TC ? (char *)ws + pops_bytes(m, n) : nullptr;
+    size_t tcbytes = variant == SNP_VARIANT_TC ? ws_bytes - pops_bytes(m, n) : 0;
+    return run_gemm(a, EPI_LD, variant, tcws, tcbytes, s);
+}
+
+snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t *popQ,
+                      const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD,
+                      int64_t nbits, int op, uint32_t *out, int64_t ldo, int accumulate,
+                      void *ws, size_t ws_bytes, void *stream) {
+    snp_status st;
+    if (nq < 0 || nd < 0) return SNP_E_SHAPE;
+    if (op < SNP_OP_AND || op > SNP_OP_NOTAND) return SNP_E_OP;
+    if ((st = check_nbits(nbits)) != SNP_OK) return st;
+    if ((st = check_packed(Q, nq, ldq, nbits)) != SNP_OK) return st;
+    if ((st = check_packed(D, nd, ldd, nbits)) != SNP_OK) return st;
+    if (nq == 0 || nd == 0) return SNP_OK;
+    if (!out) return SNP_E_NULL;
+    if (ldo < nd) return SNP_E_SHAPE;
+    if (!aligned16(out)) return SNP_E_ALIGN;
+    const int variant = choose_variant(nq, nd, nbits);
+    const size_t need = snp_fastid_workspace_bytes(nq, nd, nbits, op);
+    if (ws_bytes < need || (need && !ws)) return SNP_E_WORKSPACE;
+    if ((st = check_arch()) != SNP_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    GemmArgs a{};
+    a.A = reinterpret_cast<const uint32_t *>(Q);
+    a.B = reinterpret_cast<const uint32_t *>(D);
+    a.m = nq; a.n = nd; a.lda32 = 2 * ldq; a.ldb32 = 2 * ldd; a.nbits = nbits;
+    a.op = op; a.accumulate = accumulate ? 1 : 0; a.ldc = ldo; a.C = out;
+    if (variant == SNP_VARIANT_TC) {
+        uint32_t *pq = reinterpret_cast<uint32_t *>(ws);
+        uint32_t *pd = reinterpret_cast<uint32_t *>((char *)ws + align256((size_t)nq * 4));
+        cudaError_t e;
+        if (op != SNP_OP_AND && !popQ) {
+            if ((e = launch_row_popc(Q, nq, nbits, ldq, pq, s)) != cudaSuccess) return set_cuda_error(e);
+            popQ = pq;
+        }
+        if ((op == SNP_OP_XOR || op == SNP_OP_NOTAND) && !popD) {
+            if ((e = launch_row_popc(D, nd, nbits, ldd, pd, s)) != cudaSuccess) return set_cuda_error(e);
+            popD = pd;
+        }
+        a.popA = popQ; a.popB = popD;
+        return run_gemm(a, EPI_COUNTS, variant, (char *)ws + pops_bytes(nq, nd),
+                        ws_bytes - pops_bytes(nq, nd), s);
+    }
+    return run_gemm(a, EPI_COUNTS, variant, nullptr, 0, s);
+}
+
+snp_status snp_fastid_best(const uint32_t *counts, int64_t nq, int64_t nd, int64_t ldo,
+                           int64_t index_base, uint32_t *best_count, int64_t *best_index,
+                           void *stream) {
+    if (nq < 0 || nd < 0) return SNP_E_SHAPE;
+    if (nd > 0xfffffffeLL) return SNP_E_RANGE;
+    if (nq == 0) return SNP_OK;
+    if (!best_count || !best_index || (nd > 0 && !counts)) return SNP_E_NULL;
+    if (ldo < nd) return SNP_E_SHAPE;
+    if (((uintptr_t)best_index & 7u) || ((uintptr_t)best_count & 3u) || ((uintptr_t)counts & 3u))
+        return SNP_E_ALIGN;
+    snp_status st = check_arch();
+    if (st != SNP_OK) return st;
+    cudaError_t e = launch_best(counts, nq, nd, ldo, index_base, best_count, best_index,
+                                (cudaStream_t)stream);
+    return e == cudaSuccess ? SNP_OK : set_cuda_error(e);
+}
+
+snp_status snp_shard_plan(int64_t rows, int world, int64_t align, int64_t *bounds) {
+    if (world < 1 || align < 1 || rows < 0) return SNP_E_RANGE;
+    if (!bounds) return SNP_E_NULL;
+    const int64_t nblocks = (rows + align - 1) / align;
+    const int64_t base = nblocks / world, rem = nblocks % world;
+    int64_t blk = 0;
+    bounds[0] = 0;
+    for (int r = 0; r < world; ++r) {
+        blk += base + (r < rem ? 1 : 0);
+        const int64_t b = blk * align;
+        bounds[r + 1] = b < rows ? b : rows;
+    }
+    return SNP_OK;
+}
+
+snp_status snp_set_variant(int variant) {
+    if (variant < SNP_VARIANT_AUTO || variant > SNP_VARIANT_TC) return SNP_E_OP;
+    current_variant();
+    g_variant.store(variant);
+    return SNP_OK;
+}
+
+int snp_last_variant(void) { return g_last_variant; }
+
+int64_t snp_launch_count(void) { return (int64_t)g_launches.load(); }
+
+const char *snp_status_string(int status) {
+    switch (status) {
+    case SNP_OK: return "SNP_OK";
+    case SNP_E_NULL: return "SNP_E_NULL: a required pointer is NULL";
+    case SNP_E_SHAPE: return "SNP_E_SHAPE: invalid size or leading dimension";
+    case SNP_E_ALIGN: return "SNP_E_ALIGN: pointer not 16-byte aligned or odd packed leading dimension";
+    case SNP_E_OP: return "SNP_E_OP: unknown op or variant";
+    case SNP_E_RANGE: return "SNP_E_RANGE: value out of supported range";
+    case SNP_E_WORKSPACE: return "SNP_E_WORKSPACE: workspace too small";
+    case SNP_E_ARCH: return "SNP_E_ARCH: current device is not a compute capability 10.0 (B200) GPU";
+    case SNP_E_CUDA: return "SNP_E_CUDA: CUDA error (see snp_last_cuda_error)";
+    default: return "unknown snp_status";
+    }
+}
+
+const char *snp_last_cuda_error(void) { return g_cuda_err; }
+
+}  // extern "C"

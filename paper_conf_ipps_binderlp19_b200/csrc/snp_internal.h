@@ -1,0 +1,54 @@
+// snp_internal.h — launcher declarations shared by the library's translation units.
+// Not part of the public ABI (that is include/snp.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace snp {
+
+// Process-wide count of kernels this library launched (snp_launch_count()).
+void count_launches(int k);
+
+// Epilogue kinds of the bit-GEMM.
+enum Epi : int {
+    EPI_COUNTS = 0,   // C = / += counts                       (a3, a4 direct ops)
+    EPI_LD = 1        // r2 [, D'] [, counts] from nAB, nA, nB  (a5)
+};
+
+struct GemmArgs {
+    const uint32_t *A;   // [m][lda32] packed rows viewed as uint32 words
+    const uint32_t *B;   // [n][ldb32]
+    int64_t m, n;
+    int64_t lda32, ldb32;
+    int64_t nbits;
+    int op;              // snp_op
+    int accumulate;
+    int64_t ldc;
+    uint32_t *C;         // counts (EPI_COUNTS: required; EPI_LD: optional)
+    float *r2;           // EPI_LD
+    float *dprime;       // EPI_LD optional
+    const uint32_t *popA;  // EPI_LD (and tensor identities)
+    const uint32_t *popB;
+};
+
+// CUDA-core LOP3 + POPC variant (bitgemm_popc.cu).
+cudaError_t launch_bitgemm_popc(const GemmArgs &a, int epi, cudaStream_t s);
+
+// pack.cu
+cudaError_t launch_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg,
+                        uint64_t *packed, int64_t ldw, cudaStream_t s);
+cudaError_t launch_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int64_t ldw,
+                            uint32_t *popc, cudaStream_t s);
+
+// best.cu — scratch is best_index reinterpreted as packed (count<<32 | j) keys.
+cudaError_t launch_best(const uint32_t *counts, int64_t nq, int64_t nd, int64_t ldo,
+                        int64_t index_base, uint32_t *best_count, int64_t *best_index,
+                        cudaStream_t s);
+
+// Tensor-core tcgen05 variant (bitgemm_tc.cu).  ws: expanded operands.
+size_t tc_workspace_bytes(int64_t m, int64_t n, int64_t nbits);
+bool tc_supported(int64_t m, int64_t n, int64_t nbits);
+cudaError_t launch_bitgemm_tc(const GemmArgs &a, int epi, void *ws, size_t ws_bytes,
+                              cudaStream_t s);
+
+}  // namespace snp

@@ -25,3 +25,13 @@ def pytest_collection_modifyitems(config, items):
     for item in items:
         if "gpu" in item.keywords:
             item.add_marker(skip)
+
+
+@pytest.fixture(scope="session")
+def snplib():
+    """The product binding with libsnp.so built (in-tree) if missing or stale."""
+    from paper_conf_ipps_binderlp19_b200.build import build_library
+    build_library()
+    import paper_conf_ipps_binderlp19_b200 as snp
+    snp.lib()
+    return snp

@@ -1,0 +1,140 @@
+"""Boundary tests that need no GPU: the C-ABI library loads, exports every symbol
+include/snp.h declares, and validates arguments synchronously (before touching
+CUDA).  Host-only logic (snp_words, snp_shard_plan) is checked here too."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "snp.h")
+
+OK, E_NULL, E_SHAPE, E_ALIGN, E_OP, E_RANGE, E_WORKSPACE, E_ARCH, E_CUDA = range(9)
+
+
+def declared_symbols():
+    text = open(HEADER).read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    return sorted(set(re.findall(r"\b(snp_[a-z0-9_]+)\s*\(", text)))
+
+
+def test_header_declares_expected_calls():
+    syms = declared_symbols()
+    for name in ("snp_pack", "snp_row_popc", "snp_ld_counts", "snp_ld_r2", "snp_fastid",
+                 "snp_fastid_best", "snp_shard_plan", "snp_words", "snp_status_string"):
+        assert name in syms
+
+
+def test_library_exports_every_declared_symbol(snplib):
+    L = snplib.lib()
+    from paper_conf_ipps_binderlp19_b200._lib import SIGNATURES
+    for name in declared_symbols():
+        assert hasattr(L, name), name
+        assert name in SIGNATURES, f"binding lacks {name}"
+    # and the binding exposes a Python function of the same name for each call
+    for name in declared_symbols():
+        if name in ("snp_status_string", "snp_last_cuda_error"):
+            continue
+        assert hasattr(snplib, name), name
+
+
+def test_library_is_sm100a_only(snplib):
+    import subprocess
+    from paper_conf_ipps_binderlp19_b200._lib import LIB_PATH
+    out = subprocess.run(["cuobjdump", "--list-elf", LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    assert "sm_90" not in out and "sm_80" not in out
+
+
+def test_snp_words():
+    from paper_conf_ipps_binderlp19_b200 import snp_words
+    assert snp_words(0) == 0 and snp_words(-5) == 0
+    assert snp_words(1) == 8 and snp_words(512) == 8 and snp_words(513) == 16
+    assert snp_words(4096) == 64 and snp_words(16384) == 256
+
+
+@pytest.mark.parametrize("rows,world,align", [(0, 1, 128), (1, 1, 128), (1000, 3, 128),
+                                              (32768, 8, 128), (20_000_000, 8, 128),
+                                              (129, 2, 128), (5, 8, 1), (7, 8, 2)])
+def test_shard_plan_properties(snplib, rows, world, align):
+    b = snplib.snp_shard_plan(rows, world, align)
+    assert len(b) == world + 1 and b[0] == 0 and b[-1] == rows
+    assert all(b[r] <= b[r + 1] for r in range(world))               # contiguous, disjoint
+    assert all(x % align == 0 or x == rows for x in b)                # aligned (or the end)
+    blocks = [(b[r + 1] - b[r] + align - 1) // align for r in range(world)]
+    assert max(blocks) - min(blocks) <= 1 or rows < align * world    # balanced
+    assert sum(b[r + 1] - b[r] for r in range(world)) == rows         # covers
+    assert b == snplib.snp_shard_plan(rows, world, align)             # deterministic
+
+
+def test_shard_plan_bad_args(snplib):
+    L = snplib.lib()
+    arr = (ctypes.c_int64 * 4)()
+    p = ctypes.cast(arr, ctypes.c_void_p)
+    assert L.snp_shard_plan(10, 0, 128, p) == E_RANGE
+    assert L.snp_shard_plan(10, 2, 0, p) == E_RANGE
+    assert L.snp_shard_plan(-1, 2, 128, p) == E_RANGE
+    assert L.snp_shard_plan(10, 2, 128, None) == E_NULL
+
+
+def test_status_strings(snplib):
+    L = snplib.lib()
+    for s in range(9):
+        assert L.snp_status_string(s).decode().startswith("SNP_")
+    assert b"unknown" in L.snp_status_string(99)
+
+
+FAKE = 0x10000  # a 16-byte aligned non-NULL address: never dereferenced (validation fails first)
+
+
+def test_validation_errors_before_launch(snplib):
+    L = snplib.lib()
+    p = ctypes.c_void_p(FAKE)
+    odd = ctypes.c_void_p(FAKE + 8)
+    null = None
+    # snp_ld_counts(A, m, lda, B, n, ldb, nbits, C, ldc, acc, ws, ws_bytes, stream)
+    assert L.snp_ld_counts(null, 4, 2, p, 4, 2, 100, p, 4, 0, null, 0, null) == E_NULL
+    assert L.snp_ld_counts(p, -1, 2, p, 4, 2, 100, p, 4, 0, null, 0, null) == E_SHAPE
+    assert L.snp_ld_counts(p, 4, 1, p, 4, 2, 100, p, 4, 0, null, 0, null) == E_SHAPE   # lda < words
+    assert L.snp_ld_counts(p, 4, 3, p, 4, 2, 100, p, 4, 0, null, 0, null) == E_ALIGN   # odd ld
+    assert L.snp_ld_counts(odd, 4, 2, p, 4, 2, 100, p, 4, 0, null, 0, null) == E_ALIGN
+    assert L.snp_ld_counts(p, 4, 2, p, 4, 2, 0, p, 4, 0, null, 0, null) == E_SHAPE     # nbits < 1
+    assert L.snp_ld_counts(p, 4, 2, p, 4, 2, 100, p, 3, 0, null, 0, null) == E_SHAPE   # ldc < n
+    assert L.snp_ld_counts(p, 4, 2, p, 4, 2, 100, null, 4, 0, null, 0, null) == E_NULL
+    assert L.snp_ld_counts(p, 4, 2, p, 4, 2, 1 << 33, p, 4, 0, null, 0, null) == E_RANGE
+    # zero-sized problems are valid no-ops
+    assert L.snp_ld_counts(p, 0, 2, p, 4, 2, 100, null, 4, 0, null, 0, null) == OK
+    assert L.snp_fastid(p, 4, 2, null, p, 0, 2, null, 100, 1, null, 0, 0, null, 0, null) == OK
+    # bad op
+    assert L.snp_fastid(p, 4, 2, null, p, 4, 2, null, 100, 7, p, 4, 0, null, 0, null) == E_OP
+    # r2 requires the workspace returned by the query
+    assert L.snp_ld_r2(p, 4, 2, null, p, 4, 2, null, 100, p, null, null, 4, null, 0, null) == E_WORKSPACE
+    # pack validation
+    assert L.snp_pack(null, 3, 100, 100, p, 2, null) == E_NULL
+    assert L.snp_pack(p, 3, 100, 99, p, 2, null) == E_SHAPE
+    assert L.snp_pack(p, 3, 100, 100, p, 1, null) == E_SHAPE
+    assert L.snp_pack(p, 3, 100, 100, odd, 2, null) == E_ALIGN
+    # best
+    assert L.snp_fastid_best(p, 2, 10, 5, 0, p, p, null) == E_SHAPE
+    assert L.snp_set_variant(9) == E_OP
+
+
+def test_valid_call_without_b200_is_refused(snplib):
+    """No fallback: on a host without a compute-capability-10.0 GPU a valid call
+    returns SNP_E_ARCH (this CPU box has no GPU at all)."""
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    L = snplib.lib()
+    p = ctypes.c_void_p(FAKE)
+    ws = snplib.snp_ld_workspace_bytes(4, 4, 100)
+    assert L.snp_ld_counts(p, 4, 2, p, 4, 2, 100, p, 4, 0, p, ws, None) == E_ARCH
+    with pytest.raises(snplib.SnpError):
+        snplib._lib.check(E_ARCH, "x")
+
+
+def test_workspace_queries(snplib):
+    assert snplib.snp_ld_workspace_bytes(0, 5, 100) == 0
+    assert snplib.snp_ld_workspace_bytes(300, 500, 100) >= 4 * 800
+    assert snplib.snp_fastid_workspace_bytes(0, 5, 100) == 0

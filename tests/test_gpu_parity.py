@@ -1,0 +1,290 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
+
+Integer outputs must be bit-exact; r2 / D' within 1e-6 relative of the fp64 oracle
+and exactly 0 where the oracle is 0 (BASELINE.json north_star).  Inputs come from
+snpgen (seeded); the oracle always sees the generator's unpacked bytes, never
+anything the CUDA path produced.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import snpgen
+
+pytestmark = pytest.mark.gpu
+
+DEV = "cuda"
+VARIANTS = ["popc", "tc"]
+
+
+@pytest.fixture(scope="module")
+def snp(snplib):
+    torch.cuda.set_device(0)
+    yield snplib
+    snplib.snp_set_variant("auto")
+
+
+def _variant(snp, v):
+    snp.snp_set_variant(v)
+
+
+def to_dev(g):
+    return torch.from_numpy(np.ascontiguousarray(g)).to(DEV)
+
+
+def pack_dev(snp, g, ldw=None, garbage_seed=None):
+    """snp_pack on device; optionally fill every padding bit with garbage."""
+    nbits = g.shape[1]
+    P = snp.snp_pack(to_dev(g), nbits=nbits, ldw=ldw)
+    if garbage_seed is not None:
+        rng = np.random.default_rng(garbage_seed)
+        junk = torch.from_numpy(rng.integers(0, 2**63, size=tuple(P.shape), dtype=np.int64)).to(DEV)
+        words = (nbits + 63) // 64
+        pv = P.view(torch.int64)
+        tail = nbits % 64
+        if tail:
+            keep = (1 << tail) - 1
+            pv[:, words - 1] = (pv[:, words - 1] & keep) | (junk[:, words - 1] & ~keep)
+        pv[:, words:] = junk[:, words:]
+    return P
+
+
+def u32(t):
+    return t.cpu().numpy().astype(np.uint32)
+
+
+# ------------------------------------------------------------------ a1 / a2
+
+@pytest.mark.parametrize("nbits", [1, 63, 64, 65, 127, 129, 1000, 4095, 4097])
+def test_pack_bit_exact(snp, nbits):
+    rng = np.random.default_rng(nbits)
+    g = (rng.random((37, nbits)) < 0.4).astype(np.uint8) * snpgen.random_bytes_nonzero((37, nbits), 1)
+    ldw = snp.snp_words(nbits) + 2
+    P = snp.snp_pack(to_dev(g), ldw=ldw)
+    torch.cuda.synchronize()
+    assert np.array_equal(P.cpu().numpy(), oracle.pack(g, ldw))
+
+
+def test_pack_unaligned_rows(snp):
+    rng = np.random.default_rng(5)
+    nbits = 300
+    big = (rng.random((20, nbits + 7)) < 0.5).astype(np.uint8)
+    gd = to_dev(big)[:, 3:3 + nbits]          # odd offset and ldg = nbits + 7
+    P = snp.snp_pack(gd, nbits=nbits)
+    assert np.array_equal(P.cpu().numpy(), oracle.pack(big[:, 3:3 + nbits], snp.snp_words(nbits)))
+
+
+@pytest.mark.parametrize("nbits", [1, 64, 65, 1000, 4097])
+def test_row_popc_ignores_padding(snp, nbits):
+    g = snpgen.fastid_db(7, np.arange(300), nbits)
+    P = pack_dev(snp, g, garbage_seed=nbits)
+    pc = snp.snp_row_popc(P, nbits)
+    assert np.array_equal(u32(pc), oracle.row_popc(g))
+
+
+# ------------------------------------------------------------------ a3 / a4 counts
+
+SHAPES = [(1, 1, 1), (3, 700, 129), (64, 1000, 4096), (70, 513, 1000), (130, 300, 777),
+          (257, 129, 2049)]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("nq,nd,nbits", SHAPES)
+def test_fastid_all_ops(snp, variant, nq, nd, nbits):
+    db = snpgen.fastid_db(11, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(11, nq, nd, nbits)
+    D = pack_dev(snp, db, garbage_seed=1)
+    Q = pack_dev(snp, q, garbage_seed=2)
+    _variant(snp, variant)
+    for op in ("and", "xor", "andnot", "notand"):
+        try:
+            out = snp.snp_fastid(Q, D, nbits, op)
+        except snp.SnpError as e:
+            if variant == "tc" and e.status == 2:
+                pytest.skip("tc variant does not support this shape")
+            raise
+        assert np.array_equal(u32(out), oracle.counts(q, db, op)), (op, variant)
+    _variant(snp, "auto")
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_ld_counts_accumulate_and_selfld(snp, variant):
+    nbits = 1500
+    g = snpgen.ld_genotypes(21, np.arange(260), nbits, structure=True)
+    _variant(snp, variant)
+    try:
+        A = pack_dev(snp, g, garbage_seed=3)
+        C = snp.snp_ld_counts(A, A, nbits)              # self-LD, B aliases A
+        ref = oracle.counts(g, g, "and")
+        assert np.array_equal(u32(C), ref)
+        # K split into two chunks with accumulate (paper's gamma += form)
+        k1 = 640
+        A1 = pack_dev(snp, g[:, :k1])
+        A2 = pack_dev(snp, g[:, k1:])
+        C2 = snp.snp_ld_counts(A1, A1, k1)
+        snp.snp_ld_counts(A2, A2, nbits - k1, C=C2, accumulate=True)
+        assert np.array_equal(u32(C2), ref)
+    except snp.SnpError as e:
+        if variant == "tc" and e.status == 2:
+            pytest.skip("tc variant does not support this shape")
+        raise
+    finally:
+        _variant(snp, "auto")
+
+
+def test_leading_dimensions(snp):
+    """ld > words for A, B and C (ldc > n) — only the first n columns are written."""
+    nbits = 200
+    ga = snpgen.fastid_db(31, np.arange(50), nbits)
+    gb = snpgen.fastid_db(32, np.arange(90), nbits)
+    A = pack_dev(snp, ga, ldw=12, garbage_seed=4)
+    B = pack_dev(snp, gb, ldw=6, garbage_seed=5)
+    Cbig = torch.full((50, 100), 0xDEAD, dtype=torch.int32, device=DEV).view(torch.uint32)
+    snp.snp_fastid(A, B, nbits, "xor", out=Cbig[:, :90])
+    c = u32(Cbig)
+    assert np.array_equal(c[:, :90], oracle.counts(ga, gb, "xor"))
+    assert (c[:, 90:] == 0xDEAD).all()
+
+
+# ------------------------------------------------------------------ a5 LD r2 / D'
+
+def check_r2(got, ref):
+    got = got.astype(np.float64)
+    zero = ref == 0
+    assert (got[zero] == 0).all(), "must be exactly 0 where the oracle is 0"
+    rel = np.abs(got[~zero] - ref[~zero]) / np.abs(ref[~zero])
+    assert rel.size == 0 or rel.max() <= 1e-6, rel.max()
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("m,n,nbits", [(200, 200, 300), (130, 257, 4096), (1, 5, 7), (300, 129, 1025)])
+def test_ld_r2_dprime(snp, variant, m, n, nbits):
+    ga = snpgen.ld_genotypes(41, np.arange(m), nbits, structure=True)
+    gb = snpgen.ld_genotypes(41, np.arange(n) + 50, nbits, structure=True)
+    A = pack_dev(snp, ga, garbage_seed=6)
+    B = pack_dev(snp, gb, garbage_seed=7)
+    _variant(snp, variant)
+    try:
+        r2, dp, cnt = snp.snp_ld_r2(A, B, nbits, dprime=True, counts=True)
+    except snp.SnpError as e:
+        if variant == "tc" and e.status == 2:
+            pytest.skip("tc variant does not support this shape")
+        raise
+    finally:
+        _variant(snp, "auto")
+    r2_ref, dp_ref, n_ref = oracle.ld(ga, gb)
+    assert np.array_equal(u32(cnt), n_ref)
+    check_r2(r2.cpu().numpy(), r2_ref)
+    check_r2(dp.cpu().numpy(), dp_ref)
+
+
+def test_ld_r2_with_given_popcounts(snp):
+    nbits = 513
+    g = snpgen.ld_genotypes(43, np.arange(150), nbits, structure=True)
+    A = pack_dev(snp, g)
+    pa = snp.snp_row_popc(A, nbits)
+    r2, _, _ = snp.snp_ld_r2(A, A, nbits, popA=pa, popB=pa)
+    check_r2(r2.cpu().numpy(), oracle.ld(g, g)[0])
+
+
+# ------------------------------------------------------------------ a6 best
+
+def test_best_ties_and_base(snp):
+    rng = np.random.default_rng(8)
+    c = rng.integers(0, 4, size=(33, 20001)).astype(np.uint32)
+    ct = torch.from_numpy(c.view(np.int32)).to(DEV).view(torch.uint32)
+    b, i = snp.snp_fastid_best(ct, index_base=123456789)
+    rb, ri = oracle.best(c, 123456789)
+    assert np.array_equal(u32(b), rb) and np.array_equal(i.cpu().numpy(), ri)
+    # unaligned row starts (ldo odd) and nd = 0
+    sub = ct[:, 1:]
+    b, i = snp.snp_fastid_best(sub)
+    rb, ri = oracle.best(c[:, 1:])
+    assert np.array_equal(u32(b), rb) and np.array_equal(i.cpu().numpy(), ri)
+    b, i = snp.snp_fastid_best(ct[:, :0])
+    assert (i.cpu().numpy() == -1).all() and (u32(b) == 0xFFFFFFFF).all()
+
+
+# ------------------------------------------------------------------ BASELINE configs
+
+def _gen_dev_fastid(seed, nd, nbits, chunk=65536):
+    """Full DB generated on device in row chunks and packed by snp_pack."""
+    import paper_conf_ipps_binderlp19_b200 as snp
+    D = torch.empty((nd, snp.snp_words(nbits)), dtype=torch.uint64, device=DEV)
+    for r0 in range(0, nd, chunk):
+        r1 = min(nd, r0 + chunk)
+        g = snpgen.fastid_db(seed, torch.arange(r0, r1, device=DEV), nbits, xp="torch", device=DEV)
+        snp.snp_pack(g, out=D[r0:r1])
+    return D
+
+
+def _sample_cols(n, tile, k, seed):
+    rng = np.random.default_rng(seed)
+    s = set(rng.integers(0, n, size=k).tolist())
+    for b in range(tile, n, tile * 97):
+        s.update([b - 1, b, b + 1])
+    s.update([0, 1, n - 2, n - 1])
+    return np.array(sorted(x for x in s if 0 <= x < n))
+
+
+@pytest.mark.parametrize("variant", ["auto", "popc"])
+def test_cfg2_fastid_1m_sampled(snp, variant):
+    """configs[1]: 64 queries x 1,000,000 profiles x 4,096 SNPs, XOR and ANDNOT,
+    the launch configuration bench.py times; sampled DB rows vs the oracle, planted
+    matches found, best == numpy min/argmin of the produced counts."""
+    nq, nd, nbits, seed = 64, 1_000_000, 4096, 1002
+    D = _gen_dev_fastid(seed, nd, nbits)
+    q, plan = snpgen.fastid_queries(seed, nq, nd, nbits)
+    Q = snp.snp_pack(to_dev(q))
+    cols = _sample_cols(nd, 128, 600, 9)
+    dbs = snpgen.fastid_db(seed, cols, nbits)
+    _variant(snp, variant)
+    try:
+        for op in ("xor", "andnot"):
+            out = snp.snp_fastid(Q, D, nbits, op)
+            got = u32(out[:, torch.from_numpy(cols).to(DEV)])
+            assert np.array_equal(got, oracle.counts(q, dbs, op)), op
+            if op == "xor":
+                b, i = snp.snp_fastid_best(out)
+                full = out.cpu().numpy().astype(np.uint32)
+                assert np.array_equal(u32(b), full.min(1))
+                assert np.array_equal(i.cpu().numpy(), full.argmin(1))
+                for qi, (kind, js, flips) in enumerate(plan):
+                    if kind == "copy":
+                        assert full[qi, js[0]] == len(flips) and u32(b)[qi] <= len(flips)
+            del out
+    finally:
+        _variant(snp, "auto")
+
+
+def test_cfg1_ld_full(snp):
+    """configs[0]: LD 2,048 SNPs x 4,096 samples, counts + r2 + D', full oracle."""
+    m, nbits = 2048, 4096
+    g = snpgen.ld_genotypes(1001, np.arange(m), nbits, structure=True)
+    A = snp.snp_pack(to_dev(g))
+    r2, dp, cnt = snp.snp_ld_r2(A, A, nbits, dprime=True, counts=True)
+    r2_ref, dp_ref, n_ref = oracle.ld(g, g)
+    assert np.array_equal(u32(cnt), n_ref)
+    check_r2(r2.cpu().numpy(), r2_ref)
+    check_r2(dp.cpu().numpy(), dp_ref)
+
+
+def test_cfg3_ld_32k_sampled_rows(snp):
+    """configs[2]: LD 32,768 x 32,768 SNPs x 16,384 samples (counts + r2); sampled
+    rows including tile boundaries vs the oracle over all columns."""
+    m, nbits, seed = 32768, 16384, 1003
+    A = torch.empty((m, snp.snp_words(nbits)), dtype=torch.uint64, device=DEV)
+    for r0 in range(0, m, 4096):
+        gg = snpgen.ld_genotypes(seed, torch.arange(r0, r0 + 4096, device=DEV), nbits,
+                                 structure=True, xp="torch", device=DEV)
+        snp.snp_pack(gg, out=A[r0:r0 + 4096])
+    r2, _, cnt = snp.snp_ld_r2(A, A, nbits, counts=True)
+    rows = np.array([0, 1, 127, 128, 4095, 4096, 20000, m - 1])
+    ga = snpgen.ld_genotypes(seed, rows, nbits, structure=True)
+    gall = np.concatenate([snpgen.ld_genotypes(seed, np.arange(r0, r0 + 1024), nbits, structure=True)
+                           for r0 in range(0, m, 1024)])
+    r2_ref, _, n_ref = oracle.ld(ga, gall)
+    ridx = torch.from_numpy(rows).to(DEV)
+    assert np.array_equal(u32(cnt[ridx]), n_ref)
+    check_r2(r2[ridx].cpu().numpy(), r2_ref)
