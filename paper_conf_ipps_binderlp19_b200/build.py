@@ -47,14 +47,33 @@ def nvcc() -> str:
 
 
 def build_library(force: bool = False, verbose: bool = False) -> str:
-    """Compile csrc/*.cu into libsnp.so if missing/stale (or force)."""
+    """Compile csrc/*.cu (in parallel) and link libsnp.so if missing/stale (or force)."""
     if not force and not stale():
         return LIB
+    import concurrent.futures as cf
+    import tempfile
+    objdir = tempfile.mkdtemp(prefix="snp_build_")
+    compile_flags = [f for f in NVCC_FLAGS if f != "-shared"]
+    jobs = []
+    for src in sources():
+        obj = os.path.join(objdir, os.path.basename(src) + ".o")
+        jobs.append((obj, [nvcc(), *compile_flags, "-c", src, "-o", obj]))
+    with cf.ThreadPoolExecutor(max_workers=min(8, len(jobs))) as ex:
+        futs = [ex.submit(subprocess.run, cmd, capture_output=True, text=True) for _, cmd in jobs]
+        for (obj, cmd), f in zip(jobs, futs):
+            r = f.result()
+            if verbose:
+                print(" ".join(cmd))
+            if r.stdout or r.stderr:
+                print(r.stdout + r.stderr)
+            if r.returncode != 0:
+                raise subprocess.CalledProcessError(r.returncode, cmd)
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [nvcc(), *NVCC_FLAGS, "-o", tmp, *sources()]
+    link = [nvcc(), "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-cudart", "static",
+            "-o", tmp, *[o for o, _ in jobs]]
     if verbose:
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
+        print(" ".join(link))
+    subprocess.check_call(link)
     os.replace(tmp, LIB)
     return LIB
 
