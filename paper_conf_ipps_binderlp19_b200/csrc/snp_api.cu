@@ -103,7 +103,14 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
     cudaError_t e;
     if (variant == SNP_VARIANT_TC) {
         if (!tc_supported(a.m, a.n, a.nbits)) return SNP_E_SHAPE;
-        e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
+        // kind::mxf4 (2x the int8 rate, half the expanded bytes) unless K is too long
+        // for exact fp32 accumulation or SNP_TC_KIND=i8 asks for the int8 kernel.
+        const char *kind = std::getenv("SNP_TC_KIND");
+        const bool want_i8 = kind && !std::strcmp(kind, "i8");
+        if (!want_i8 && tc4_supported(a.m, a.n, a.nbits))
+            e = launch_bitgemm_tc4(a, epi, s);
+        else
+            e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
     } else {
         e = launch_bitgemm_popc(a, epi, s);
     }
