@@ -1,0 +1,76 @@
+"""Multi-GPU driver for the SNP-comparison path — one process per GPU.
+
+The path shards with ONE exchange step and no collective inside the hot loop:
+
+* FastID: database rows are sharded (``snp_shard_plan``, 128-row aligned);
+  the packed query batch is broadcast from rank 0 (NCCL over NVLink/NVSwitch),
+  every rank computes its ``out[nq][nd_r]`` and its per-query best match with
+  ``index_base = b_r``; the (count, index) pairs are all-gathered and merged with
+  the lowest-global-index tie-break (reading R4).
+* LD: output row blocks are sharded; the packed matrix is broadcast from rank 0
+  and rank r computes rows ``[b_r, b_{r+1})`` against all columns.
+
+The compute callables default to the CUDA library; tests inject oracle-backed
+callables to exercise the same exchange logic with the gloo backend on CPU.
+The merge is plain tensor plumbing over ``world x nq`` values.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+
+def shard_bounds(rows: int, world: int, align: int = 128) -> list[int]:
+    from . import snp_shard_plan
+    return snp_shard_plan(rows, world, align)
+
+
+def merge_best(gc: torch.Tensor, gi: torch.Tensor):
+    """gc, gi: [world, nq] per-rank (best count, best global index) -> global best.
+
+    Shards are contiguous and ordered by rank, so among equal counts the lowest
+    rank holds the lowest global index; a rank with no rows reports index -1 and
+    count 0xFFFFFFFF and never wins unless every rank is empty."""
+    c = gc.to(torch.int64) & 0xFFFFFFFF
+    idx = gi.to(torch.int64)
+    c = torch.where(idx < 0, torch.full_like(c, 1 << 33), c)
+    m = c.min(dim=0).values
+    first = (c == m).to(torch.int32).argmax(dim=0)        # argmax returns the first maximum
+    cols = torch.arange(c.shape[1], device=c.device)
+    best_idx = idx[first, cols]
+    best_cnt = torch.where(m >= (1 << 33), torch.full_like(m, 0xFFFFFFFF), m)
+    return best_cnt, best_idx
+
+
+def fastid_step(Q: torch.Tensor, D_shard: torch.Tensor, nbits: int, op: str, index_base: int,
+                out: torch.Tensor | None = None, compute=None, best=None, group=None):
+    """One sharded FastID step.  Q must be allocated on every rank (its content on
+    rank 0 is broadcast).  Returns (local counts, global best count, global best index)."""
+    from . import snp_fastid, snp_fastid_best
+    compute = compute or (lambda Q_, D_, o_: snp_fastid(Q_, D_, nbits, op, out=o_))
+    best = best or (lambda c_, base_: snp_fastid_best(c_, index_base=base_))
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    if world > 1:
+        dist.broadcast(Q, src=0, group=group)
+    counts = compute(Q, D_shard, out)
+    bc, bi = best(counts, index_base)
+    if world == 1:
+        return counts, bc.to(torch.int64), bi
+    nq = bc.numel()
+    bc = bc.view(torch.int32) if bc.dtype == torch.uint32 else bc
+    gc = torch.empty(world * nq, dtype=bc.dtype, device=bc.device)
+    gi = torch.empty(world * nq, dtype=bi.dtype, device=bi.device)
+    dist.all_gather_into_tensor(gc, bc.contiguous(), group=group)
+    dist.all_gather_into_tensor(gi, bi.contiguous(), group=group)
+    c, i = merge_best(gc.view(world, nq).to(torch.int64), gi.view(world, nq))
+    return counts, c, i
+
+
+def ld_step(B: torch.Tensor, nbits: int, lo: int, hi: int, compute=None, group=None):
+    """One sharded LD step: broadcast the packed matrix from rank 0, compute rows [lo, hi)."""
+    from . import snp_ld_r2
+    compute = compute or (lambda A_, B_: snp_ld_r2(A_, B_, nbits, counts=True))
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    if world > 1:
+        dist.broadcast(B, src=0, group=group)
+    return compute(B[lo:hi], B)

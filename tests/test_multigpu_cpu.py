@@ -1,0 +1,115 @@
+"""World-size-2 gloo tests (CPU) of the multi-GPU exchange logic.
+
+The compute steps are oracle-backed here (no GPU); what is under test is the
+sharding (snp_shard_plan via the C ABI, host-only), the query / matrix broadcast,
+the all-gather of per-shard best matches and the lowest-global-index merge.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import snpgen
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, q):
+    try:
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        from paper_conf_ipps_binderlp19_b200 import multigpu
+
+        # ---------------- FastID: DB sharded, queries broadcast, best gathered
+        nd, nbits, nq = 700, 300, 9
+        db = snpgen.fastid_db(77, np.arange(nd), nbits)
+        # plant ties across the shard boundary: rows 100 and 600 identical
+        db[600] = db[100]
+        b = multigpu.shard_bounds(nd, world, 128)
+        lo, hi = b[rank], b[rank + 1]
+        Dsh = torch.from_numpy(oracle.pack(db[lo:hi], 6).view(np.int64))
+        if rank == 0:
+            qg, _ = snpgen.fastid_queries(77, nq, nd, nbits)
+            qg[0] = db[100]
+            Q = torch.from_numpy(oracle.pack(qg, 6).view(np.int64))
+        else:
+            Q = torch.zeros((nq, 6), dtype=torch.int64)
+
+        def compute(Q_, D_, out_):
+            qq = oracle.unpack(Q_.numpy().view(np.uint64), nbits)
+            dd = oracle.unpack(D_.numpy().view(np.uint64), nbits)
+            return torch.from_numpy(oracle.counts(qq, dd, "xor").astype(np.int64))
+
+        def best(c_, base_):
+            bc, bi = oracle.best(c_.numpy().astype(np.uint32), base_)
+            return torch.from_numpy(bc.astype(np.int64)), torch.from_numpy(bi)
+
+        counts, bc, bi = multigpu.fastid_step(Q, Dsh, nbits, "xor", lo, compute=compute, best=best)
+        qfull = oracle.unpack(Q.numpy().view(np.uint64), nbits)
+        ref_c, ref_i = oracle.best(oracle.counts(qfull, db, "xor"))
+        ok_fastid = bool(np.array_equal(bc.numpy(), ref_c.astype(np.int64)) and np.array_equal(bi.numpy(), ref_i))
+        ok_tie = int(bi[0]) == 100 and int(bc[0]) == 0
+        ok_local = bool(np.array_equal(counts.numpy(), oracle.counts(qfull, db[lo:hi], "xor")))
+
+        # ---------------- LD: packed matrix broadcast, row blocks sharded
+        m, nb2 = 300, 130
+        g = snpgen.ld_genotypes(78, np.arange(m), nb2, structure=True)
+        bb = multigpu.shard_bounds(m, world, 128)
+        B = torch.from_numpy(oracle.pack(g, 4).view(np.int64)) if rank == 0 else torch.zeros((m, 4), dtype=torch.int64)
+
+        def ld_compute(A_, B_):
+            aa = oracle.unpack(A_.numpy().view(np.uint64), nb2)
+            bbm = oracle.unpack(B_.numpy().view(np.uint64), nb2)
+            return oracle.ld(aa, bbm)
+
+        r2, dp, nab = multigpu.ld_step(B, nb2, bb[rank], bb[rank + 1], compute=ld_compute)
+        r2_ref, _, _ = oracle.ld(g, g)
+        ok_ld = bool(np.array_equal(r2, r2_ref[bb[rank]:bb[rank + 1]]))
+        q.put((rank, ok_fastid, ok_tie, ok_local, ok_ld, (lo, hi)))
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover
+        import traceback
+        q.put((rank, "error", traceback.format_exc()))
+
+
+def test_two_rank_gloo_fastid_and_ld():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for r in res:
+        assert r[1] != "error", r[2]
+        rank, ok_fastid, ok_tie, ok_local, ok_ld, rng = r
+        assert ok_fastid, f"rank {rank}: merged best != oracle"
+        assert ok_tie, f"rank {rank}: tie across shards must go to the lowest global index"
+        assert ok_local, f"rank {rank}: local counts wrong for rows {rng}"
+        assert ok_ld, f"rank {rank}: LD row block wrong"
+
+
+def test_merge_best_edge_cases():
+    from paper_conf_ipps_binderlp19_b200.multigpu import merge_best
+    gc = torch.tensor([[5, 3, 0xFFFFFFFF], [3, 3, 7]], dtype=torch.int64)
+    gi = torch.tensor([[10, 11, -1], [200, 201, 202]], dtype=torch.int64)
+    c, i = merge_best(gc, gi)
+    assert c.tolist() == [3, 3, 7]
+    assert i.tolist() == [200, 11, 202]
+    c, i = merge_best(torch.tensor([[0xFFFFFFFF]]), torch.tensor([[-1]]))
+    assert c.tolist() == [0xFFFFFFFF] and i.tolist() == [-1]
