@@ -1,0 +1,408 @@
+// fastid_tc4.cu — FastID-shaped tensor-core bit-GEMM: a small query batch (<= 128
+// profiles) against a huge database streamed from HBM.
+//
+//   out[q][d] = sum_k op(Q_qk, D_dk),  op in {AND, XOR, ANDNOT, NOTAND}  (Eqs. 1-3,
+//   P:L52-78), via the AND count and the popcount identities of SURVEY §8a a4.
+//
+// For a few queries the path is bound by streaming the database, so this kernel is
+// built around the database stream:
+//   * the query batch is expanded ONCE per CTA into shared memory (e2m1 nibbles, K-major
+//     no-swizzle UMMA layout, the whole K range) and stays resident — it is the MMA B
+//     operand for every database tile;
+//   * database tiles (128 rows) are streamed by TMA (2-D tensor map, 128 rows x 256 bits
+//     per stage) into a 16-deep shared-memory ring: up to 64 KB in flight per SM without
+//     spending registers;
+//   * 8 expander warps turn each stage into e2m1 nibbles and write them straight into
+//     TMEM (tcgen05.st) as the MMA A operand, accumulating database-row popcounts;
+//   * one thread issues tcgen05.mma kind::mxf4 (M = 128 database rows, N = queries,
+//     K = 64) from TMEM-A x SMEM-B into one of two TMEM accumulators;
+//   * 4 epilogue warps apply the popcount identity and write out[q][d] coalesced along d
+//     while the next tile is being multiplied.
+// Exactness: see bitgemm_tc4.cu (products in {0, 1}, fp32 sums exact below 2^24).
+#include "snp_internal.h"
+#include "tc_ptx.cuh"
+
+#include <cuda.h>
+
+namespace snp {
+namespace {
+
+constexpr int BM = 128;
+constexpr int KBITS = 256;
+constexpr int KSTEPS = KBITS / 64;
+constexpr int NP = 16;                  // packed TMA ring depth
+constexpr int PSTAGE = BM * KBITS / 8;  // 4 KB packed per stage
+constexpr int NEXP = 8;
+constexpr int MMA_WARP = 8;
+constexpr int EPI_WARP0 = 9;
+constexpr int TMA_WARP = 13;
+constexpr int NTHREADS = 14 * 32;
+constexpr size_t MAX_SMEM = 232448;     // 227 KB opt-in
+
+template <int BN>
+struct FCfg {
+    static constexpr int NS = BN <= 64 ? 8 : 6;     // TMEM A stages
+    static constexpr int ACC_COLS = BN;
+    static constexpr int A_COL0 = 2 * ACC_COLS;
+    static constexpr int SF_COL = A_COL0 + NS * 32;
+    static_assert(SF_COL + 32 <= 512, "TMEM budget");
+};
+
+struct FArgs {
+    const uint32_t *Q;   // queries (column side), packed u32 view
+    int64_t nq, ldq32;
+    int64_t nd;          // database rows (lane side)
+    int64_t nbits;
+    int op, accumulate;
+    int64_t ldo;
+    uint32_t *out;
+    int64_t ntiles;
+    int nst;
+    size_t qbytes;       // expanded query bytes in shared memory
+};
+
+__device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
+    const int64_t lo = w * 32;
+    if (lo + 32 <= nbits) return 0xffffffffu;
+    if (lo >= nbits) return 0u;
+    return (1u << (uint32_t)(nbits - lo)) - 1u;
+}
+
+__device__ __forceinline__ void expand4(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
+    const uint32_t M = 0x22222222u;   // e2m1 1.0 = 0b0010 in every nibble where the bit is set
+    o0 = (x << 1) & M;
+    o1 = x & M;
+    o2 = (x >> 1) & M;
+    o3 = (x >> 2) & M;
+}
+
+__host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
+    return (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a_tmem, uint64_t bdesc, uint32_t idesc,
+                                            uint32_t accumulate, uint32_t sfa, uint32_t sfb) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}" ::"r"(d),
+        "r"(a_tmem), "l"(bdesc), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb));
+}
+
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+            taddr),
+        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
+        "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+        : "memory");
+}
+
+template <int BN>
+__global__ void __launch_bounds__(NTHREADS, 1)
+fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
+    using C = FCfg<BN>;
+    constexpr int NS = C::NS;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *qsm = smem;                                            // [nst*8 chunks][BN][16 B]
+    uint8_t *ring = smem + args.qbytes;                             // [NP][PSTAGE]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(ring + NP * PSTAGE);
+    uint64_t *pfull = bars;                  // [NP] TMA -> expanders
+    uint64_t *pempty = pfull + NP;           // [NP] expanders -> TMA
+    uint64_t *full = pempty + NP;            // [NS] expanders -> MMA
+    uint64_t *empty = full + NS;             // [NS] MMA -> expanders
+    uint64_t *accf = empty + NS;             // [2]
+    uint64_t *acce = accf + 2;               // [2]
+    uint64_t *popf = acce + 2;               // [2]
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popf + 2);
+    uint32_t *popQ = tmem_slot + 4;          // [BN]
+    uint32_t *popD = popQ + BN;              // [2 acc][2 half][BM]
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int64_t nbits = args.nbits;
+    const int nst = args.nst;
+    const int64_t my_tiles = args.ntiles > blockIdx.x ? (args.ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const int64_t total_it = my_tiles * nst;
+    const int64_t full32 = nbits / 32;
+
+    if (tid == 0) {
+        for (int i = 0; i < NP; ++i) {
+            ptx::mbar_init(&pfull[i], 1);
+            ptx::mbar_init(&pempty[i], NEXP);
+        }
+        for (int i = 0; i < NS; ++i) {
+            ptx::mbar_init(&full[i], NEXP);
+            ptx::mbar_init(&empty[i], 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            ptx::mbar_init(&accf[i], 1);
+            ptx::mbar_init(&acce[i], 4);
+            ptx::mbar_init(&popf[i], NEXP);
+        }
+        ptx::fence_mbar_init();
+    }
+    if (warp == TMA_WARP && lane == 0) ptx::prefetch_tensormap(&tmD);
+    for (int r = tid; r < BN; r += NTHREADS) popQ[r] = 0;
+    if (warp == MMA_WARP) ptx::tmem_alloc<512>(tmem_slot);
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    // ---- prologue: expand the whole query batch once (resident MMA B operand)
+    {
+        const int64_t nchunks = (int64_t)nst * (KBITS / 32);
+        const int64_t nw32 = ((nbits + 127) / 128) * 4;
+        for (int64_t idx = tid; idx < (int64_t)BN * nchunks; idx += NTHREADS) {
+            const int row = (int)(idx % BN);
+            const int64_t w = idx / BN;
+            uint32_t x = 0;
+            if (row < args.nq && w < nw32) x = __ldg(args.Q + row * args.ldq32 + w) & word_mask(w, nbits);
+            if (x) atomicAdd(&popQ[row], (uint32_t)__popc(x));
+            uint4 o;
+            expand4(x, o.x, o.y, o.z, o.w);
+            *reinterpret_cast<uint4 *>(qsm + (size_t)w * BN * 16 + row * 16) = o;
+        }
+    }
+    if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {
+        const int q = warp & 3;
+        uint32_t v[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) v[i] = 0x7F7F7F7Fu;   // ue8m0 scale 2^0 in every byte
+        tmem_st16(tmem + ((uint32_t)(q * 32) << 16) + C::SF_COL, v);
+        tmem_st16(tmem + ((uint32_t)(q * 32) << 16) + C::SF_COL + 16, v);
+        ptx::tmem_st_wait();
+    }
+    ptx::fence_proxy_async_smem();
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::tc_fence_after();
+
+    if (warp == TMA_WARP) {
+        // ------------------------------------------------------------ TMA producer
+        if (lane == 0) {
+            int p = 0;
+            uint32_t round = 0;   // how many times the ring has wrapped
+            for (int64_t tl = 0; tl < my_tiles; ++tl) {
+                const int64_t t = blockIdx.x + tl * gridDim.x;
+                const int32_t row0 = (int32_t)(t * BM);
+                for (int s = 0; s < nst; ++s) {
+                    if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);
+                    ptx::mbar_arrive_expect_tx(&pfull[p], PSTAGE);
+                    ptx::tma_load_2d(ring + p * PSTAGE, &tmD, &pfull[p], s * (KBITS / 32), row0);
+                    if (++p == NP) { p = 0; ++round; }
+                }
+            }
+        }
+    } else if (warp < NEXP) {
+        // ------------------------------------------------------------ expanders
+        const int qa = warp & 3, ha = warp >> 2;
+        const int arow = qa * 32 + lane;
+        uint32_t popa = 0;
+        int p = 0, b = 0, s = 0;
+        uint32_t pround = 0, bround = 0;
+        int64_t tl = 0;
+        for (int64_t it = 0; it < total_it; ++it) {
+            ptx::mbar_wait(&pfull[p], pround & 1);
+            if (bround > 0) ptx::mbar_wait(&empty[b], (bround - 1) & 1);
+            const uint4 x = *reinterpret_cast<const uint4 *>(ring + p * PSTAGE + arow * 32 + ha * 16);
+            const int64_t w0 = (int64_t)s * (KBITS / 32) + 4 * ha;
+            uint32_t wv[4] = {x.x, x.y, x.z, x.w};
+            if (w0 + 4 > full32) {
+#pragma unroll
+                for (int i = 0; i < 4; ++i) wv[i] &= word_mask(w0 + i, nbits);
+            }
+            uint32_t v[16];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                popa += __popc(wv[i]);
+                expand4(wv[i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+            }
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&pempty[p]);
+            tmem_st16(tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + 32 * b + 16 * ha), v);
+            ptx::tmem_st_wait();
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&full[b]);
+            if (++s == nst) {
+                s = 0;
+                const int acc = (int)(tl & 1);
+                if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+                popD[(acc * 2 + ha) * BM + arow] = popa;
+                popa = 0;
+                __syncwarp();
+                if (lane == 0) ptx::mbar_arrive(&popf[acc]);
+                ++tl;
+            }
+            if (++p == NP) { p = 0; ++pround; }
+            if (++b == NS) { b = 0; ++bround; }
+        }
+    } else if (warp == MMA_WARP) {
+        // ------------------------------------------------------------ MMA issuer
+        if (lane == 0) {
+            constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
+            const uint32_t sfa = tmem + C::SF_COL, sfb = tmem + C::SF_COL + 16;
+            const uint32_t qaddr = ptx::smem_u32(qsm);
+            int b = 0;
+            uint32_t bround = 0;
+            for (int64_t tl = 0; tl < my_tiles; ++tl) {
+                const int acc = (int)(tl & 1);
+                if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+                ptx::tc_fence_after();
+                const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
+                for (int s = 0; s < nst; ++s) {
+                    ptx::mbar_wait(&full[b], bround & 1);
+                    ptx::tc_fence_after();
+#pragma unroll
+                    for (int j = 0; j < KSTEPS; ++j) {
+                        const uint64_t bd = ptx::smem_desc_kmajor_noswizzle(
+                            qaddr + (uint32_t)((s * (KBITS / 32) + 2 * j) * BN * 16), BN * 16, 128);
+                        mma_mxf4_ts(d, tmem + (uint32_t)(C::A_COL0 + 32 * b + 8 * j), bd, IDESC,
+                                    (s | j) != 0 ? 1u : 0u, sfa, sfb);
+                    }
+                    ptx::mma_commit(&empty[b]);
+                    if (++b == NS) { b = 0; ++bround; }
+                }
+                ptx::mma_commit(&accf[acc]);
+            }
+        }
+        __syncwarp();
+    } else {
+        // ------------------------------------------------------------ epilogue (warps 9-12)
+        const int q = warp & 3;
+        const int li = q * 32 + lane;
+        for (int64_t tl = 0; tl < my_tiles; ++tl) {
+            const int acc = (int)(tl & 1);
+            const uint32_t ph = (uint32_t)((tl >> 1) & 1);
+            const int64_t t = blockIdx.x + tl * gridDim.x;
+            ptx::mbar_wait(&popf[acc], ph);
+            ptx::mbar_wait(&accf[acc], ph);
+            ptx::tc_fence_after();
+            const int64_t gd = t * BM + li;
+            const bool valid = gd < args.nd;
+            const int64_t pd = (int64_t)popD[(acc * 2) * BM + li] + popD[(acc * 2 + 1) * BM + li];
+            for (int cb = 0; cb < BN; cb += 8) {
+                uint32_t v[8];
+                ptx::tmem_ld8(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + cb), v);
+                ptx::tmem_ld_wait();
+                if (!valid) continue;
+#pragma unroll
+                for (int u = 0; u < 8; ++u) {
+                    const int64_t gq = cb + u;
+                    if (gq >= args.nq) break;
+                    const int64_t c = (int64_t)__float2uint_rn(__uint_as_float(v[u]));
+                    const int64_t pq = popQ[cb + u];
+                    int64_t x;
+                    switch (args.op) {
+                    case 0: x = c; break;
+                    case 1: x = pq + pd - 2 * c; break;
+                    case 2: x = pq - c; break;
+                    default: x = pd - c; break;
+                    }
+                    uint32_t *o = args.out + gq * args.ldo + gd;
+                    *o = args.accumulate ? *o + (uint32_t)x : (uint32_t)x;
+                }
+            }
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&acce[acc]);
+        }
+    }
+
+    ptx::tc_fence_before();
+    __syncthreads();
+    if (warp == MMA_WARP) {
+        ptx::tc_fence_after();
+        ptx::tmem_dealloc<512>(tmem);
+    }
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+    static EncodeTiledFn fn = nullptr;
+    if (!fn) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(p);
+    }
+    return fn;
+}
+
+int num_sms() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+size_t smem_bytes(int bn, int64_t nbits) {
+    const int64_t nst = (nbits + KBITS - 1) / KBITS;
+    return (size_t)bn * (size_t)nst * (KBITS / 32) * 16 + NP * PSTAGE + 4096;   // + barriers, pops (2.8 KB)
+}
+
+template <int BN>
+cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
+    // the database is the B operand of the user call (Q op D), on TMEM lanes here
+    FArgs f{};
+    f.Q = a.A;
+    f.nq = a.m;
+    f.ldq32 = a.lda32;
+    f.nd = a.n;
+    f.nbits = a.nbits;
+    f.op = a.op;
+    f.accumulate = a.accumulate;
+    f.ldo = a.ldc;
+    f.out = a.C;
+    f.ntiles = (a.n + BM - 1) / BM;
+    f.nst = (int)((a.nbits + KBITS - 1) / KBITS);
+    f.qbytes = (size_t)BN * f.nst * (KBITS / 32) * 16;
+    const size_t smem = smem_bytes(BN, a.nbits);
+
+    EncodeTiledFn enc = encode_fn();
+    if (!enc) return cudaErrorNotSupported;
+    CUtensorMap tm;
+    const cuuint64_t dims[2] = {(cuuint64_t)a.ldb32, (cuuint64_t)a.n};
+    const cuuint64_t strides[1] = {(cuuint64_t)a.ldb32 * 4};
+    const cuuint32_t box[2] = {KBITS / 32, BM};
+    const cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(a.B), dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+
+    auto kern = fastid_tc4_kernel<BN>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const int grid = (int)(f.ntiles < num_sms() ? f.ntiles : num_sms());
+    kern<<<grid, NTHREADS, smem, s>>>(tm, f);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+// Shape filter: queries on the column side (<= 128 rows, the user's first operand),
+// their whole expanded K range resident in shared memory, exact fp32 range.
+bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
+    if (m < 1 || m > 128 || n < 1 || nbits < 1 || nbits >= (1LL << 24)) return false;
+    if (n < 4 * m) return false;
+    if (n > (int64_t)0x7fffffff - BM) return false;
+    return smem_bytes(m <= 64 ? 64 : 128, nbits) <= MAX_SMEM;
+}
+
+cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
+    if (epi != EPI_COUNTS) return cudaErrorNotSupported;
+    return a.m <= 64 ? launch_f<64>(a, s) : launch_f<128>(a, s);
+}
+
+}  // namespace snp

@@ -107,7 +107,11 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
         // for exact fp32 accumulation or SNP_TC_KIND=i8 asks for the int8 kernel.
         const char *kind = std::getenv("SNP_TC_KIND");
         const bool want_i8 = kind && !std::strcmp(kind, "i8");
-        if (!want_i8 && tc4_supported(a.m, a.n, a.nbits))
+        const char *ff = std::getenv("SNP_FASTID_KERNEL");
+        const bool no_fastid = ff && !std::strcmp(ff, "0");
+        if (!want_i8 && !no_fastid && epi == EPI_COUNTS && fastid_tc4_supported(a.m, a.n, a.nbits))
+            e = launch_fastid_tc4(a, epi, s);
+        else if (!want_i8 && tc4_supported(a.m, a.n, a.nbits))
             e = launch_bitgemm_tc4(a, epi, s);
         else
             e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);

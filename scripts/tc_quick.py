@@ -8,12 +8,13 @@ import paper_conf_ipps_binderlp19_b200 as snp
 torch.cuda.set_device(0)
 snp.snp_set_variant(os.environ.get("V", "tc"))
 bad_total = 0
-for (m, n, nbits) in [(128, 64, 256), (130, 70, 300), (200, 300, 1000), (64, 1000, 4096), (300, 129, 2049)]:
+for (m, n, nbits) in [(128, 64, 256), (130, 70, 300), (200, 300, 1000), (64, 1000, 4096), (300, 129, 2049),
+                      (1, 5000, 100), (64, 3000, 4097), (100, 2000, 777), (33, 40000, 256)]:
     ga = snpgen.fastid_db(5, np.arange(m), nbits)
     gb = snpgen.fastid_db(6, np.arange(n), nbits)
     A = snp.snp_pack(torch.from_numpy(ga).cuda())
     B = snp.snp_pack(torch.from_numpy(gb).cuda())
-    for op in ("and", "xor"):
+    for op in ("and", "xor", "andnot", "notand"):
         out = snp.snp_fastid(A, B, nbits, op)
         torch.cuda.synchronize()
         got = out.cpu().numpy().astype(np.int64)
