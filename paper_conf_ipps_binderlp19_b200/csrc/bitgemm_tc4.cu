@@ -34,7 +34,7 @@ namespace {
 
 constexpr int BM = 128;            // MMA M = TMEM lanes (lane-side rows per tile)
 constexpr int KBITS = 256;         // bits per pipeline stage
-constexpr int KSTEPS = KBITS / 64; // MMA instructions per stage (K = 64 per instruction)
+static_assert(KBITS == 256, "a stage is exactly the 4 K=64 MMAs of mma4_mxf4_ts_commit");
 constexpr int NS = 4;              // pipeline stages
 constexpr int PF = 4;              // register prefetch depth (stages)
 constexpr int NEXP = 8;            // expander warps
@@ -98,14 +98,6 @@ __host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
     return (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
 }
 
-__device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a_tmem, uint64_t bdesc, uint32_t idesc,
-                                            uint32_t accumulate, uint32_t sfa, uint32_t sfb) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}" ::"r"(d),
-        "r"(a_tmem), "l"(bdesc), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb));
-}
 
 __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
     asm volatile(
@@ -288,31 +280,27 @@ __global__ void __launch_bounds__(NTHREADS, 1) bitgemm_tc4_kernel(const Tc4Args 
         }
     } else if (warp == MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
-        if (lane == 0) {
-            constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
-            const uint32_t sfa = tmem + C::SF_COL, sfb = tmem + C::SF_COL + 16;
-            const uint32_t bsm = ptx::smem_u32(bstage);
-            int64_t it = 0;
-            for (int64_t tl = 0; tl < my_tiles; ++tl) {
-                const int acc = (int)(tl & 1);
-                if (tl >= 2) ptx::mbar_wait(&acce_bar[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+        // whole warp converged; one elected lane issues a stage's 4 MMAs + commit
+        constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
+        const uint32_t sfa = tmem + C::SF_COL, sfb = tmem + C::SF_COL + 16;
+        const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(bstage), BN * 16, 128);
+        constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;
+        int b = 0;
+        uint32_t bround = 0;
+        for (int64_t tl = 0; tl < my_tiles; ++tl) {
+            const int acc = (int)(tl & 1);
+            if (tl >= 2) ptx::mbar_wait(&acce_bar[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            ptx::tc_fence_after();
+            const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
+            for (int s = 0; s < nst; ++s) {
+                ptx::mbar_wait(&full_bar[b], bround & 1);
                 ptx::tc_fence_after();
-                const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
-                for (int s = 0; s < nst; ++s, ++it) {
-                    const int b = (int)(it % NS);
-                    ptx::mbar_wait(&full_bar[b], (uint32_t)((it / NS) & 1));
-                    ptx::tc_fence_after();
-#pragma unroll
-                    for (int j = 0; j < KSTEPS; ++j) {
-                        const uint64_t bd = ptx::smem_desc_kmajor_noswizzle(
-                            bsm + (uint32_t)(b * C::B_STAGE + 2 * j * BN * 16), BN * 16, 128);
-                        mma_mxf4_ts(d, tmem + (uint32_t)(C::A_COL0 + 32 * b + 8 * j), bd, IDESC,
-                                    (s | j) != 0 ? 1u : 0u, sfa, sfb);
-                    }
-                    ptx::mma_commit(&empty_bar[b]);
-                }
-                ptx::mma_commit(&accf_bar[acc]);
+                ptx::mma4_mxf4_ts_commit(d, tmem + (uint32_t)(C::A_COL0 + 32 * b),
+                                         bdesc0 + (uint64_t)((b * C::B_STAGE) >> 4), BSTEP, IDESC,
+                                         s != 0 ? 1u : 0u, sfa, sfb, &empty_bar[b]);
+                if (++b == NS) { b = 0; ++bround; }
             }
+            ptx::mma_commit_elect(&accf_bar[acc]);
         }
         __syncwarp();
     } else {

@@ -29,19 +29,21 @@ namespace {
 
 constexpr int BM = 128;
 constexpr int KBITS = 256;
-constexpr int KSTEPS = KBITS / 64;
+static_assert(KBITS == 256, "a stage is exactly the 4 K=64 MMAs of mma4_mxf4_ts_commit");
 constexpr int NP = 16;                  // packed TMA ring depth
 constexpr int PSTAGE = BM * KBITS / 8;  // 4 KB packed per stage
-constexpr int NEXP = 8;
-constexpr int MMA_WARP = 8;
-constexpr int EPI_WARP0 = 9;
-constexpr int TMA_WARP = 13;
-constexpr int NTHREADS = 14 * 32;
+constexpr int G = 4;                    // expander groups (group g takes stages it = g mod G)
+constexpr int NEXP = 4 * G;             // expander warps: group g = warps 4g..4g+3 (one per lane quarter)
+constexpr int MMA_WARP = NEXP;          // 16
+constexpr int EPI_WARP0 = NEXP + 1;     // 17..20 -> lane quarters 1,2,3,0
+constexpr int TMA_WARP = NEXP + 5;      // 21
+constexpr int NTHREADS = (NEXP + 6) * 32;
 constexpr size_t MAX_SMEM = 232448;     // 227 KB opt-in
 
 template <int BN>
 struct FCfg {
-    static constexpr int NS = BN <= 64 ? 8 : 6;     // TMEM A stages
+    static constexpr int NS = BN <= 64 ? 8 : 4;     // TMEM A stages (multiple of G)
+    static_assert(NS % G == 0 && NP % G == 0, "rings must be multiples of the group count");
     static constexpr int ACC_COLS = BN;
     static constexpr int A_COL0 = 2 * ACC_COLS;
     static constexpr int SF_COL = A_COL0 + NS * 32;
@@ -80,14 +82,6 @@ __host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
     return (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
 }
 
-__device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a_tmem, uint64_t bdesc, uint32_t idesc,
-                                            uint32_t accumulate, uint32_t sfa, uint32_t sfb) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}" ::"r"(d),
-        "r"(a_tmem), "l"(bdesc), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb));
-}
 
 __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
     asm volatile(
@@ -98,7 +92,18 @@ __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16
         : "memory");
 }
 
-template <int BN>
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+        "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
+        "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]),
+        "r"(v[17]), "r"(v[18]), "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]),
+        "r"(v[25]), "r"(v[26]), "r"(v[27]), "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
+        : "memory");
+}
+
+template <int BN, int OP>
 __global__ void __launch_bounds__(NTHREADS, 1)
 fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     using C = FCfg<BN>;
@@ -116,7 +121,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     uint64_t *popf = acce + 2;               // [2]
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popf + 2);
     uint32_t *popQ = tmem_slot + 4;          // [BN]
-    uint32_t *popD = popQ + BN;              // [2 acc][2 half][BM]
+    uint32_t *popD = popQ + BN;              // [2 acc][G][BM]
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t nbits = args.nbits;
@@ -128,10 +133,10 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     if (tid == 0) {
         for (int i = 0; i < NP; ++i) {
             ptx::mbar_init(&pfull[i], 1);
-            ptx::mbar_init(&pempty[i], NEXP);
+            ptx::mbar_init(&pempty[i], 4);
         }
         for (int i = 0; i < NS; ++i) {
-            ptx::mbar_init(&full[i], NEXP);
+            ptx::mbar_init(&full[i], 4);
             ptx::mbar_init(&empty[i], 1);
         }
         for (int i = 0; i < 2; ++i) {
@@ -196,76 +201,87 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         }
     } else if (warp < NEXP) {
         // ------------------------------------------------------------ expanders
-        const int qa = warp & 3, ha = warp >> 2;
+        // group g = warp / 4 handles iterations it = g, g+G, ...; warp (g, q) handles the
+        // 32 database rows of lane quarter q for all 256 bits of the stage.
+        const int g = warp >> 2, qa = warp & 3;
         const int arow = qa * 32 + lane;
         uint32_t popa = 0;
-        int p = 0, b = 0, s = 0;
+        int64_t cur_tl = 0;   // tile whose popcount partial is being accumulated
+        auto publish_until = [&](int64_t upto) {
+            for (; cur_tl < upto; ++cur_tl) {
+                const int acc = (int)(cur_tl & 1);
+                if (cur_tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((cur_tl >> 1) - 1) & 1));
+                popD[(acc * G + g) * BM + arow] = popa;
+                popa = 0;
+                __syncwarp();
+                if (lane == 0) ptx::mbar_arrive(&popf[acc]);
+            }
+        };
+        int64_t tl = g / nst;
+        int s = g % nst;
+        int p = g, b = g;
         uint32_t pround = 0, bround = 0;
-        int64_t tl = 0;
-        for (int64_t it = 0; it < total_it; ++it) {
+        for (int64_t it = g; it < total_it; it += G) {
+            publish_until(tl);
             ptx::mbar_wait(&pfull[p], pround & 1);
             if (bround > 0) ptx::mbar_wait(&empty[b], (bround - 1) & 1);
-            const uint4 x = *reinterpret_cast<const uint4 *>(ring + p * PSTAGE + arow * 32 + ha * 16);
-            const int64_t w0 = (int64_t)s * (KBITS / 32) + 4 * ha;
-            uint32_t wv[4] = {x.x, x.y, x.z, x.w};
-            if (w0 + 4 > full32) {
+            const uint8_t *src = ring + p * PSTAGE + arow * 32;
+            const uint4 x0 = *reinterpret_cast<const uint4 *>(src);
+            const uint4 x1 = *reinterpret_cast<const uint4 *>(src + 16);
+            uint32_t wv[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+            const int64_t w0 = (int64_t)s * (KBITS / 32);
+            if (w0 + 8 > full32) {
 #pragma unroll
-                for (int i = 0; i < 4; ++i) wv[i] &= word_mask(w0 + i, nbits);
+                for (int i = 0; i < 8; ++i) wv[i] &= word_mask(w0 + i, nbits);
             }
-            uint32_t v[16];
+            uint32_t v[32];
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
+            for (int i = 0; i < 8; ++i) {
                 popa += __popc(wv[i]);
                 expand4(wv[i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
             }
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&pempty[p]);
-            tmem_st16(tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + 32 * b + 16 * ha), v);
+            tmem_st32(tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + 32 * b), v);
             ptx::tmem_st_wait();
             ptx::tc_fence_before();
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&full[b]);
-            if (++s == nst) {
-                s = 0;
-                const int acc = (int)(tl & 1);
-                if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
-                popD[(acc * 2 + ha) * BM + arow] = popa;
-                popa = 0;
-                __syncwarp();
-                if (lane == 0) ptx::mbar_arrive(&popf[acc]);
-                ++tl;
-            }
-            if (++p == NP) { p = 0; ++pround; }
-            if (++b == NS) { b = 0; ++bround; }
+            s += G;
+            while (s >= nst) { s -= nst; ++tl; }
+            p += G;
+            if (p >= NP) { p -= NP; ++pround; }
+            b += G;
+            if (b >= NS) { b -= NS; ++bround; }
         }
+        publish_until(my_tiles);
     } else if (warp == MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
-        if (lane == 0) {
-            constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
-            const uint32_t sfa = tmem + C::SF_COL, sfb = tmem + C::SF_COL + 16;
-            const uint32_t qaddr = ptx::smem_u32(qsm);
-            int b = 0;
-            uint32_t bround = 0;
-            for (int64_t tl = 0; tl < my_tiles; ++tl) {
-                const int acc = (int)(tl & 1);
-                if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+        // The whole warp runs the loop (converged, uniform values); one elected lane issues
+        // the 4 MMAs of a stage and the commit in a single asm block.  Descriptors are
+        // precomputed: stepping K only adds to the start-address field.
+        constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
+        const uint32_t sfa = tmem + C::SF_COL, sfb = tmem + C::SF_COL + 16;
+        const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(qsm), BN * 16, 128);
+        constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;           // one K-step = 2 chunks
+        constexpr uint32_t SSTEP = ((KBITS / 32) * BN * 16) >> 4; // one stage = 8 chunks
+        int b = 0;
+        uint32_t bround = 0;
+        for (int64_t tl = 0; tl < my_tiles; ++tl) {
+            const int acc = (int)(tl & 1);
+            if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            ptx::tc_fence_after();
+            const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
+            uint64_t bd = bdesc0;
+            for (int s = 0; s < nst; ++s) {
+                ptx::mbar_wait(&full[b], bround & 1);
                 ptx::tc_fence_after();
-                const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
-                for (int s = 0; s < nst; ++s) {
-                    ptx::mbar_wait(&full[b], bround & 1);
-                    ptx::tc_fence_after();
-#pragma unroll
-                    for (int j = 0; j < KSTEPS; ++j) {
-                        const uint64_t bd = ptx::smem_desc_kmajor_noswizzle(
-                            qaddr + (uint32_t)((s * (KBITS / 32) + 2 * j) * BN * 16), BN * 16, 128);
-                        mma_mxf4_ts(d, tmem + (uint32_t)(C::A_COL0 + 32 * b + 8 * j), bd, IDESC,
-                                    (s | j) != 0 ? 1u : 0u, sfa, sfb);
-                    }
-                    ptx::mma_commit(&empty[b]);
-                    if (++b == NS) { b = 0; ++bround; }
-                }
-                ptx::mma_commit(&accf[acc]);
+                ptx::mma4_mxf4_ts_commit(d, tmem + (uint32_t)(C::A_COL0 + 32 * b), bd, BSTEP, IDESC,
+                                         s != 0 ? 1u : 0u, sfa, sfb, &empty[b]);
+                bd += SSTEP;
+                if (++b == NS) { b = 0; ++bround; }
             }
+            ptx::mma_commit_elect(&accf[acc]);
         }
         __syncwarp();
     } else {
@@ -281,27 +297,28 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             ptx::tc_fence_after();
             const int64_t gd = t * BM + li;
             const bool valid = gd < args.nd;
-            const int64_t pd = (int64_t)popD[(acc * 2) * BM + li] + popD[(acc * 2 + 1) * BM + li];
+            uint32_t pd = 0;
+#pragma unroll
+            for (int gg = 0; gg < G; ++gg) pd += popD[(acc * G + gg) * BM + li];
+            uint32_t *col = args.out + gd;
+            const int64_t ldo = args.ldo;
+            const int nq = (int)args.nq;
             for (int cb = 0; cb < BN; cb += 8) {
                 uint32_t v[8];
                 ptx::tmem_ld8(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + cb), v);
                 ptx::tmem_ld_wait();
-                if (!valid) continue;
+                if (!valid || cb >= nq) continue;
 #pragma unroll
                 for (int u = 0; u < 8; ++u) {
-                    const int64_t gq = cb + u;
-                    if (gq >= args.nq) break;
-                    const int64_t c = (int64_t)__float2uint_rn(__uint_as_float(v[u]));
-                    const int64_t pq = popQ[cb + u];
-                    int64_t x;
-                    switch (args.op) {
-                    case 0: x = c; break;
-                    case 1: x = pq + pd - 2 * c; break;
-                    case 2: x = pq - c; break;
-                    default: x = pd - c; break;
-                    }
-                    uint32_t *o = args.out + gq * args.ldo + gd;
-                    *o = args.accumulate ? *o + (uint32_t)x : (uint32_t)x;
+                    if (cb + u >= nq) break;
+                    const uint32_t c = __float2uint_rn(__uint_as_float(v[u]));
+                    uint32_t x;   // exact: every result is a count in [0, 2^31)
+                    if (OP == 0) x = c;
+                    else if (OP == 1) x = popQ[cb + u] + pd - 2u * c;
+                    else if (OP == 2) x = popQ[cb + u] - c;
+                    else x = pd - c;
+                    uint32_t *o = col + (int64_t)(cb + u) * ldo;
+                    *o = args.accumulate ? *o + x : x;
                 }
             }
             ptx::tc_fence_before();
@@ -347,7 +364,7 @@ int num_sms() {
 
 size_t smem_bytes(int bn, int64_t nbits) {
     const int64_t nst = (nbits + KBITS - 1) / KBITS;
-    return (size_t)bn * (size_t)nst * (KBITS / 32) * 16 + NP * PSTAGE + 4096;   // + barriers, pops (2.8 KB)
+    return (size_t)bn * (size_t)nst * (KBITS / 32) * 16 + NP * PSTAGE + 8192;   // + barriers, pops (~5 KB)
 }
 
 template <int BN>
@@ -380,7 +397,10 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
 
-    auto kern = fastid_tc4_kernel<BN>;
+    void (*kern)(const CUtensorMap, const FArgs) = a.op == 0   ? fastid_tc4_kernel<BN, 0>
+                                                   : a.op == 1 ? fastid_tc4_kernel<BN, 1>
+                                                   : a.op == 2 ? fastid_tc4_kernel<BN, 2>
+                                                               : fastid_tc4_kernel<BN, 3>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     const int grid = (int)(f.ntiles < num_sms() ? f.ntiles : num_sms());

@@ -145,6 +145,37 @@ __device__ __forceinline__ void mma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, uint
         "r"(tmem_a), "l"(bdesc), "r"(idesc), "r"(accumulate), "r"(0), "r"(0), "r"(0), "r"(0));
 }
 
+// Four K-steps of tcgen05.mma kind::mxf4 (block32 scales) with A from TMEM, then a
+// commit to `bar`, issued by ONE elected lane of a converged warp (the whole warp
+// must call it).  K-step i uses A columns a0 + 8 i and B descriptor b0 + i * bstep
+// (descriptor start-address field, 16-byte units).  The first MMA accumulates iff
+// `accumulate`; the other three always accumulate.
+__device__ __forceinline__ void mma4_mxf4_ts_commit(uint32_t d, uint32_t a0, uint64_t b0, uint32_t bstep,
+                                                    uint32_t idesc, uint32_t accumulate, uint32_t sfa,
+                                                    uint32_t sfb, uint64_t *bar) {
+    const uint64_t b1 = b0 + bstep, b2 = b0 + 2 * bstep, b3 = b0 + 3 * bstep;
+    asm volatile(
+        "{\n\t.reg .pred e, p, t;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "setp.ne.b32 p, %9, 0;\n\t"
+        "setp.eq.b32 t, 0, 0;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %5, %10, [%11], [%12], p;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%2], %6, %10, [%11], [%12], t;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%3], %7, %10, [%11], [%12], t;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%4], %8, %10, [%11], [%12], t;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%13];\n\t}" ::"r"(d),
+        "r"(a0), "r"(a0 + 8), "r"(a0 + 16), "r"(a0 + 24), "l"(b0), "l"(b1), "l"(b2), "l"(b3), "r"(accumulate),
+        "r"(idesc), "r"(sfa), "r"(sfb), "r"(smem_u32(bar))
+        : "memory");
+}
+// Commit by one elected lane of a converged warp.
+__device__ __forceinline__ void mma_commit_elect(uint64_t *bar) {
+    asm volatile(
+        "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
+        : "memory");
+}
+
 // Arrive on an mbarrier when all previously issued tcgen05.mma of this thread finish.
 __device__ __forceinline__ void mma_commit(uint64_t *bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(

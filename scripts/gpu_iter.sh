@@ -7,5 +7,5 @@ timeout 300 python bench.py --workload $w --steps 10 --warmup 3 --variant tc --n
 done
 python scripts/summarize.py gpurun_out/bench_fastid1m.log gpurun_out/bench_ld32k.log gpurun_out/bench_ld2k.log
 if [ -n "$NCU" ]; then
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:bitgemm_tc4 -s 4 -c 1 -o gpurun_out/prof_iter python bench.py --steps 2 --warmup 3 --variant tc --no-cpu-baseline --no-e2e > gpurun_out/ncu_iter.log 2>&1; echo ncu=$?
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:${KREGEX:-tc4_kernel} -s 4 -c 1 -o gpurun_out/prof_iter python bench.py --steps 2 --warmup 3 --variant tc --no-cpu-baseline --no-e2e > gpurun_out/ncu_iter.log 2>&1; echo ncu=$?
 fi

@@ -1,0 +1,81 @@
+// mma_probe.cu — microbenchmark of tcgen05.mma issue throughput on B200 (one CTA per SM,
+// one issuing thread, back-to-back MMAs on garbage operands, clock64 around them).
+// Used to pick the tensor-core kernel shapes.  Not part of the library.
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "../paper_conf_ipps_binderlp19_b200/csrc/tc_ptx.cuh"
+using namespace snp;
+
+__host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
+    return (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
+}
+__device__ __forceinline__ void mma_mxf4_ss(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc, uint32_t sfa, uint32_t sfb) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], %1, %2, %3, [%5], [%6], p;\n\t}"
+                 :: "r"(d), "l"(a), "l"(b), "r"(idesc), "r"(acc), "r"(sfa), "r"(sfb));
+}
+__device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a, uint64_t b, uint32_t idesc, uint32_t acc, uint32_t sfa, uint32_t sfb) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}"
+                 :: "r"(d), "r"(a), "l"(b), "r"(idesc), "r"(acc), "r"(sfa), "r"(sfb));
+}
+
+template <int MODE, int N>   // MODE 0: mxf4 SS, 1: mxf4 TS, 2: i8 SS, 3: i8 TS
+__global__ void probe(int iters, long long *out) {
+    extern __shared__ __align__(1024) uint8_t sm[];
+    __shared__ uint64_t bar;
+    __shared__ uint32_t slot;
+    if (threadIdx.x < 32) ptx::tmem_alloc<512>(&slot);
+    if (threadIdx.x == 0) { ptx::mbar_init(&bar, 1); ptx::fence_mbar_init(); }
+    ptx::tc_fence_before(); __syncthreads(); ptx::tc_fence_after();
+    uint32_t tmem = slot;
+    if (threadIdx.x == 0) {
+        const uint32_t sa = ptx::smem_u32(sm), sb = sa + 128 * 32;
+        const uint64_t ad = ptx::smem_desc_kmajor_noswizzle(sa, 128 * 16, 128);
+        const uint64_t bd = ptx::smem_desc_kmajor_noswizzle(sb, N * 16, 128);
+        long long t0 = clock64();
+        for (int i = 0; i < iters; ++i) {
+            if (MODE == 0) mma_mxf4_ss(tmem, ad, bd, idesc_mxf4(128, N), 1, tmem + 480, tmem + 496);
+            else if (MODE == 1) mma_mxf4_ts(tmem, tmem + 256 + (i & 7) * 8, bd, idesc_mxf4(128, N), 1, tmem + 480, tmem + 496);
+            else if (MODE == 2) ptx::mma_i8_ss(tmem, ad, bd, ptx::idesc_u8_s32(128, N), 1);
+            else ptx::mma_i8_ts(tmem, tmem + 256 + (i & 7) * 8, bd, ptx::idesc_u8_s32(128, N), 1);
+        }
+        ptx::mma_commit(&bar);
+        ptx::mbar_wait(&bar, 0);
+        long long t1 = clock64();
+        out[blockIdx.x] = t1 - t0;
+    }
+    ptx::tc_fence_before(); __syncthreads();
+    if (threadIdx.x < 32) { ptx::tc_fence_after(); ptx::tmem_dealloc<512>(tmem); }
+}
+
+template <int MODE, int N>
+void run(const char *name) {
+    long long *d; cudaMalloc(&d, 148 * sizeof(long long));
+    const int iters = 4096;
+    auto k = probe<MODE, N>;
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    k<<<148, 128, 64 * 1024>>>(iters, d);
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    cudaEventRecord(e0);
+    k<<<148, 128, 64 * 1024>>>(iters, d);
+    cudaEventRecord(e1); cudaEventSynchronize(e1);
+    float ms; cudaEventElapsedTime(&ms, e0, e1);
+    long long h[148]; cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
+    cudaError_t err = cudaGetLastError();
+    double cyc = (double)h[0] / iters;
+    const int K = (MODE <= 1) ? 64 : 32;
+    double macs = 128.0 * N * K * iters * 148;
+    printf("%-14s N=%3d  %7.1f cycles/MMA  %8.1f MAC/clk/SM  %7.0f TMAC/s (event %.3f ms) %s\n", name, N, cyc,
+           128.0 * N * K / cyc, macs / (ms * 1e-3) / 1e12, ms, err == cudaSuccess ? "" : cudaGetErrorString(err));
+    cudaFree(d);
+}
+
+int main() {
+    run<0, 64>("mxf4 SS"); run<0, 128>("mxf4 SS"); run<0, 256>("mxf4 SS");
+    run<1, 64>("mxf4 TS"); run<1, 128>("mxf4 TS"); run<1, 256>("mxf4 TS");
+    run<2, 64>("i8 SS"); run<2, 128>("i8 SS"); run<2, 256>("i8 SS");
+    run<3, 64>("i8 TS"); run<3, 128>("i8 TS"); run<3, 256>("i8 TS");
+    return 0;
+}
