@@ -23,30 +23,40 @@
 #include "tc_ptx.cuh"
 
 #include <cuda.h>
+#include <cstdlib>
 
 namespace snp {
+
+// Pipeline trace (profiling aid, read with snp_debug_fastid_trace): CTA 0 records
+// clock64 stamps per iteration: [0] expander before waits, [1] after pfull+empty,
+// [2] before full arrive, [3] MMA after full wait.  Enabled by SNP_TRACE=1.
+__device__ long long g_fastid_trace[8 * 1024];
+
 namespace {
 
 constexpr int BM = 128;
-constexpr int KBITS = 256;
-static_assert(KBITS == 256, "a stage is exactly the 4 K=64 MMAs of mma4_mxf4_ts_commit");
-constexpr int NP = 16;                  // packed TMA ring depth
-constexpr int PSTAGE = BM * KBITS / 8;  // 4 KB packed per stage
+constexpr int KBITS = 512;
+static_assert(KBITS == 512, "a stage is exactly the 8 K=64 MMAs of mma8_mxf4_ts_commit");
+constexpr int NP = 8;                   // packed TMA ring depth (64 KB in flight per SM)
+constexpr int PSTAGE = BM * KBITS / 8;  // 8 KB packed per stage, 64-byte rows, 64B-swizzled
 constexpr int G = 4;                    // expander groups (group g takes stages it = g mod G)
 constexpr int NEXP = 4 * G;             // expander warps: group g = warps 4g..4g+3 (one per lane quarter)
-constexpr int MMA_WARP = NEXP;          // 16
-constexpr int EPI_WARP0 = NEXP + 1;     // 17..20 -> lane quarters 1,2,3,0
-constexpr int TMA_WARP = NEXP + 5;      // 21
-constexpr int NTHREADS = (NEXP + 6) * 32;
+// The warp scheduler favours higher warp ids, so the latency-critical single-thread
+// roles get the highest ids: MMA issuer last, TMA producer next, epilogue below them.
+constexpr int NEPI = 8;                 // epilogue warps 16..23: lane quarter w % 4, column half
+constexpr int EPI_WARP0 = NEXP;
+constexpr int TMA_WARP = NEXP + NEPI;   // 24
+constexpr int MMA_WARP = NEXP + NEPI + 1;   // 25
+constexpr int NTHREADS = (NEXP + NEPI + 2) * 32;
 constexpr size_t MAX_SMEM = 232448;     // 227 KB opt-in
 
 template <int BN>
 struct FCfg {
-    static constexpr int NS = BN <= 64 ? 8 : 4;     // TMEM A stages (multiple of G)
+    static constexpr int NS = 4;                    // TMEM A stages of 64 columns (multiple of G)
     static_assert(NS % G == 0 && NP % G == 0, "rings must be multiples of the group count");
     static constexpr int ACC_COLS = BN;
     static constexpr int A_COL0 = 2 * ACC_COLS;
-    static constexpr int SF_COL = A_COL0 + NS * 32;
+    static constexpr int SF_COL = A_COL0 + NS * 64;
     static_assert(SF_COL + 32 <= 512, "TMEM budget");
 };
 
@@ -61,6 +71,7 @@ struct FArgs {
     int64_t ntiles;
     int nst;
     size_t qbytes;       // expanded query bytes in shared memory
+    int trace;
 };
 
 __device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
@@ -103,6 +114,17 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32
         : "memory");
 }
 
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+        "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
+          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+        : "r"(taddr));
+}
+
 template <int BN, int OP>
 __global__ void __launch_bounds__(NTHREADS, 1)
 fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
@@ -141,7 +163,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         }
         for (int i = 0; i < 2; ++i) {
             ptx::mbar_init(&accf[i], 1);
-            ptx::mbar_init(&acce[i], 4);
+            ptx::mbar_init(&acce[i], NEPI);
             ptx::mbar_init(&popf[i], NEXP);
         }
         ptx::fence_mbar_init();
@@ -169,7 +191,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             *reinterpret_cast<uint4 *>(qsm + (size_t)w * BN * 16 + row * 16) = o;
         }
     }
-    if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {
+    if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {   // one warp per lane quarter
         const int q = warp & 3;
         uint32_t v[16];
 #pragma unroll
@@ -223,29 +245,43 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         uint32_t pround = 0, bround = 0;
         for (int64_t it = g; it < total_it; it += G) {
             publish_until(tl);
+            const bool tr = args.trace && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
+            if (tr) g_fastid_trace[8 * it + 0] = clock64();
             ptx::mbar_wait(&pfull[p], pround & 1);
             if (bround > 0) ptx::mbar_wait(&empty[b], (bround - 1) & 1);
-            const uint8_t *src = ring + p * PSTAGE + arow * 32;
-            const uint4 x0 = *reinterpret_cast<const uint4 *>(src);
-            const uint4 x1 = *reinterpret_cast<const uint4 *>(src + 16);
-            uint32_t wv[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+            if (tr) g_fastid_trace[8 * it + 1] = clock64();
+            // 64-byte row of the stage; TMA 64B swizzle: 16-byte chunk c of row r sits at
+            // chunk c ^ ((r >> 1) & 3)  (conflict-free LDS.128 across the warp)
+            const uint8_t *src = ring + p * PSTAGE + arow * 64;
+            const int sw = (arow >> 1) & 3;
+            uint32_t wv[16];
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const uint4 x = *reinterpret_cast<const uint4 *>(src + ((c ^ sw) << 4));
+                wv[4 * c] = x.x; wv[4 * c + 1] = x.y; wv[4 * c + 2] = x.z; wv[4 * c + 3] = x.w;
+            }
             const int64_t w0 = (int64_t)s * (KBITS / 32);
-            if (w0 + 8 > full32) {
+            if (w0 + 16 > full32) {
 #pragma unroll
-                for (int i = 0; i < 8; ++i) wv[i] &= word_mask(w0 + i, nbits);
+                for (int i = 0; i < 16; ++i) wv[i] &= word_mask(w0 + i, nbits);
             }
-            uint32_t v[32];
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                popa += __popc(wv[i]);
-                expand4(wv[i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-            }
+            for (int i = 0; i < 16; ++i) popa += __popc(wv[i]);
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&pempty[p]);
-            tmem_st32(tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + 32 * b), v);
+            const uint32_t tbase = tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + 64 * b);
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                uint32_t v[32];
+#pragma unroll
+                for (int i = 0; i < 8; ++i)
+                    expand4(wv[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+                tmem_st32(tbase + 32 * h, v);
+            }
             ptx::tmem_st_wait();
             ptx::tc_fence_before();
             __syncwarp();
+            if (tr) g_fastid_trace[8 * it + 2] = clock64();
             if (lane == 0) ptx::mbar_arrive(&full[b]);
             s += G;
             while (s >= nst) { s -= nst; ++tl; }
@@ -264,20 +300,25 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         const uint32_t sfa = tmem + C::SF_COL, sfb = tmem + C::SF_COL + 16;
         const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(qsm), BN * 16, 128);
         constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;           // one K-step = 2 chunks
-        constexpr uint32_t SSTEP = ((KBITS / 32) * BN * 16) >> 4; // one stage = 8 chunks
+        constexpr uint32_t SSTEP = ((KBITS / 32) * BN * 16) >> 4; // one stage = 16 chunks
         int b = 0;
         uint32_t bround = 0;
+        int64_t itm = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
             if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
             ptx::tc_fence_after();
             const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
             uint64_t bd = bdesc0;
-            for (int s = 0; s < nst; ++s) {
+            for (int s = 0; s < nst; ++s, ++itm) {
                 ptx::mbar_wait(&full[b], bround & 1);
+                const bool trm = args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024;
+                if (trm) g_fastid_trace[8 * itm + 3] = clock64();
                 ptx::tc_fence_after();
-                ptx::mma4_mxf4_ts_commit(d, tmem + (uint32_t)(C::A_COL0 + 32 * b), bd, BSTEP, IDESC,
+
+                ptx::mma8_mxf4_ts_commit(d, tmem + (uint32_t)(C::A_COL0 + 64 * b), bd, BSTEP, IDESC,
                                          s != 0 ? 1u : 0u, sfa, sfb, &empty[b]);
+
                 bd += SSTEP;
                 if (++b == NS) { b = 0; ++bround; }
             }
@@ -285,9 +326,14 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         }
         __syncwarp();
     } else {
-        // ------------------------------------------------------------ epilogue (warps 9-12)
-        const int q = warp & 3;
+        // ------------------------------------------------------------ epilogue (8 warps)
+        // warp e: TMEM lane quarter e % 4 (database rows), query columns [32 h, 32 h + 32)
+        const int e = warp - EPI_WARP0;
+        const int q = e & 3, h = e >> 2;
         const int li = q * 32 + lane;
+        const int c0 = 32 * h;
+        const int ncols = (int)(args.nq - c0 < 32 ? (args.nq - c0 > 0 ? args.nq - c0 : 0) : 32);
+        const int64_t ldo = args.ldo;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
@@ -295,35 +341,45 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             ptx::mbar_wait(&popf[acc], ph);
             ptx::mbar_wait(&accf[acc], ph);
             ptx::tc_fence_after();
-            const int64_t gd = t * BM + li;
-            const bool valid = gd < args.nd;
-            uint32_t pd = 0;
+            uint32_t v[32];
+            tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
+            uint32_t pd = 0;   // read the popcount partials BEFORE releasing the buffer pair
 #pragma unroll
             for (int gg = 0; gg < G; ++gg) pd += popD[(acc * G + gg) * BM + li];
-            uint32_t *col = args.out + gd;
-            const int64_t ldo = args.ldo;
-            const int nq = (int)args.nq;
-            for (int cb = 0; cb < BN; cb += 8) {
-                uint32_t v[8];
-                ptx::tmem_ld8(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + cb), v);
-                ptx::tmem_ld_wait();
-                if (!valid || cb >= nq) continue;
-#pragma unroll
-                for (int u = 0; u < 8; ++u) {
-                    if (cb + u >= nq) break;
-                    const uint32_t c = __float2uint_rn(__uint_as_float(v[u]));
-                    uint32_t x;   // exact: every result is a count in [0, 2^31)
-                    if (OP == 0) x = c;
-                    else if (OP == 1) x = popQ[cb + u] + pd - 2u * c;
-                    else if (OP == 2) x = popQ[cb + u] - c;
-                    else x = pd - c;
-                    uint32_t *o = col + (int64_t)(cb + u) * ldo;
-                    *o = args.accumulate ? *o + x : x;
-                }
-            }
+            ptx::tmem_ld_wait();
             ptx::tc_fence_before();
             __syncwarp();
-            if (lane == 0) ptx::mbar_arrive(&acce[acc]);
+            if (lane == 0) ptx::mbar_arrive(&acce[acc]);   // accumulator + pops drained: reusable
+            const int64_t gd = t * BM + li;
+            if (gd < args.nd && ncols > 0) {
+                uint32_t *o = args.out + (int64_t)c0 * ldo + gd;
+                if (ncols == 32 && !args.accumulate) {
+#pragma unroll
+                    for (int u = 0; u < 32; ++u) {
+                        const uint32_t c = __float2uint_rn(__uint_as_float(v[u]));
+                        uint32_t x;   // exact: every result is a count in [0, 2^31)
+                        if (OP == 0) x = c;
+                        else if (OP == 1) x = popQ[c0 + u] + pd - 2u * c;
+                        else if (OP == 2) x = popQ[c0 + u] - c;
+                        else x = pd - c;
+                        __stcs(o, x);          // streaming store: written once, never re-read here
+                        o += ldo;
+                    }
+                } else {
+#pragma unroll
+                    for (int u = 0; u < 32; ++u) {
+                        if (u >= ncols) break;
+                        const uint32_t c = __float2uint_rn(__uint_as_float(v[u]));
+                        uint32_t x;
+                        if (OP == 0) x = c;
+                        else if (OP == 1) x = popQ[c0 + u] + pd - 2u * c;
+                        else if (OP == 2) x = popQ[c0 + u] - c;
+                        else x = pd - c;
+                        *o = args.accumulate ? *o + x : x;
+                        o += ldo;
+                    }
+                }
+            }
         }
     }
 
@@ -383,6 +439,8 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
     f.ntiles = (a.n + BM - 1) / BM;
     f.nst = (int)((a.nbits + KBITS - 1) / KBITS);
     f.qbytes = (size_t)BN * f.nst * (KBITS / 32) * 16;
+    static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
+    f.trace = trace ? 1 : 0;
     const size_t smem = smem_bytes(BN, a.nbits);
 
     EncodeTiledFn enc = encode_fn();
@@ -393,7 +451,7 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
     const cuuint32_t box[2] = {KBITS / 32, BM};
     const cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(a.B), dims, strides, box, estr,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
 
@@ -401,8 +459,12 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
                                                    : a.op == 1 ? fastid_tc4_kernel<BN, 1>
                                                    : a.op == 2 ? fastid_tc4_kernel<BN, 2>
                                                                : fastid_tc4_kernel<BN, 3>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
+    static size_t attr_set[4] = {0, 0, 0, 0};   // max dynamic smem already granted, per op kernel
+    if (attr_set[a.op & 3] < smem) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)MAX_SMEM);
+        if (e != cudaSuccess) return e;
+        attr_set[a.op & 3] = MAX_SMEM;
+    }
     const int grid = (int)(f.ntiles < num_sms() ? f.ntiles : num_sms());
     kern<<<grid, NTHREADS, smem, s>>>(tm, f);
     count_launches(1);
@@ -414,15 +476,22 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
 // Shape filter: queries on the column side (<= 128 rows, the user's first operand),
 // their whole expanded K range resident in shared memory, exact fp32 range.
 bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
-    if (m < 1 || m > 128 || n < 1 || nbits < 1 || nbits >= (1LL << 24)) return false;
+    if (m < 1 || m > 64 || n < 1 || nbits < 1 || nbits >= (1LL << 24)) return false;
     if (n < 4 * m) return false;
     if (n > (int64_t)0x7fffffff - BM) return false;
-    return smem_bytes(m <= 64 ? 64 : 128, nbits) <= MAX_SMEM;
+    return smem_bytes(64, nbits) <= MAX_SMEM;
 }
 
 cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     if (epi != EPI_COUNTS) return cudaErrorNotSupported;
-    return a.m <= 64 ? launch_f<64>(a, s) : launch_f<128>(a, s);
+    return launch_f<64>(a, s);   // queries <= 64 (fastid_tc4_supported)
 }
 
 }  // namespace snp
+
+// Profiling aid (not part of include/snp.h): copy the pipeline trace of the last
+// traced fastid_tc4 launch (4 x 1024 clock64 stamps) to host memory.
+extern "C" int snp_debug_fastid_trace(long long *host, int n) {
+    if (n > 8 * 1024) n = 8 * 1024;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_trace, sizeof(long long) * n);
+}

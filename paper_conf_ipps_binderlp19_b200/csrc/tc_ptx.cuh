@@ -168,6 +168,37 @@ __device__ __forceinline__ void mma4_mxf4_ts_commit(uint32_t d, uint32_t a0, uin
         "r"(idesc), "r"(sfa), "r"(sfb), "r"(smem_u32(bar))
         : "memory");
 }
+// Eight K-steps (K = 512 nibbles) of tcgen05.mma kind::mxf4 with A from TMEM (columns
+// a0 + 8 i) and B descriptors b0 + i * bstep, then a commit to `bar`; one elected lane.
+__device__ __forceinline__ void mma8_mxf4_ts_commit(uint32_t d, uint32_t a0, uint64_t b0, uint32_t bstep,
+                                                    uint32_t idesc, uint32_t accumulate, uint32_t sfa,
+                                                    uint32_t sfb, uint64_t *bar) {
+    asm volatile(
+        "{\n\t.reg .pred e, p, t;\n\t.reg .b64 bd;\n\t.reg .b32 ad;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "setp.ne.b32 p, %5, 0;\n\t"
+        "setp.eq.b32 t, 0, 0;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %4, [%6], [%7], p;\n\t"
+        "add.u32 ad, %1, 8;  add.u64 bd, %2, %3;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [ad], bd, %4, [%6], [%7], t;\n\t"
+        "add.u32 ad, ad, 8;  add.u64 bd, bd, %3;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [ad], bd, %4, [%6], [%7], t;\n\t"
+        "add.u32 ad, ad, 8;  add.u64 bd, bd, %3;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [ad], bd, %4, [%6], [%7], t;\n\t"
+        "add.u32 ad, ad, 8;  add.u64 bd, bd, %3;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [ad], bd, %4, [%6], [%7], t;\n\t"
+        "add.u32 ad, ad, 8;  add.u64 bd, bd, %3;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [ad], bd, %4, [%6], [%7], t;\n\t"
+        "add.u32 ad, ad, 8;  add.u64 bd, bd, %3;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [ad], bd, %4, [%6], [%7], t;\n\t"
+        "add.u32 ad, ad, 8;  add.u64 bd, bd, %3;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [ad], bd, %4, [%6], [%7], t;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%8];\n\t}" ::"r"(d),
+        "r"(a0), "l"(b0), "l"((uint64_t)bstep), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb),
+        "r"(smem_u32(bar))
+        : "memory");
+}
+
 // Commit by one elected lane of a converged warp.
 __device__ __forceinline__ void mma_commit_elect(uint64_t *bar) {
     asm volatile(

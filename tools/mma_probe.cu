@@ -21,7 +21,8 @@ __device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a, uint64_t b, 
                  :: "r"(d), "r"(a), "l"(b), "r"(idesc), "r"(acc), "r"(sfa), "r"(sfb));
 }
 
-template <int MODE, int N>   // MODE 0: mxf4 SS, 1: mxf4 TS, 2: i8 SS, 3: i8 TS
+template <int MODE, int N, int CONTEND = 0>   // MODE 0: mxf4 SS, 1: mxf4 TS, 2: i8 SS, 3: i8 TS
+// CONTEND 1: warps 1-4 hammer tcgen05.st into other TMEM columns; 2: tcgen05.ld
 __global__ void probe(int iters, long long *out) {
     extern __shared__ __align__(1024) uint8_t sm[];
     __shared__ uint64_t bar;
@@ -45,21 +46,29 @@ __global__ void probe(int iters, long long *out) {
         ptx::mbar_wait(&bar, 0);
         long long t1 = clock64();
         out[blockIdx.x] = t1 - t0;
+    } else if (CONTEND && threadIdx.x >= 32 && threadIdx.x < 160) {
+        const int w = threadIdx.x >> 5, q = w & 3;
+        uint32_t v[8] = {1, 2, 3, 4, 5, 6, 7, 8};
+        for (int i = 0; i < iters / 2; ++i) {
+            const uint32_t a = tmem + ((uint32_t)(q * 32) << 16) + 384 + (i & 7) * 8;
+            if (CONTEND == 1) { ptx::tmem_st8(a, v); ptx::tmem_st_wait(); }
+            else { ptx::tmem_ld8(a, v); ptx::tmem_ld_wait(); }
+        }
     }
     ptx::tc_fence_before(); __syncthreads();
     if (threadIdx.x < 32) { ptx::tc_fence_after(); ptx::tmem_dealloc<512>(tmem); }
 }
 
-template <int MODE, int N>
+template <int MODE, int N, int CONTEND = 0>
 void run(const char *name) {
     long long *d; cudaMalloc(&d, 148 * sizeof(long long));
     const int iters = 4096;
-    auto k = probe<MODE, N>;
+    auto k = probe<MODE, N, CONTEND>;
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-    k<<<148, 128, 64 * 1024>>>(iters, d);
+    k<<<148, 192, 64 * 1024>>>(iters, d);
     cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
     cudaEventRecord(e0);
-    k<<<148, 128, 64 * 1024>>>(iters, d);
+    k<<<148, 192, 64 * 1024>>>(iters, d);
     cudaEventRecord(e1); cudaEventSynchronize(e1);
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     long long h[148]; cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
@@ -77,5 +86,7 @@ int main() {
     run<1, 64>("mxf4 TS"); run<1, 128>("mxf4 TS"); run<1, 256>("mxf4 TS");
     run<2, 64>("i8 SS"); run<2, 128>("i8 SS"); run<2, 256>("i8 SS");
     run<3, 64>("i8 TS"); run<3, 128>("i8 TS"); run<3, 256>("i8 TS");
+    run<1, 64, 1>("mxf4 TS +st"); run<1, 128, 1>("mxf4 TS +st"); run<0, 64, 1>("mxf4 SS +st");
+    run<1, 64, 2>("mxf4 TS +ld"); run<0, 64, 2>("mxf4 SS +ld");
     return 0;
 }
