@@ -54,6 +54,8 @@ def parse():
     p.add_argument("--variant", default="auto", choices=["auto", "popc", "tc"])
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-graph", dest="graph", action="store_false",
+                   help="run the timed steps eagerly instead of replaying a captured CUDA graph")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target oracle CPU time")
     a = p.parse_args()
     if a.warmup < 3:
@@ -291,10 +293,19 @@ def setup_fastid(wl, rank, world, dev):
                 res_host[op][0].copy_(bc, non_blocking=True)
                 res_host[op][1].copy_(bi, non_blocking=True)
 
+    # the same device-resident step as separately capturable parts (N=1 graph mode)
+    def _fast(op):
+        return lambda: snp.snp_fastid(Q, D, nbits, op, out=outs[op], ws=ws[op] if ws[op].numel() else None)
+
+    def _best(op):
+        return lambda: snp.snp_fastid_best(outs[op], index_base=lo, best_count=best[op][0], best_index=best[op][1])
+    parts = [(lambda: snp.snp_pack(qbytes, nbits=nbits, out=Q), False),
+             (_fast("xor"), True), (_best("xor"), False), (_fast("andnot"), True), (_best("andnot"), False)]
+
     # algorithmic bytes of the dominant kernel per launch: DB + queries read, counts written
     words = (nbits + 63) // 64
     alg_bytes = (nd + nq) * words * 8 + nq * nd * 4
-    return dict(step=step, cmp_rank=cmp_rank, cmp_all=cmp_all, kernel_launches_per_step=2,
+    return dict(step=step, parts=parts, cmp_rank=cmp_rank, cmp_all=cmp_all, kernel_launches_per_step=2,
                 kernel_cmp=nq * nd * nbits, kernel_bytes=alg_bytes,
                 h2d=nq * nbits, d2h=2 * nq * 12, l2_flush=False,
                 l2_note=f"inputs larger than L2 ({nd * snp.snp_words(nbits) * 8 / 1e6:.0f} MB database per rank)",
@@ -347,8 +358,11 @@ def setup_ld(wl, rank, world, dev):
     def l2flush():
         flush.add_(1)
 
+    parts = [(lambda: snp.snp_pack(G, nbits=nbits, out=B), False),
+             (lambda: snp.snp_ld_r2(B[lo:hi], B, nbits, r2=r2, counts=cnt, ws=ws), True)] if rank == 0 else None
+
     alg_bytes = (rows + m) * words * 8 + rows * m * 8
-    return dict(step=step, cmp_rank=rows * m * nbits, cmp_all=m * m * nbits, kernel_launches_per_step=1,
+    return dict(step=step, parts=parts, cmp_rank=rows * m * nbits, cmp_all=m * m * nbits, kernel_launches_per_step=1,
                 kernel_cmp=rows * m * nbits, kernel_bytes=alg_bytes, h2d=(m * nbits if rank == 0 else 0),
                 d2h=4, l2_flush=True, flush=l2flush,
                 l2_note="L2 flushed (256 MB write) between timed steps, outside the per-step events",
@@ -357,24 +371,42 @@ def setup_ld(wl, rank, world, dev):
 
 # ----------------------------------------------------------------------------- main timing
 
-def timed(wlrun, steps, host, world, kernel_events=True):
-    """Time `steps` steps; returns (total_ms max over ranks, per-kernel mean ms)."""
+def timed(wlrun, steps, host, world, kernel_events=True, graph=None):
+    """Time `steps` steps; returns (total_ms max over ranks, per-kernel mean ms).
+
+    With `graph` (a captured CUDA graph of one step, N=1) each step is one graph
+    replay, so the device time excludes Python/launch overhead; the per-kernel
+    events were captured inside the graph.  Without it the step runs eagerly."""
     import torch
     s = torch.cuda.current_stream()
     nk = 2 * wlrun["kernel_launches_per_step"]
     kevs = [[torch.cuda.Event(enable_timing=True) for _ in range(nk)] for _ in range(steps)]
     sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+
+    def one(i):
+        if graph is not None:
+            j = 0
+            for g, is_kernel in graph["parts"]:
+                if is_kernel and kernel_events:
+                    kevs[i][j].record(s)
+                g.replay()
+                if is_kernel and kernel_events:
+                    kevs[i][j + 1].record(s)
+                    j += 2
+        else:
+            wlrun["step"](kevs[i] if kernel_events else None, host)
+
     barrier(world)
     if wlrun["l2_flush"]:
         for i in range(steps):
             wlrun["flush"]()
             sev[i][0].record(s)
-            wlrun["step"](kevs[i] if kernel_events else None, host)
+            one(i)
             sev[i][1].record(s)
     else:
         sev[0][0].record(s)
         for i in range(steps):
-            wlrun["step"](kevs[i] if kernel_events else None, host)
+            one(i)
         sev[-1][1].record(s)
     torch.cuda.synchronize()
     barrier(world)
@@ -389,6 +421,29 @@ def timed(wlrun, steps, host, world, kernel_events=True):
                 kms.append(ev[j].elapsed_time(ev[j + 1]))
     total = max_over_ranks(total, world)
     return total, (statistics.mean(kms) if kms else None)
+
+
+def capture(wlrun):
+    """Capture every part of one device-resident step in its own CUDA graph (N=1).
+
+    Replaying part by part keeps host overhead out of the device timing while the
+    per-kernel CUDA events stay on the launching stream between replays."""
+    import torch
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        for fn, _ in wlrun["parts"]:
+            fn()                                   # warm the capture stream
+    torch.cuda.current_stream().wait_stream(side)
+    torch.cuda.synchronize()
+    graphs = []
+    for fn, is_kernel in wlrun["parts"]:
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            fn()
+        graphs.append((g, is_kernel))
+    torch.cuda.synchronize()
+    return {"parts": graphs}
 
 
 def run_ours(args):
@@ -408,10 +463,22 @@ def run_ours(args):
     for _ in range(args.warmup):
         wlrun["step"](None, False)
     torch.cuda.synchronize()
+    graph = None
+    use_graph = args.graph and world == 1 and wlrun.get("parts") is not None
     n0 = snp.snp_launch_count()
+    if use_graph:
+        graph = capture(wlrun)
+        per_step_launches = snp.snp_launch_count() - n0
+        for _ in range(args.warmup):
+            for g, _ in graph["parts"]:
+                g.replay()
+        torch.cuda.synchronize()
+        n0 = snp.snp_launch_count()
     with ClockSampler(local) as clk:
-        total_ms, kern_ms = timed(wlrun, steps, False, world)
+        total_ms, kern_ms = timed(wlrun, steps, False, world, graph=graph)
     launches = snp.snp_launch_count() - n0
+    if use_graph:
+        launches = per_step_launches * steps     # kernels replayed from the graph
     variant = snp.snp_last_variant()
     ms = total_ms / steps
     value = wlrun["cmp_all"] / (ms / 1e3)
@@ -464,6 +531,7 @@ def run_ours(args):
             "config": {"workload": args.workload, "desc": wl["desc"],
                        **{k: v for k, v in wl.items() if k in ("nq", "nd", "m", "nbits")},
                        "variant": variant, "l2": wlrun["l2_note"],
+                       "launch": "cuda-graph replay per step" if use_graph else "eager",
                        "parallelism": f"{'db' if wl['kind'] == 'fastid' else 'row'}-shard x{world}"},
             "word_ops_per_s": value / 64, "tops_eq": 2 * value / 1e12,
             "roofline": roof, "roofline_hbm": roof_hbm,

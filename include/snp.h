@@ -126,9 +126,11 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
 /* a3 + a4 — FastID comparison counts (Eqs. 2-3):
  *   out[i*ldo + j] (=|+=) sum_k op(Q_ik, D_jk)   for queries i < nq, DB rows j < nd.
  * Q: [nq][ldq] packed query profiles over SNPs, D: [nd][ldd] database profiles.
- * popQ/popD: optional row popcounts (used by the tensor variant's identities
- * XOR = pQ + pD - 2 AND, ANDNOT = pQ - AND, NOTAND = pD - AND; NULL = computed
- * internally).  out: uint32 [nq][ldo], ldo >= nd. */
+ * popQ/popD: optional row popcounts; may be NULL.  Every current variant derives
+ * the popcounts it needs itself (the tensor-core kernels accumulate them from the
+ * packed words they already stream for the identities XOR = pQ + pD - 2 AND,
+ * ANDNOT = pQ - AND, NOTAND = pD - AND), so they are accepted but not read.
+ * out: uint32 [nq][ldo], ldo >= nd. */
 snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t *popQ,
                       const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD,
                       int64_t nbits, int op, uint32_t *out, int64_t ldo, int accumulate,

@@ -31,6 +31,9 @@ namespace snp {
 // clock64 stamps per iteration: [0] expander before waits, [1] after pfull+empty,
 // [2] before full arrive, [3] MMA after full wait.  Enabled by SNP_TRACE=1.
 __device__ long long g_fastid_trace[8 * 1024];
+__device__ long long g_fastid_cta_time[3 * 1024];
+__device__ long long g_fastid_launch_time[2 * 64];   // CTA 0: start / end globaltimer per launch
+__device__ unsigned int g_fastid_launch_ctr;   // per CTA: start, main loop start, end (globaltimer ns)
 
 namespace {
 
@@ -72,6 +75,7 @@ struct FArgs {
     int nst;
     size_t qbytes;       // expanded query bytes in shared memory
     int trace;
+    int nostore;         // profiling experiment: skip the output stores
 };
 
 __device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
@@ -146,6 +150,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     uint32_t *popD = popQ + BN;              // [2 acc][G][BM]
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    __shared__ unsigned int launch_k;
+    if (args.trace && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x] = (long long)ptx::globaltimer_ns();
+    if (args.trace && tid == 0 && blockIdx.x == 0) {
+        launch_k = atomicAdd(&g_fastid_launch_ctr, 1u) & 63u;
+        g_fastid_launch_time[2 * launch_k] = (long long)ptx::globaltimer_ns();
+    }
     const int64_t nbits = args.nbits;
     const int nst = args.nst;
     const int64_t my_tiles = args.ntiles > blockIdx.x ? (args.ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
@@ -205,6 +215,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     __syncthreads();
     ptx::tc_fence_after();
 
+    if (args.trace && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 1] = (long long)ptx::globaltimer_ns();
     if (warp == TMA_WARP) {
         // ------------------------------------------------------------ TMA producer
         if (lane == 0) {
@@ -351,7 +362,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&acce[acc]);   // accumulator + pops drained: reusable
             const int64_t gd = t * BM + li;
-            if (gd < args.nd && ncols > 0) {
+            if (gd < args.nd && ncols > 0 && !args.nostore) {
                 uint32_t *o = args.out + (int64_t)c0 * ldo + gd;
                 if (ncols == 32 && !args.accumulate) {
 #pragma unroll
@@ -385,6 +396,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 
     ptx::tc_fence_before();
     __syncthreads();
+    if (args.trace && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 2] = (long long)ptx::globaltimer_ns();
+    if (args.trace && tid == 0 && blockIdx.x == 0) g_fastid_launch_time[2 * launch_k + 1] = (long long)ptx::globaltimer_ns();
     if (warp == MMA_WARP) {
         ptx::tc_fence_after();
         ptx::tmem_dealloc<512>(tmem);
@@ -441,6 +454,8 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
     f.qbytes = (size_t)BN * f.nst * (KBITS / 32) * 16;
     static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
     f.trace = trace ? 1 : 0;
+    static const bool nostore = std::getenv("SNP_DEBUG_NOSTORE") && std::getenv("SNP_DEBUG_NOSTORE")[0] == '1';
+    f.nostore = nostore ? 1 : 0;
     const size_t smem = smem_bytes(BN, a.nbits);
 
     EncodeTiledFn enc = encode_fn();
@@ -461,9 +476,10 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
                                                                : fastid_tc4_kernel<BN, 3>;
     static size_t attr_set[4] = {0, 0, 0, 0};   // max dynamic smem already granted, per op kernel
     if (attr_set[a.op & 3] < smem) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)MAX_SMEM);
+        const size_t grant = MAX_SMEM - 1024;   // leave room for the kernel's static shared memory
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)grant);
         if (e != cudaSuccess) return e;
-        attr_set[a.op & 3] = MAX_SMEM;
+        attr_set[a.op & 3] = grant;
     }
     const int grid = (int)(f.ntiles < num_sms() ? f.ntiles : num_sms());
     kern<<<grid, NTHREADS, smem, s>>>(tm, f);
@@ -479,7 +495,7 @@ bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
     if (m < 1 || m > 64 || n < 1 || nbits < 1 || nbits >= (1LL << 24)) return false;
     if (n < 4 * m) return false;
     if (n > (int64_t)0x7fffffff - BM) return false;
-    return smem_bytes(64, nbits) <= MAX_SMEM;
+    return smem_bytes(64, nbits) <= MAX_SMEM - 1024;
 }
 
 cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
@@ -491,6 +507,16 @@ cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
 
 // Profiling aid (not part of include/snp.h): copy the pipeline trace of the last
 // traced fastid_tc4 launch (4 x 1024 clock64 stamps) to host memory.
+extern "C" int snp_debug_fastid_launch_times(long long *host, int n) {
+    if (n > 128) n = 128;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_launch_time, sizeof(long long) * n);
+}
+
+extern "C" int snp_debug_fastid_cta_times(long long *host, int n) {
+    if (n > 3 * 1024) n = 3 * 1024;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_cta_time, sizeof(long long) * n);
+}
+
 extern "C" int snp_debug_fastid_trace(long long *host, int n) {
     if (n > 8 * 1024) n = 8 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_trace, sizeof(long long) * n);

@@ -147,7 +147,7 @@ size_t snp_fastid_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op)
     (void)op;
     if (nq <= 0 || nd <= 0 || nbits <= 0) return 0;
     if (choose_variant(nq, nd, nbits) != SNP_VARIANT_TC) return 0;
-    return pops_bytes(nq, nd) + tc_workspace_bytes(nq, nd, nbits);
+    return tc_workspace_bytes(nq, nd, nbits);
 }
 
 snp_status snp_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg_bytes,
@@ -226,11 +226,13 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
     uint32_t *pa = reinterpret_cast<uint32_t *>(ws);
     uint32_t *pb = reinterpret_cast<uint32_t *>((char *)ws + align256((size_t)m * 4));
     cudaError_t e;
-    if (!popA) {
+    // the CUDA-core variant reads row popcounts; the tensor-core kernels compute them
+    // from the packed words they stream, so no pre-pass is launched for them
+    if (variant != SNP_VARIANT_TC && !popA) {
         if ((e = launch_row_popc(A, m, nbits, lda, pa, s)) != cudaSuccess) return set_cuda_error(e);
         popA = pa;
     }
-    if (!popB) {
+    if (variant != SNP_VARIANT_TC && !popB) {
         if ((e = launch_row_popc(B, n, nbits, ldb, pb, s)) != cudaSuccess) return set_cuda_error(e);
         popB = pb;
     }
@@ -270,20 +272,9 @@ snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t
     a.m = nq; a.n = nd; a.lda32 = 2 * ldq; a.ldb32 = 2 * ldd; a.nbits = nbits;
     a.op = op; a.accumulate = accumulate ? 1 : 0; a.ldc = ldo; a.C = out;
     if (variant == SNP_VARIANT_TC) {
-        uint32_t *pq = reinterpret_cast<uint32_t *>(ws);
-        uint32_t *pd = reinterpret_cast<uint32_t *>((char *)ws + align256((size_t)nq * 4));
-        cudaError_t e;
-        if (op != SNP_OP_AND && !popQ) {
-            if ((e = launch_row_popc(Q, nq, nbits, ldq, pq, s)) != cudaSuccess) return set_cuda_error(e);
-            popQ = pq;
-        }
-        if ((op == SNP_OP_XOR || op == SNP_OP_NOTAND) && !popD) {
-            if ((e = launch_row_popc(D, nd, nbits, ldd, pd, s)) != cudaSuccess) return set_cuda_error(e);
-            popD = pd;
-        }
-        a.popA = popQ; a.popB = popD;
-        return run_gemm(a, EPI_COUNTS, variant, (char *)ws + pops_bytes(nq, nd),
-                        ws_bytes - pops_bytes(nq, nd), s);
+        // every tensor-core kernel accumulates both operands' popcounts from the packed
+        // words it streams (no extra pass over the database); popQ/popD are not needed
+        return run_gemm(a, EPI_COUNTS, variant, ws, ws_bytes, s);
     }
     return run_gemm(a, EPI_COUNTS, variant, nullptr, 0, s);
 }

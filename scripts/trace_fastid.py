@@ -37,3 +37,44 @@ print("expander wait: median", np.median(t[v, 1] - t[v, 0]))
 print("full arrive -> MMA issue: median", np.median(t[v, 3] - t[v, 2]))
 print("MMA: fence", np.median(t[v, 4] - t[v, 3]), "asm", np.median(t[v, 5] - t[v, 4]),
       "asm-end -> next full-wait-done", np.median(t[9:nit, 3] - t[8:nit - 1, 5]))
+
+ct = (ctypes.c_longlong * (3 * 148))()
+snp.lib().snp_debug_fastid_cta_times(ct, 3 * 148)
+c = np.array(ct, dtype=np.int64).reshape(148, 3)
+st = c[:, 0].min()
+print("CTA start spread (us):", (c[:, 0].max() - st) / 1e3, " prologue median (us):", np.median(c[:, 1] - c[:, 0]) / 1e3)
+print("CTA end (us) min/median/max:", (c[:, 2].min() - st) / 1e3, np.median(c[:, 2] - st) / 1e3, (c[:, 2].max() - st) / 1e3)
+ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+ev0.record(); snp.snp_fastid(Q, D, nbits, "xor", out=out); ev1.record(); torch.cuda.synchronize()
+print("event-timed single call (ms):", ev0.elapsed_time(ev1))
+# timing methodology check
+g = torch.cuda.CUDAGraph()
+side = torch.cuda.Stream(); side.wait_stream(torch.cuda.current_stream())
+with torch.cuda.stream(side):
+    snp.snp_fastid(Q, D, nbits, "xor", out=out)
+torch.cuda.current_stream().wait_stream(side); torch.cuda.synchronize()
+with torch.cuda.graph(g):
+    snp.snp_fastid(Q, D, nbits, "xor", out=out)
+for _ in range(3): g.replay()
+torch.cuda.synchronize()
+ev0.record()
+for _ in range(20): g.replay()
+ev1.record(); torch.cuda.synchronize()
+print("20 back-to-back graph replays: per call (ms)", ev0.elapsed_time(ev1) / 20)
+ev0.record()
+for _ in range(20): snp.snp_fastid(Q, D, nbits, "xor", out=out)
+ev1.record(); torch.cuda.synchronize()
+print("20 back-to-back eager calls: per call (ms)", ev0.elapsed_time(ev1) / 20)
+evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(20)]
+for a, b in evs:
+    a.record(); g.replay(); b.record()
+torch.cuda.synchronize()
+print("per-replay events (ms):", [round(a.elapsed_time(b), 4) for a, b in evs][:10])
+
+lt = (ctypes.c_longlong * 128)()
+snp.lib().snp_debug_fastid_launch_times(lt, 128)
+L = np.array(lt, dtype=np.int64).reshape(64, 2)
+L = L[L[:, 0] > 0]
+L = L[np.argsort(L[:, 0])]
+print("last launches: CTA0 run (us)", ((L[-8:, 1] - L[-8:, 0]) / 1e3).round(1).tolist())
+print("              gap to next start (us)", ((L[-7:, 0] - L[-8:-1, 1]) / 1e3).round(1).tolist())
