@@ -84,6 +84,8 @@ def load_peaks():
         "popc_tops": 2 * 148 * 16 * 32 * sm_mhz * 1e6 / 1e12,
         # int8 tensor: measured bf16 dense x nominal i8:bf16 ratio 2 (4.5 vs 2.25 PF spec).
         "i8_tops": 2.0 * float(pk["bf16_tflops"]),
+        # fp4 (kind::mxf4) tensor: measured bf16 dense x nominal fp4:bf16 ratio 4 (9 vs 2.25 PF).
+        "f4_tops": 4.0 * float(pk["bf16_tflops"]),
         "i8_tops_sustained": 2.0 * float(pk.get("bf16_tflops_sustained", pk["bf16_tflops"])),
         "sm_max_mhz": sm_mhz,
     }
@@ -480,6 +482,7 @@ def run_ours(args):
     if use_graph:
         launches = per_step_launches * steps     # kernels replayed from the graph
     variant = snp.snp_last_variant()
+    kernel = snp.snp_last_kernel()
     ms = total_ms / steps
     value = wlrun["cmp_all"] / (ms / 1e3)
 
@@ -496,27 +499,37 @@ def run_ours(args):
     # roofline of the dominant kernel (the bit-GEMM launch), live CUDA-event durations
     kcmp = wlrun["kernel_cmp"]
     tops = 2 * kcmp / (kern_ms / 1e3) / 1e12
-    if variant == "tc":
+    if kernel in ("tc_mxf4", "fastid_mxf4"):
+        roof = {"bound": "tensor", "achieved": tops, "peak": peaks["f4_tops"], "unit": "TOPS",
+                "peak_src": f"fp4 dense = 4 x bf16 burst ({peaks['src']} MEASURED_PEAKS.json)"}
+    elif kernel == "tc_i8":
         roof = {"bound": "tensor", "achieved": tops, "peak": peaks["i8_tops"], "unit": "TOPS",
-                "peak_src": f"int8 = 2 x bf16 burst ({peaks['src']} MEASURED_PEAKS.json)"}
+                "peak_src": f"int8 dense = 2 x bf16 burst ({peaks['src']} MEASURED_PEAKS.json)"}
     else:
         roof = {"bound": "alu", "achieved": tops, "peak": peaks["popc_tops"], "unit": "TOPS",
                 "peak_src": "POPC pipe: 148 SM x 16/clk x 32 bit x 1965 MHz (DESIGN.md §6)"}
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["kernel_ms"] = kern_ms
-    roof["traffic"] = None
+    roof["kernel"] = kernel
+    traffic = None   # dram bytes read+write per launch from one ncu --set full capture (profiles/)
     prof = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(prof):
         try:
             with open(prof) as f:
-                tr = json.load(f).get(f"{args.workload}:{variant}")
-            if tr:
-                roof["traffic"] = tr
+                traffic = json.load(f).get(f"{args.workload}:{kernel}")
         except Exception:
-            pass
+            traffic = None
     hbm_gbs = wlrun["kernel_bytes"] / (kern_ms / 1e3) / 1e9
-    roof_hbm = {"achieved": hbm_gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": hbm_gbs / peaks["hbm_gbs"], "alg_bytes": wlrun["kernel_bytes"]}
+    roof_hbm = {"bound": "hbm", "achieved": hbm_gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": hbm_gbs / peaks["hbm_gbs"], "alg_bytes_per_launch": wlrun["kernel_bytes"],
+                "kernel_ms": kern_ms, "kernel": kernel, "peak_src": f"{peaks['src']} MEASURED_PEAKS.json copy"}
+    roof["traffic"] = roof_hbm["traffic"] = traffic
+    roof["alg_cmp_per_launch"] = wlrun["kernel_cmp"]
+    # north_star: LD against the chosen pipe's peak, FastID against HBM bandwidth
+    if wl["kind"] == "fastid":
+        roof_primary, roof_secondary = roof_hbm, roof
+    else:
+        roof_primary, roof_secondary = roof, roof_hbm
 
     out = None
     if rank == 0:
@@ -530,11 +543,11 @@ def run_ours(args):
             "data": "synthetic (seeded counter-based genotype generator, MAF ~ U[0.05,0.5))",
             "config": {"workload": args.workload, "desc": wl["desc"],
                        **{k: v for k, v in wl.items() if k in ("nq", "nd", "m", "nbits")},
-                       "variant": variant, "l2": wlrun["l2_note"],
+                       "variant": variant, "kernel": kernel, "l2": wlrun["l2_note"],
                        "launch": "cuda-graph replay per step" if use_graph else "eager",
                        "parallelism": f"{'db' if wl['kind'] == 'fastid' else 'row'}-shard x{world}"},
             "word_ops_per_s": value / 64, "tops_eq": 2 * value / 1e12,
-            "roofline": roof, "roofline_hbm": roof_hbm,
+            "roofline": roof_primary, "roofline_secondary": roof_secondary,
             "gpu_launches": launches,
             "clocks": clk.summary(),
             "e2e": e2e,

@@ -158,6 +158,16 @@ snp_status snp_set_variant(int variant);
 /* Variant used by the most recent successful compute call on this thread. */
 int snp_last_variant(void);
 
+/* Kernel family behind that variant (evidence for benchmarks and tests). */
+typedef enum {
+    SNP_KERNEL_NONE = 0,
+    SNP_KERNEL_POPC = 1,        /* CUDA-core LOP3 + POPC                          */
+    SNP_KERNEL_TC_I8 = 2,       /* tcgen05 kind::i8 on u8-expanded operands        */
+    SNP_KERNEL_TC_MXF4 = 3,     /* tcgen05 kind::mxf4 on e2m1-expanded operands    */
+    SNP_KERNEL_FASTID_MXF4 = 4  /* kind::mxf4, resident queries, TMA-streamed DB   */
+} snp_kernel;
+int snp_last_kernel(void);
+
 /* Cumulative number of CUDA kernels this library has launched in this process
  * (evidence for benchmarks: every launch is one of the library's own kernels). */
 int64_t snp_launch_count(void);

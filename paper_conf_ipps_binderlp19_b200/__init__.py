@@ -21,7 +21,7 @@ __all__ = [
     "SnpError", "OPS", "VARIANTS", "snp_words", "snp_ld_workspace_bytes",
     "snp_fastid_workspace_bytes", "snp_pack", "snp_row_popc", "snp_ld_counts",
     "snp_ld_r2", "snp_fastid", "snp_fastid_best", "snp_shard_plan", "snp_set_variant",
-    "snp_last_variant", "snp_launch_count", "status_string",
+    "snp_last_variant", "snp_last_kernel", "snp_launch_count", "status_string",
 ]
 
 OPS = {"and": 0, "xor": 1, "andnot": 2, "notand": 3}
@@ -217,6 +217,14 @@ def snp_set_variant(variant) -> None:
 def snp_launch_count() -> int:
     """Cumulative number of kernels libsnp.so launched in this process."""
     return int(lib().snp_launch_count())
+
+
+KERNELS = {0: "none", 1: "popc", 2: "tc_i8", 3: "tc_mxf4", 4: "fastid_mxf4"}
+
+
+def snp_last_kernel() -> str:
+    """Kernel family of the most recent compute call on this thread."""
+    return KERNELS.get(int(lib().snp_last_kernel()), "?")
 
 
 def snp_last_variant() -> str:

@@ -28,6 +28,7 @@ SIGNATURES = {
     "snp_set_variant": (_int, [_int]),
     "snp_last_variant": (_int, []),
     "snp_launch_count": (_i64, []),
+    "snp_last_kernel": (_int, []),
     "snp_status_string": (ctypes.c_char_p, [_int]),
     "snp_last_cuda_error": (ctypes.c_char_p, []),
 }

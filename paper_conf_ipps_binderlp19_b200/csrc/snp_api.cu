@@ -15,6 +15,7 @@ namespace {
 
 thread_local char g_cuda_err[256] = "";
 thread_local int g_last_variant = 0;
+thread_local int g_last_kernel = 0;
 
 std::atomic<int> g_variant{-1};   // -1: not yet read from the environment
 std::atomic<long long> g_launches{0};
@@ -109,14 +110,19 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
         const bool want_i8 = kind && !std::strcmp(kind, "i8");
         const char *ff = std::getenv("SNP_FASTID_KERNEL");
         const bool no_fastid = ff && !std::strcmp(ff, "0");
-        if (!want_i8 && !no_fastid && epi == EPI_COUNTS && fastid_tc4_supported(a.m, a.n, a.nbits))
+        if (!want_i8 && !no_fastid && epi == EPI_COUNTS && fastid_tc4_supported(a.m, a.n, a.nbits)) {
             e = launch_fastid_tc4(a, epi, s);
-        else if (!want_i8 && tc4_supported(a.m, a.n, a.nbits))
+            g_last_kernel = SNP_KERNEL_FASTID_MXF4;
+        } else if (!want_i8 && tc4_supported(a.m, a.n, a.nbits)) {
             e = launch_bitgemm_tc4(a, epi, s);
-        else
+            g_last_kernel = SNP_KERNEL_TC_MXF4;
+        } else {
             e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
+            g_last_kernel = SNP_KERNEL_TC_I8;
+        }
     } else {
         e = launch_bitgemm_popc(a, epi, s);
+        g_last_kernel = SNP_KERNEL_POPC;
     }
     if (e != cudaSuccess) return set_cuda_error(e);
     g_last_variant = variant;
@@ -319,6 +325,8 @@ snp_status snp_set_variant(int variant) {
 }
 
 int snp_last_variant(void) { return g_last_variant; }
+
+int snp_last_kernel(void) { return g_last_kernel; }
 
 int64_t snp_launch_count(void) { return (int64_t)g_launches.load(); }
 
