@@ -1,0 +1,520 @@
+// gemm_tc4.cu — general tensor-core bit-GEMM (LD all pairs, FastID with many queries):
+//
+//   C[i][j] = sum_k A_ik & B_jk        (Eq. 1; GEMM form P:L116)
+//   + fused epilogue: counts / FastID op identities / LD r2, D' (a5)
+//
+// Bits become e2m1 nibbles (1 -> 1.0) and are multiplied with tcgen05.mma kind::mxf4
+// (scale factors 2^0, exact fp32 sums below 2^24; see bitgemm_tc4.cu / DESIGN.md §6).
+// 128 x 128 output tiles, persistent CTAs (one per SM), K in 512-bit stages.
+//
+// Per stage, for the 128 lane rows (A) and 128 column rows (B) of the tile:
+//   TMA warp      one 2-D TMA load per operand (128 rows x 64 B, 64B-swizzled) into
+//                 the packed ring slot of the stage;
+//   expander group g (stages it = g mod 3; 4 warps, one per TMEM lane quarter):
+//                 LDS the packed rows, accumulate row popcounts, expand each 32-bit word
+//                 to four words of nibbles (shifts on the FMA pipe via IMAD.HI), write A
+//                 into TMEM (tcgen05.st; MMA operand A from TMEM) and B into the stage's
+//                 K-major no-swizzle shared-memory operand;
+//   MMA warp      8 x tcgen05.mma (M = N = 128, K = 64) from one elected lane, commit;
+//   8 epilogue warps  drain the other TMEM accumulator (double-buffered), apply the
+//                 identity / LD statistic, store.
+// Resource plan: TMEM 2 x 128 accumulator + 3 x 64 A-stage + 32 scale-factor columns;
+// shared memory 3 x 16 KB packed + 3 x 32 KB expanded B + barriers/popcounts.
+#include "snp_internal.h"
+#include "tc_ptx.cuh"
+
+#include <cuda.h>
+#include <cstdlib>
+
+namespace snp {
+namespace {
+
+constexpr int BM = 128, BN = 128;
+constexpr int KBITS = 512;
+constexpr int KW = KBITS / 32;                 // 16 packed words per row per stage
+constexpr int G = 3;                           // expander groups == stage slots
+constexpr int NEXP = 4 * G;                    // 12 expander warps
+constexpr int NEPI = 8;
+constexpr int EPI_WARP0 = NEXP;                // 12..19
+constexpr int TMA_WARP = NEXP + NEPI;          // 20
+constexpr int MMA_WARP = NEXP + NEPI + 1;      // 21 (highest id: scheduler priority)
+constexpr int NTHREADS = (NEXP + NEPI + 2) * 32;
+constexpr int PROW = KBITS / 8;                // 64 packed bytes per row per stage
+constexpr int PSLOT = (BM + BN) * PROW;        // 16 KB packed per slot (A then B)
+constexpr int BSLOT = BN * KBITS / 2;          // 32 KB expanded B per slot
+constexpr int ACC_COLS = BN;
+constexpr int A_COL0 = 2 * ACC_COLS;           // 256
+constexpr int SF_COL = A_COL0 + G * 64;        // 448
+static_assert(SF_COL + 32 <= 512, "TMEM budget");
+constexpr int NPB = 4;                         // popcount buffers (tiles in flight)
+constexpr size_t SMEM = (size_t)G * PSLOT + (size_t)G * BSLOT + 16384;
+
+struct GArgs {
+    int64_t nl, nc, nbits;
+    int swap, op, accumulate;
+    int64_t ldo;
+    uint32_t *C;
+    float *r2, *dprime;
+    int64_t nlb, ncb;
+    int nst;
+};
+
+__device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
+    const int64_t lo = w * 32;
+    if (lo + 32 <= nbits) return 0xffffffffu;
+    if (lo >= nbits) return 0u;
+    return (1u << (uint32_t)(nbits - lo)) - 1u;
+}
+
+// 32 bits -> 4 words of 8 e2m1 nibbles (1.0 = 0b0010 where the bit is set); nibble n of
+// output t holds bit 4n + t.  The two right shifts run on the FMA pipe (IMAD.HI).
+__device__ __forceinline__ void expand4(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
+    const uint32_t M = 0x22222222u;
+    o0 = (x << 1) & M;
+    o1 = x & M;
+    o2 = __umulhi(x, 0x80000000u) & M;   // x >> 1
+    o3 = __umulhi(x, 0x40000000u) & M;   // x >> 2
+}
+
+__host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
+    return (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+        "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
+        "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]),
+        "r"(v[17]), "r"(v[18]), "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]),
+        "r"(v[25]), "r"(v[26]), "r"(v[27]), "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
+        : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+        "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
+          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+        : "r"(taddr));
+}
+
+// LD statistics in fp32 from exact integers (reading R3).  num, nA(n-nA), nB(n-nB) are
+// exact integers; each is rounded once to fp32, so r2 and D' carry a relative error of
+// a few 2^-24 (< 1e-6), and are exactly 0 where the exact value is 0.
+__device__ __forceinline__ void ld_stats_f32(int64_t n, int64_t na, int64_t nb, int64_t nab, float &r2,
+                                             float &dp) {
+    const int64_t num = n * nab - na * nb;
+    const int64_t da = na * (n - na), db = nb * (n - nb);
+    if (num == 0 || da == 0 || db == 0) {
+        r2 = 0.f;
+        dp = 0.f;
+        return;
+    }
+    const float fn = (float)num;
+    r2 = __fdiv_rn(fn, (float)da) * __fdiv_rn(fn, (float)db);
+    int64_t dmax;
+    if (num > 0) {
+        const int64_t x = na * (n - nb), y = (n - na) * nb;
+        dmax = x < y ? x : y;
+    } else {
+        const int64_t x = na * nb, y = (n - na) * (n - nb);
+        dmax = x < y ? x : y;
+    }
+    dp = __fdiv_rn(fn, (float)dmax);
+}
+
+template <int EPI>
+__global__ void __launch_bounds__(NTHREADS, 1)
+gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
+                const GArgs args) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *ring = smem;                                        // [G][PSLOT]
+    uint8_t *bexp = smem + (size_t)G * PSLOT;                    // [G][BSLOT]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(bexp + (size_t)G * BSLOT);
+    uint64_t *pfull = bars;            // [G] TMA -> expanders
+    uint64_t *pempty = pfull + G;      // [G] expanders -> TMA
+    uint64_t *full = pempty + G;       // [G] expanders -> MMA
+    uint64_t *empty = full + G;        // [G] MMA -> expanders
+    uint64_t *accf = empty + G;        // [2]
+    uint64_t *acce = accf + 2;         // [2]
+    uint64_t *popf = acce + 2;         // [NPB] expanders -> epilogue (popcounts of a tile written)
+    uint64_t *popfree = popf + NPB;    // [NPB] epilogue -> expanders (popcount buffer reusable)
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popfree + NPB);
+    uint32_t *popA = tmem_slot + 4;    // [NPB][G][BM]
+    uint32_t *popB = popA + NPB * G * BM;  // [NPB][G][BN]
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int64_t nbits = args.nbits;
+    const int nst = args.nst;
+    const int64_t ntiles = args.nlb * args.ncb;
+    const int64_t my_tiles = ntiles > blockIdx.x ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const int64_t total_it = my_tiles * nst;
+    const int64_t full32 = nbits / 32;
+
+    if (tid == 0) {
+        for (int i = 0; i < G; ++i) {
+            ptx::mbar_init(&pfull[i], 1);
+            ptx::mbar_init(&pempty[i], 4);
+            ptx::mbar_init(&full[i], 4);
+            ptx::mbar_init(&empty[i], 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            ptx::mbar_init(&accf[i], 1);
+            ptx::mbar_init(&acce[i], NEPI);
+        }
+        for (int i = 0; i < NPB; ++i) {
+            ptx::mbar_init(&popf[i], NEXP);
+            ptx::mbar_init(&popfree[i], NEPI);
+        }
+        ptx::fence_mbar_init();
+    }
+    if (warp == TMA_WARP && lane == 0) {
+        ptx::prefetch_tensormap(&tmL);
+        ptx::prefetch_tensormap(&tmC);
+    }
+    if (warp == MMA_WARP) ptx::tmem_alloc<512>(tmem_slot);
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+    if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {
+        const int q = warp & 3;
+        uint32_t v[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = 0x7F7F7F7Fu;   // ue8m0 2^0 in every scale byte
+        tmem_st32(tmem + ((uint32_t)(q * 32) << 16) + SF_COL, v);
+        ptx::tmem_st_wait();
+    }
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::tc_fence_after();
+
+    if (warp == TMA_WARP) {
+        // ------------------------------------------------------------ TMA producer
+        if (lane == 0) {
+            int p = 0;
+            uint32_t round = 0;
+            for (int64_t tl = 0; tl < my_tiles; ++tl) {
+                const int64_t t = blockIdx.x + tl * gridDim.x;
+                const int32_t rl = (int32_t)((t % args.nlb) * BM), rc = (int32_t)((t / args.nlb) * BN);
+                for (int s = 0; s < nst; ++s) {
+                    if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);
+                    ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
+                    ptx::tma_load_2d(ring + p * PSLOT, &tmL, &pfull[p], s * KW, rl);
+                    ptx::tma_load_2d(ring + p * PSLOT + BM * PROW, &tmC, &pfull[p], s * KW, rc);
+                    if (++p == G) { p = 0; ++round; }
+                }
+            }
+        }
+    } else if (warp < NEXP) {
+        // ------------------------------------------------------------ expanders
+        const int g = warp >> 2, q = warp & 3;
+        const int row = q * 32 + lane;                  // A row (TMEM lane) and B row of this thread
+        const int sw = (row >> 1) & 3;                  // TMA 64B swizzle of a 64-byte row
+        uint32_t pa = 0, pb = 0;
+        int64_t cur_tl = 0;
+        auto publish_until = [&](int64_t upto) {
+            for (; cur_tl < upto; ++cur_tl) {
+                const int pbuf = (int)(cur_tl % NPB);
+                if (cur_tl >= NPB) ptx::mbar_wait(&popfree[pbuf], (uint32_t)(((cur_tl / NPB) - 1) & 1));
+                popA[(pbuf * G + g) * BM + row] = pa;
+                popB[(pbuf * G + g) * BN + row] = pb;
+                pa = pb = 0;
+                __syncwarp();
+                if (lane == 0) ptx::mbar_arrive(&popf[pbuf]);
+            }
+        };
+        int64_t tl = g / nst;
+        int s = g % nst;
+        uint32_t round = 0;
+        const uint8_t *srcA = ring + g * PSLOT + row * PROW;
+        const uint8_t *srcB = srcA + BM * PROW;
+        uint8_t *dstB = bexp + (size_t)g * BSLOT + row * 16;
+        const uint32_t tA = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(A_COL0 + 64 * g);
+        for (int64_t it = g; it < total_it; it += G) {
+            publish_until(tl);
+            ptx::mbar_wait(&pfull[g], round & 1);
+            if (round > 0) ptx::mbar_wait(&empty[g], (round - 1) & 1);
+            uint32_t wa[KW], wb[KW];
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const uint4 xa = *reinterpret_cast<const uint4 *>(srcA + ((c ^ sw) << 4));
+                const uint4 xb = *reinterpret_cast<const uint4 *>(srcB + ((c ^ sw) << 4));
+                wa[4 * c] = xa.x; wa[4 * c + 1] = xa.y; wa[4 * c + 2] = xa.z; wa[4 * c + 3] = xa.w;
+                wb[4 * c] = xb.x; wb[4 * c + 1] = xb.y; wb[4 * c + 2] = xb.z; wb[4 * c + 3] = xb.w;
+            }
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&pempty[g]);
+            const int64_t w0 = (int64_t)s * KW;
+            if (w0 + KW > full32) {
+#pragma unroll
+                for (int i = 0; i < KW; ++i) {
+                    const uint32_t mk = word_mask(w0 + i, nbits);
+                    wa[i] &= mk;
+                    wb[i] &= mk;
+                }
+            }
+#pragma unroll
+            for (int i = 0; i < KW; ++i) {
+                pa += __popc(wa[i]);
+                pb += __popc(wb[i]);
+            }
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                uint32_t v[32];
+#pragma unroll
+                for (int i = 0; i < 8; ++i)
+                    expand4(wa[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+                tmem_st32(tA + 32 * h, v);
+            }
+#pragma unroll
+            for (int i = 0; i < KW; ++i) {          // chunk i of the K-major operand = word i
+                uint4 o;
+                expand4(wb[i], o.x, o.y, o.z, o.w);
+                *reinterpret_cast<uint4 *>(dstB + (size_t)i * BN * 16) = o;
+            }
+            ptx::tmem_st_wait();
+            ptx::fence_proxy_async_smem();
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&full[g]);
+            s += G;
+            while (s >= nst) { s -= nst; ++tl; }
+            ++round;
+        }
+        publish_until(my_tiles);
+    } else if (warp == MMA_WARP) {
+        // ------------------------------------------------------------ MMA issuer
+        constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
+        const uint32_t sfa = tmem + SF_COL, sfb = tmem + SF_COL + 16;
+        const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(bexp), BN * 16, 128);
+        constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;
+        int b = 0;
+        uint32_t round = 0;
+        for (int64_t tl = 0; tl < my_tiles; ++tl) {
+            const int acc = (int)(tl & 1);
+            if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            ptx::tc_fence_after();
+            const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS);
+            for (int s = 0; s < nst; ++s) {
+                ptx::mbar_wait(&full[b], round & 1);
+                ptx::tc_fence_after();
+                ptx::mma8_mxf4_ts_commit(d, tmem + (uint32_t)(A_COL0 + 64 * b),
+                                         bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4), BSTEP, IDESC,
+                                         s != 0 ? 1u : 0u, sfa, sfb, &empty[b]);
+                if (++b == G) { b = 0; ++round; }
+            }
+            ptx::mma_commit_elect(&accf[acc]);
+        }
+        __syncwarp();
+    } else {
+        // ------------------------------------------------------------ epilogue (8 warps)
+        const int e = warp - EPI_WARP0;
+        const int q = e & 3, h = e >> 2;
+        const int li = q * 32 + lane;
+        const int c0 = 64 * h;                           // this warp's 64 accumulator columns
+        const int64_t ldo = args.ldo;
+        const int64_t n = nbits;
+        for (int64_t tl = 0; tl < my_tiles; ++tl) {
+            const int acc = (int)(tl & 1);
+            const uint32_t ph = (uint32_t)((tl >> 1) & 1);
+            const int64_t t = blockIdx.x + tl * gridDim.x;
+            const int64_t gl = (t % args.nlb) * BM + li;
+            const int64_t gc0 = (t / args.nlb) * BN + c0;
+            const int pbuf = (int)(tl % NPB);
+            ptx::mbar_wait(&popf[pbuf], (uint32_t)((tl / NPB) & 1));
+            ptx::mbar_wait(&accf[acc], ph);
+            ptx::tc_fence_after();
+            uint32_t pl = 0;
+#pragma unroll
+            for (int gg = 0; gg < G; ++gg) pl += popA[(pbuf * G + gg) * BM + li];
+            const uint32_t *pB = popB + pbuf * G * BN + c0;
+            const bool rows_ok = gl < args.nl && gc0 < args.nc;
+            const int ncols = rows_ok ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
+            const bool full_vec = ncols == 64 && !args.swap;
+            const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * ACC_COLS + c0);
+            // two halves of 32 accumulator columns; the accumulator is released right after
+            // the second TMEM load, before that half is processed
+#pragma unroll 1
+            for (int hh = 0; hh < 2; ++hh) {
+                uint32_t v[32];
+                tmem_ld32(ta + 32 * hh, v);
+                ptx::tmem_ld_wait();
+                if (hh == 1) {
+                    ptx::tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) ptx::mbar_arrive(&acce[acc]);   // accumulator drained
+                }
+                if (!rows_ok) continue;
+#pragma unroll
+                for (int uu = 0; uu < 32; uu += 4) {
+                    const int u0 = 32 * hh + uu;
+                    uint32_t c[4], pc[4];
+                    {
+                        uint4 s4 = *reinterpret_cast<const uint4 *>(pB + u0);
+#pragma unroll
+                        for (int gg = 1; gg < G; ++gg) {
+                            const uint4 t4 = *reinterpret_cast<const uint4 *>(pB + gg * BN + u0);
+                            s4.x += t4.x; s4.y += t4.y; s4.z += t4.z; s4.w += t4.w;
+                        }
+                        pc[0] = s4.x; pc[1] = s4.y; pc[2] = s4.z; pc[3] = s4.w;
+                    }
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) c[k] = __float2uint_rn(__uint_as_float(v[uu + k]));   // exact
+                    if (EPI == EPI_COUNTS) {
+                        uint32_t r[4];
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            const uint32_t pq = args.swap ? pc[k] : pl, pd = args.swap ? pl : pc[k];
+                            const int op = args.op;
+                            r[k] = op == 0 ? c[k] : op == 1 ? pq + pd - 2u * c[k] : op == 2 ? pq - c[k] : pd - c[k];
+                        }
+                        if (full_vec) {
+                            uint32_t *o = args.C + gl * ldo + gc0 + u0;
+                            if (((uintptr_t)o & 15u) == 0) {
+                                uint4 rr = make_uint4(r[0], r[1], r[2], r[3]);
+                                if (args.accumulate) {
+                                    const uint4 pv = *reinterpret_cast<const uint4 *>(o);
+                                    rr.x += pv.x; rr.y += pv.y; rr.z += pv.z; rr.w += pv.w;
+                                }
+                                *reinterpret_cast<uint4 *>(o) = rr;
+                                continue;
+                            }
+                        }
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            if (u0 + k >= ncols) break;
+                            uint32_t *o = args.swap ? args.C + (gc0 + u0 + k) * ldo + gl : args.C + gl * ldo + gc0 + u0 + k;
+                            *o = args.accumulate ? *o + r[k] : r[k];
+                        }
+                    } else {
+                        float r2v[4], dpv[4];
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            const int64_t pa_ = args.swap ? pc[k] : pl, pb_ = args.swap ? pl : pc[k];
+                            ld_stats_f32(n, pa_, pb_, (int64_t)c[k], r2v[k], dpv[k]);
+                        }
+                        if (full_vec) {
+                            const int64_t o = gl * ldo + gc0 + u0;
+                            if ((o & 3) == 0) {
+                                *reinterpret_cast<float4 *>(args.r2 + o) = make_float4(r2v[0], r2v[1], r2v[2], r2v[3]);
+                                if (args.dprime)
+                                    *reinterpret_cast<float4 *>(args.dprime + o) = make_float4(dpv[0], dpv[1], dpv[2], dpv[3]);
+                                if (args.C) *reinterpret_cast<uint4 *>(args.C + o) = make_uint4(c[0], c[1], c[2], c[3]);
+                                continue;
+                            }
+                        }
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            if (u0 + k >= ncols) break;
+                            const int64_t o = args.swap ? (gc0 + u0 + k) * ldo + gl : gl * ldo + gc0 + u0 + k;
+                            args.r2[o] = r2v[k];
+                            if (args.dprime) args.dprime[o] = dpv[k];
+                            if (args.C) args.C[o] = c[k];
+                        }
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&popfree[pbuf]);
+        }
+    }
+
+    ptx::tc_fence_before();
+    __syncthreads();
+    if (warp == MMA_WARP) {
+        ptx::tc_fence_after();
+        ptx::tmem_dealloc<512>(tmem);
+    }
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+    static EncodeTiledFn fn = nullptr;
+    if (!fn) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(p);
+    }
+    return fn;
+}
+
+bool make_map(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32) {
+    EncodeTiledFn enc = encode_fn();
+    if (!enc) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)ld32, (cuuint64_t)rows};
+    const cuuint64_t strides[1] = {(cuuint64_t)ld32 * 4};
+    const cuuint32_t box[2] = {KW, 128};
+    const cuuint32_t estr[2] = {1, 1};
+    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(base), dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+int num_sms() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+template <int EPI>
+cudaError_t launch_g(const GArgs &g, const uint32_t *L, int64_t ldl32, const uint32_t *Cn, int64_t ldc32,
+                     cudaStream_t s) {
+    CUtensorMap tmL, tmC;
+    if (!make_map(&tmL, L, g.nl, ldl32) || !make_map(&tmC, Cn, g.nc, ldc32)) return cudaErrorInvalidValue;
+    auto kern = gemm_tc4_kernel<EPI>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    const int64_t ntiles = g.nlb * g.ncb;
+    const int grid = (int)(ntiles < num_sms() ? ntiles : num_sms());
+    kern<<<grid, NTHREADS, SMEM, s>>>(tmL, tmC, g);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
+    return m >= 1 && n >= 1 && nbits >= 1 && nbits < (1LL << 24) && m < (1LL << 31) && n < (1LL << 31);
+}
+
+cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
+    GArgs g{};
+    const bool swap = a.m < a.n;     // larger operand on TMEM lanes
+    const uint32_t *L = swap ? a.B : a.A, *Cn = swap ? a.A : a.B;
+    const int64_t ldl32 = swap ? a.ldb32 : a.lda32, ldc32 = swap ? a.lda32 : a.ldb32;
+    g.nl = swap ? a.n : a.m;
+    g.nc = swap ? a.m : a.n;
+    g.nbits = a.nbits;
+    g.swap = swap ? 1 : 0;
+    g.op = a.op;
+    g.accumulate = a.accumulate;
+    g.ldo = a.ldc;
+    g.C = a.C;
+    g.r2 = a.r2;
+    g.dprime = a.dprime;
+    g.nlb = (g.nl + BM - 1) / BM;
+    g.ncb = (g.nc + BN - 1) / BN;
+    g.nst = (int)((a.nbits + KBITS - 1) / KBITS);
+    return epi == EPI_LD ? launch_g<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
+}
+
+}  // namespace snp

@@ -113,8 +113,8 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
         if (!want_i8 && !no_fastid && epi == EPI_COUNTS && fastid_tc4_supported(a.m, a.n, a.nbits)) {
             e = launch_fastid_tc4(a, epi, s);
             g_last_kernel = SNP_KERNEL_FASTID_MXF4;
-        } else if (!want_i8 && tc4_supported(a.m, a.n, a.nbits)) {
-            e = launch_bitgemm_tc4(a, epi, s);
+        } else if (!want_i8 && gemm_tc4_supported(a.m, a.n, a.nbits)) {
+            e = launch_gemm_tc4(a, epi, s);
             g_last_kernel = SNP_KERNEL_TC_MXF4;
         } else {
             e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
