@@ -10,7 +10,7 @@ import ctypes
 import os
 import threading
 
-LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libsnp.so")
+LIB_PATH = os.environ.get("SNP_LIB_PATH") or os.path.join(os.path.dirname(os.path.abspath(__file__)), "libsnp.so")
 
 # Every symbol include/snp.h declares: name -> (restype, argtypes)
 _i64, _int, _sz, _p = ctypes.c_int64, ctypes.c_int, ctypes.c_size_t, ctypes.c_void_p

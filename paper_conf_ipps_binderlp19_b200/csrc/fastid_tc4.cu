@@ -18,7 +18,7 @@
 //     K = 64) from TMEM-A x SMEM-B into one of two TMEM accumulators;
 //   * 4 epilogue warps apply the popcount identity and write out[q][d] coalesced along d
 //     while the next tile is being multiplied.
-// Exactness: see bitgemm_tc4.cu (products in {0, 1}, fp32 sums exact below 2^24).
+// Exactness: products are in {0, 1}, fp32 sums of them are exact below 2^24.
 #include "snp_internal.h"
 #include "tc_ptx.cuh"
 
@@ -99,6 +99,7 @@ __host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
 
 
 __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile(
         "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
             taddr),
@@ -108,6 +109,7 @@ __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16
 }
 
 __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile(
         "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
         "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
@@ -119,6 +121,7 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32
 }
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
         "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
@@ -225,7 +228,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 const int64_t t = blockIdx.x + tl * gridDim.x;
                 const int32_t row0 = (int32_t)(t * BM);
                 for (int s = 0; s < nst; ++s) {
-                    if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);
+                    if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
                     ptx::mbar_arrive_expect_tx(&pfull[p], PSTAGE);
                     ptx::tma_load_2d(ring + p * PSTAGE, &tmD, &pfull[p], s * (KBITS / 32), row0);
                     if (++p == NP) { p = 0; ++round; }
@@ -243,7 +246,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         auto publish_until = [&](int64_t upto) {
             for (; cur_tl < upto; ++cur_tl) {
                 const int acc = (int)(cur_tl & 1);
-                if (cur_tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((cur_tl >> 1) - 1) & 1));
+                if (cur_tl >= 2) ptx::mbar_wait_warp(&acce[acc], (uint32_t)(((cur_tl >> 1) - 1) & 1));
                 popD[(acc * G + g) * BM + arow] = popa;
                 popa = 0;
                 __syncwarp();
@@ -258,8 +261,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             publish_until(tl);
             const bool tr = args.trace && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
             if (tr) g_fastid_trace[8 * it + 0] = clock64();
-            ptx::mbar_wait(&pfull[p], pround & 1);
-            if (bround > 0) ptx::mbar_wait(&empty[b], (bround - 1) & 1);
+            ptx::mbar_wait_warp(&pfull[p], pround & 1);
+            if (bround > 0) ptx::mbar_wait_warp(&empty[b], (bround - 1) & 1);
             if (tr) g_fastid_trace[8 * it + 1] = clock64();
             // 64-byte row of the stage; TMA 64B swizzle: 16-byte chunk c of row r sits at
             // chunk c ^ ((r >> 1) & 3)  (conflict-free LDS.128 across the warp)
@@ -317,12 +320,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         int64_t itm = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
-            if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            if (tl >= 2) ptx::mbar_wait_warp(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
             ptx::tc_fence_after();
             const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
             uint64_t bd = bdesc0;
             for (int s = 0; s < nst; ++s, ++itm) {
-                ptx::mbar_wait(&full[b], bround & 1);
+                ptx::mbar_wait_warp(&full[b], bround & 1);
                 const bool trm = args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024;
                 if (trm) g_fastid_trace[8 * itm + 3] = clock64();
                 ptx::tc_fence_after();
@@ -349,8 +352,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             const int acc = (int)(tl & 1);
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
             const int64_t t = blockIdx.x + tl * gridDim.x;
-            ptx::mbar_wait(&popf[acc], ph);
-            ptx::mbar_wait(&accf[acc], ph);
+            ptx::mbar_wait_warp(&popf[acc], ph);
+            ptx::mbar_wait_warp(&accf[acc], ph);
             ptx::tc_fence_after();
             uint32_t v[32];
             tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);

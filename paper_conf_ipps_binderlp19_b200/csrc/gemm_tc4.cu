@@ -4,7 +4,7 @@
 //   + fused epilogue: counts / FastID op identities / LD r2, D' (a5)
 //
 // Bits become e2m1 nibbles (1 -> 1.0) and are multiplied with tcgen05.mma kind::mxf4
-// (scale factors 2^0, exact fp32 sums below 2^24; see bitgemm_tc4.cu / DESIGN.md §6).
+// (scale factors 2^0, exact fp32 sums below 2^24).
 // 128 x 128 output tiles, persistent CTAs (one per SM), K in 512-bit stages.
 //
 // Per stage, for the 128 lane rows (A) and 128 column rows (B) of the tile:
@@ -27,27 +27,36 @@
 #include <cstdlib>
 
 namespace snp {
+
+// Pipeline trace of CTA 0 (profiling aid, SNP_TRACE=1): per iteration it < 2048,
+// [0] expander before waits, [1] after waits, [2] after packed LDS, [3] half 0 published,
+// [4] half 1 published, [5] MMA got half 0, [6] MMA got half 1, [7] MMA commit issued.
+__device__ long long g_gemm_trace[8 * 2048];
+
 namespace {
 
 constexpr int BM = 128, BN = 128;
 constexpr int KBITS = 512;
 constexpr int KW = KBITS / 32;                 // 16 packed words per row per stage
-constexpr int G = 3;                           // expander groups == stage slots
-constexpr int NEXP = 4 * G;                    // 12 expander warps
+constexpr int NS = 3;                          // pipeline slots (packed ring, TMEM A, smem B)
+#ifndef GEMM_G
+#define GEMM_G 2
+#endif
+constexpr int G = GEMM_G;                      // expander groups (group g takes stages it = g mod G)
+constexpr int NEXP = 8 * G;                    // per group: 4 A-warps (TMEM) + 4 B-warps (smem)
 constexpr int NEPI = 8;
-constexpr int EPI_WARP0 = NEXP;                // 12..19
-constexpr int TMA_WARP = NEXP + NEPI;          // 20
-constexpr int MMA_WARP = NEXP + NEPI + 1;      // 21 (highest id: scheduler priority)
+constexpr int EPI_WARP0 = NEXP;                // 16..23
+constexpr int TMA_WARP = NEXP + NEPI;          // 24
+constexpr int MMA_WARP = NEXP + NEPI + 1;      // 25 (highest id: scheduler priority)
 constexpr int NTHREADS = (NEXP + NEPI + 2) * 32;
 constexpr int PROW = KBITS / 8;                // 64 packed bytes per row per stage
 constexpr int PSLOT = (BM + BN) * PROW;        // 16 KB packed per slot (A then B)
 constexpr int BSLOT = BN * KBITS / 2;          // 32 KB expanded B per slot
 constexpr int ACC_COLS = BN;
 constexpr int A_COL0 = 2 * ACC_COLS;           // 256
-constexpr int SF_COL = A_COL0 + G * 64;        // 448
+constexpr int SF_COL = A_COL0 + NS * 64;       // 448
 static_assert(SF_COL + 32 <= 512, "TMEM budget");
-constexpr int NPB = 4;                         // popcount buffers (tiles in flight)
-constexpr size_t SMEM = (size_t)G * PSLOT + (size_t)G * BSLOT + 16384;
+constexpr size_t SMEM = (size_t)NS * PSLOT + (size_t)NS * BSLOT + 1024;
 
 struct GArgs {
     int64_t nl, nc, nbits;
@@ -57,6 +66,9 @@ struct GArgs {
     float *r2, *dprime;
     int64_t nlb, ncb;
     int nst;
+    int trace;
+    int debug_skip;   // profiling experiment: expanders only pass tokens (results invalid)
+    const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
 };
 
 __device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
@@ -81,6 +93,7 @@ __host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
 }
 
 __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile(
         "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
         "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
@@ -92,6 +105,7 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32
 }
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
         "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
@@ -132,20 +146,16 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
                 const GArgs args) {
     extern __shared__ __align__(1024) uint8_t smem[];
-    uint8_t *ring = smem;                                        // [G][PSLOT]
-    uint8_t *bexp = smem + (size_t)G * PSLOT;                    // [G][BSLOT]
-    uint64_t *bars = reinterpret_cast<uint64_t *>(bexp + (size_t)G * BSLOT);
-    uint64_t *pfull = bars;            // [G] TMA -> expanders
-    uint64_t *pempty = pfull + G;      // [G] expanders -> TMA
-    uint64_t *full = pempty + G;       // [G] expanders -> MMA
-    uint64_t *empty = full + G;        // [G] MMA -> expanders
-    uint64_t *accf = empty + G;        // [2]
+    uint8_t *ring = smem;                                        // [NS][PSLOT]
+    uint8_t *bexp = smem + (size_t)NS * PSLOT;                   // [NS][BSLOT]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(bexp + (size_t)NS * BSLOT);
+    uint64_t *pfull = bars;            // [NS] TMA -> expanders
+    uint64_t *pempty = pfull + NS;     // [NS] expanders -> TMA
+    uint64_t *full = pempty + NS;      // [NS] expanders -> MMA
+    uint64_t *empty = full + NS;       // [NS] MMA -> expanders
+    uint64_t *accf = empty + NS;       // [2]
     uint64_t *acce = accf + 2;         // [2]
-    uint64_t *popf = acce + 2;         // [NPB] expanders -> epilogue (popcounts of a tile written)
-    uint64_t *popfree = popf + NPB;    // [NPB] epilogue -> expanders (popcount buffer reusable)
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popfree + NPB);
-    uint32_t *popA = tmem_slot + 4;    // [NPB][G][BM]
-    uint32_t *popB = popA + NPB * G * BM;  // [NPB][G][BN]
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acce + 2);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t nbits = args.nbits;
@@ -156,19 +166,15 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     const int64_t full32 = nbits / 32;
 
     if (tid == 0) {
-        for (int i = 0; i < G; ++i) {
+        for (int i = 0; i < NS; ++i) {
             ptx::mbar_init(&pfull[i], 1);
-            ptx::mbar_init(&pempty[i], 4);
-            ptx::mbar_init(&full[i], 4);
+            ptx::mbar_init(&pempty[i], 8);
+            ptx::mbar_init(&full[i], 8);
             ptx::mbar_init(&empty[i], 1);
         }
         for (int i = 0; i < 2; ++i) {
             ptx::mbar_init(&accf[i], 1);
             ptx::mbar_init(&acce[i], NEPI);
-        }
-        for (int i = 0; i < NPB; ++i) {
-            ptx::mbar_init(&popf[i], NEXP);
-            ptx::mbar_init(&popfree[i], NEPI);
         }
         ptx::fence_mbar_init();
     }
@@ -202,91 +208,96 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 const int64_t t = blockIdx.x + tl * gridDim.x;
                 const int32_t rl = (int32_t)((t % args.nlb) * BM), rc = (int32_t)((t / args.nlb) * BN);
                 for (int s = 0; s < nst; ++s) {
-                    if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);
+                    if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
                     ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
                     ptx::tma_load_2d(ring + p * PSLOT, &tmL, &pfull[p], s * KW, rl);
                     ptx::tma_load_2d(ring + p * PSLOT + BM * PROW, &tmC, &pfull[p], s * KW, rc);
-                    if (++p == G) { p = 0; ++round; }
+                    if (++p == NS) { p = 0; ++round; }
                 }
             }
         }
     } else if (warp < NEXP) {
         // ------------------------------------------------------------ expanders
-        const int g = warp >> 2, q = warp & 3;
-        const int row = q * 32 + lane;                  // A row (TMEM lane) and B row of this thread
+        // group g = warp / 8 takes stages it = g, g + G, ...; within a group warps 0-3 expand
+        // the A rows of lane quarter q into TMEM, warps 4-7 the B rows into shared memory,
+        // so the TMEM and shared-memory chains of a stage run in parallel.
+        const int g = warp >> 3, r8 = warp & 7;
+        const bool is_a = r8 < 4;
+        const int q = r8 & 3;
+        const int row = q * 32 + lane;
         const int sw = (row >> 1) & 3;                  // TMA 64B swizzle of a 64-byte row
-        uint32_t pa = 0, pb = 0;
-        int64_t cur_tl = 0;
-        auto publish_until = [&](int64_t upto) {
-            for (; cur_tl < upto; ++cur_tl) {
-                const int pbuf = (int)(cur_tl % NPB);
-                if (cur_tl >= NPB) ptx::mbar_wait(&popfree[pbuf], (uint32_t)(((cur_tl / NPB) - 1) & 1));
-                popA[(pbuf * G + g) * BM + row] = pa;
-                popB[(pbuf * G + g) * BN + row] = pb;
-                pa = pb = 0;
-                __syncwarp();
-                if (lane == 0) ptx::mbar_arrive(&popf[pbuf]);
-            }
-        };
+        const uint32_t tAq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)A_COL0;
         int64_t tl = g / nst;
         int s = g % nst;
-        uint32_t round = 0;
-        const uint8_t *srcA = ring + g * PSLOT + row * PROW;
-        const uint8_t *srcB = srcA + BM * PROW;
-        uint8_t *dstB = bexp + (size_t)g * BSLOT + row * 16;
-        const uint32_t tA = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(A_COL0 + 64 * g);
+        int slot = g % NS;
+        uint32_t use = (uint32_t)(g / NS);              // how often `slot` was used before
         for (int64_t it = g; it < total_it; it += G) {
-            publish_until(tl);
-            ptx::mbar_wait(&pfull[g], round & 1);
-            if (round > 0) ptx::mbar_wait(&empty[g], (round - 1) & 1);
-            uint32_t wa[KW], wb[KW];
+            const bool tr = args.trace && blockIdx.x == 0 && r8 == 0 && lane == 0 && it < 2048;
+            if (tr) g_gemm_trace[8 * it + 0] = clock64();
+            // empty BEFORE pfull: both groups share the slots, so a warp may reach use u+2 of
+            // a slot while its pfull barrier is only at phase u+1; waiting for the MMA to
+            // release use u+1 first rules out parity aliasing on pfull (same parity as u)
+            if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
+            ptx::mbar_wait_warp(&pfull[slot], use & 1);
+            if (tr) g_gemm_trace[8 * it + 1] = clock64();
+            if (args.debug_skip) {
+                __syncwarp();
+                if (lane == 0) { ptx::mbar_arrive(&pempty[slot]); ptx::mbar_arrive(&full[slot]); }
+                s += G;
+                while (s >= nst) { s -= nst; ++tl; }
+                slot += G;
+                if (slot >= NS) { slot -= NS; ++use; }
+                continue;
+            }
+            const uint8_t *src = ring + slot * PSLOT + (is_a ? 0 : BM * PROW) + row * PROW;
+            uint32_t w[KW];
 #pragma unroll
             for (int c = 0; c < 4; ++c) {
-                const uint4 xa = *reinterpret_cast<const uint4 *>(srcA + ((c ^ sw) << 4));
-                const uint4 xb = *reinterpret_cast<const uint4 *>(srcB + ((c ^ sw) << 4));
-                wa[4 * c] = xa.x; wa[4 * c + 1] = xa.y; wa[4 * c + 2] = xa.z; wa[4 * c + 3] = xa.w;
-                wb[4 * c] = xb.x; wb[4 * c + 1] = xb.y; wb[4 * c + 2] = xb.z; wb[4 * c + 3] = xb.w;
+                const uint4 x = *reinterpret_cast<const uint4 *>(src + ((c ^ sw) << 4));
+                w[4 * c] = x.x; w[4 * c + 1] = x.y; w[4 * c + 2] = x.z; w[4 * c + 3] = x.w;
             }
-            __syncwarp();
-            if (lane == 0) ptx::mbar_arrive(&pempty[g]);
+            if (tr) g_gemm_trace[8 * it + 2] = clock64();
             const int64_t w0 = (int64_t)s * KW;
             if (w0 + KW > full32) {
 #pragma unroll
-                for (int i = 0; i < KW; ++i) {
-                    const uint32_t mk = word_mask(w0 + i, nbits);
-                    wa[i] &= mk;
-                    wb[i] &= mk;
+                for (int i = 0; i < KW; ++i) w[i] &= word_mask(w0 + i, nbits);
+            }
+            if (is_a) {
+                const uint32_t tA = tAq + 64 * slot;
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    uint32_t v[32];
+#pragma unroll
+                    for (int i = 0; i < 8; ++i)
+                        expand4(w[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+                    tmem_st32(tA + 32 * h, v);
                 }
-            }
+                ptx::tmem_st_wait();
+                ptx::tc_fence_before();
+            } else {
+                uint8_t *dstB = bexp + (size_t)slot * BSLOT + row * 16;
 #pragma unroll
-            for (int i = 0; i < KW; ++i) {
-                pa += __popc(wa[i]);
-                pb += __popc(wb[i]);
+                for (int i = 0; i < KW; ++i) {          // chunk i of the K-major operand = word i
+                    uint4 o;
+                    expand4(w[i], o.x, o.y, o.z, o.w);
+                    *reinterpret_cast<uint4 *>(dstB + (size_t)i * BN * 16) = o;
+                }
+                ptx::fence_proxy_async_smem();
             }
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                uint32_t v[32];
-#pragma unroll
-                for (int i = 0; i < 8; ++i)
-                    expand4(wa[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-                tmem_st32(tA + 32 * h, v);
-            }
-#pragma unroll
-            for (int i = 0; i < KW; ++i) {          // chunk i of the K-major operand = word i
-                uint4 o;
-                expand4(wb[i], o.x, o.y, o.z, o.w);
-                *reinterpret_cast<uint4 *>(dstB + (size_t)i * BN * 16) = o;
-            }
-            ptx::tmem_st_wait();
-            ptx::fence_proxy_async_smem();
-            ptx::tc_fence_before();
             __syncwarp();
-            if (lane == 0) ptx::mbar_arrive(&full[g]);
+            if (lane == 0) {
+                // release the packed slot only now: every lane has consumed its LDS results
+                // (an arrive right after the loads could let the next TMA overwrite data
+                // that is still in flight to registers)
+                ptx::mbar_arrive(&pempty[slot]);
+                ptx::mbar_arrive(&full[slot]);
+            }
+            if (tr) g_gemm_trace[8 * it + 3] = clock64();
             s += G;
             while (s >= nst) { s -= nst; ++tl; }
-            ++round;
+            slot += G;
+            if (slot >= NS) { slot -= NS; ++use; }
         }
-        publish_until(my_tiles);
     } else if (warp == MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
         constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
@@ -295,53 +306,65 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;
         int b = 0;
         uint32_t round = 0;
+        int64_t itm = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
-            if (tl >= 2) ptx::mbar_wait(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            if (tl >= 2) ptx::mbar_wait_warp(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
             ptx::tc_fence_after();
             const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS);
-            for (int s = 0; s < nst; ++s) {
-                ptx::mbar_wait(&full[b], round & 1);
+            for (int s = 0; s < nst; ++s, ++itm) {
+                const bool trm = args.trace && blockIdx.x == 0 && lane == 0 && itm < 2048;
+                ptx::mbar_wait_warp(&full[b], round & 1);
+                if (trm) g_gemm_trace[8 * itm + 5] = clock64();
                 ptx::tc_fence_after();
                 ptx::mma8_mxf4_ts_commit(d, tmem + (uint32_t)(A_COL0 + 64 * b),
                                          bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4), BSTEP, IDESC,
                                          s != 0 ? 1u : 0u, sfa, sfb, &empty[b]);
-                if (++b == G) { b = 0; ++round; }
+                if (trm) g_gemm_trace[8 * itm + 7] = clock64();
+                if (++b == NS) { b = 0; ++round; }
             }
             ptx::mma_commit_elect(&accf[acc]);
         }
         __syncwarp();
     } else {
         // ------------------------------------------------------------ epilogue (8 warps)
+        // warp e: TMEM lane quarter e % 4 (lane rows), accumulator columns [64 h, 64 h + 64)
         const int e = warp - EPI_WARP0;
         const int q = e & 3, h = e >> 2;
         const int li = q * 32 + lane;
-        const int c0 = 64 * h;                           // this warp's 64 accumulator columns
+        const int c0 = 64 * h;
         const int64_t ldo = args.ldo;
         const int64_t n = nbits;
+        const bool small_n = n <= 46340;                 // n^2 < 2^31: exact int32 LD arithmetic
+        const bool need_pop = EPI == EPI_LD || args.op != 0;
+        const bool want_dp = EPI == EPI_LD && args.dprime != nullptr;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
             const int64_t t = blockIdx.x + tl * gridDim.x;
             const int64_t gl = (t % args.nlb) * BM + li;
             const int64_t gc0 = (t / args.nlb) * BN + c0;
-            const int pbuf = (int)(tl % NPB);
-            ptx::mbar_wait(&popf[pbuf], (uint32_t)((tl / NPB) & 1));
-            ptx::mbar_wait(&accf[acc], ph);
-            ptx::tc_fence_after();
-            uint32_t pl = 0;
-#pragma unroll
-            for (int gg = 0; gg < G; ++gg) pl += popA[(pbuf * G + gg) * BM + li];
-            const uint32_t *pB = popB + pbuf * G * BN + c0;
             const bool rows_ok = gl < args.nl && gc0 < args.nc;
-            const int ncols = rows_ok ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
+            const int ncols = gc0 < args.nc ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
+            // popcounts: lane j holds the column popcounts of columns c0 + j and c0 + 32 + j
+            uint32_t pl = 0, pcol0 = 0, pcol1 = 0;
+            if (need_pop) {
+                if (gl < args.nl) pl = __ldg(args.popL + gl);
+                if (lane < ncols) pcol0 = __ldg(args.popC + gc0 + lane);
+                if (32 + lane < ncols) pcol1 = __ldg(args.popC + gc0 + 32 + lane);
+            }
+            ptx::mbar_wait_warp(&accf[acc], ph);
+            ptx::tc_fence_after();
             const bool full_vec = ncols == 64 && !args.swap;
             const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * ACC_COLS + c0);
+            const int32_t n32 = (int32_t)n, pl32 = (int32_t)pl;
+            const int32_t da32 = pl32 * (n32 - pl32);
             // two halves of 32 accumulator columns; the accumulator is released right after
             // the second TMEM load, before that half is processed
 #pragma unroll 1
             for (int hh = 0; hh < 2; ++hh) {
                 uint32_t v[32];
+                __syncwarp();            // tcgen05.ld is warp-collective: re-converge first
                 tmem_ld32(ta + 32 * hh, v);
                 ptx::tmem_ld_wait();
                 if (hh == 1) {
@@ -349,22 +372,19 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                     __syncwarp();
                     if (lane == 0) ptx::mbar_arrive(&acce[acc]);   // accumulator drained
                 }
-                if (!rows_ok) continue;
+                const uint32_t pcol = hh ? pcol1 : pcol0;
+                if (!__any_sync(0xffffffffu, rows_ok)) continue;   // warp-uniform skip only:
+                // the column popcounts are shuffled across the warp, so every lane runs the
+                // loop and only rows_ok lanes store
 #pragma unroll
                 for (int uu = 0; uu < 32; uu += 4) {
                     const int u0 = 32 * hh + uu;
                     uint32_t c[4], pc[4];
-                    {
-                        uint4 s4 = *reinterpret_cast<const uint4 *>(pB + u0);
 #pragma unroll
-                        for (int gg = 1; gg < G; ++gg) {
-                            const uint4 t4 = *reinterpret_cast<const uint4 *>(pB + gg * BN + u0);
-                            s4.x += t4.x; s4.y += t4.y; s4.z += t4.z; s4.w += t4.w;
-                        }
-                        pc[0] = s4.x; pc[1] = s4.y; pc[2] = s4.z; pc[3] = s4.w;
+                    for (int k = 0; k < 4; ++k) {
+                        c[k] = __float2uint_rn(__uint_as_float(v[uu + k]));    // exact count
+                        pc[k] = __shfl_sync(0xffffffffu, pcol, uu + k);
                     }
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) c[k] = __float2uint_rn(__uint_as_float(v[uu + k]));   // exact
                     if (EPI == EPI_COUNTS) {
                         uint32_t r[4];
 #pragma unroll
@@ -373,6 +393,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                             const int op = args.op;
                             r[k] = op == 0 ? c[k] : op == 1 ? pq + pd - 2u * c[k] : op == 2 ? pq - c[k] : pd - c[k];
                         }
+                        if (!rows_ok) continue;
                         if (full_vec) {
                             uint32_t *o = args.C + gl * ldo + gc0 + u0;
                             if (((uintptr_t)o & 15u) == 0) {
@@ -392,17 +413,38 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                             *o = args.accumulate ? *o + r[k] : r[k];
                         }
                     } else {
-                        float r2v[4], dpv[4];
+                        float r2v[4], dpv[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
                         for (int k = 0; k < 4; ++k) {
-                            const int64_t pa_ = args.swap ? pc[k] : pl, pb_ = args.swap ? pl : pc[k];
-                            ld_stats_f32(n, pa_, pb_, (int64_t)c[k], r2v[k], dpv[k]);
+                            // reading R3 from exact integers; (A, B) = (lane, column) or swapped
+                            if (small_n) {
+                                const int32_t pb = (int32_t)pc[k];
+                                const int32_t num = n32 * (int32_t)c[k] - pl32 * pb;
+                                const int32_t db = pb * (n32 - pb);
+                                if (num == 0 || da32 == 0 || db == 0) {
+                                    r2v[k] = 0.f;
+                                } else {
+                                    const float fn = (float)num;
+                                    r2v[k] = __fdiv_rn(fn * fn, (float)da32 * (float)db);
+                                    if (want_dp) {
+                                        const int32_t pa_ = args.swap ? pb : pl32, pb_ = args.swap ? pl32 : pb;
+                                        int32_t dmax;
+                                        if (num > 0) dmax = min(pa_ * (n32 - pb_), (n32 - pa_) * pb_);
+                                        else dmax = min(pa_ * pb_, (n32 - pa_) * (n32 - pb_));
+                                        dpv[k] = __fdiv_rn(fn, (float)dmax);
+                                    }
+                                }
+                            } else {
+                                const int64_t pa_ = args.swap ? pc[k] : pl, pb_ = args.swap ? pl : pc[k];
+                                ld_stats_f32(n, pa_, pb_, (int64_t)c[k], r2v[k], dpv[k]);
+                            }
                         }
+                        if (!rows_ok) continue;
                         if (full_vec) {
                             const int64_t o = gl * ldo + gc0 + u0;
                             if ((o & 3) == 0) {
                                 *reinterpret_cast<float4 *>(args.r2 + o) = make_float4(r2v[0], r2v[1], r2v[2], r2v[3]);
-                                if (args.dprime)
+                                if (want_dp)
                                     *reinterpret_cast<float4 *>(args.dprime + o) = make_float4(dpv[0], dpv[1], dpv[2], dpv[3]);
                                 if (args.C) *reinterpret_cast<uint4 *>(args.C + o) = make_uint4(c[0], c[1], c[2], c[3]);
                                 continue;
@@ -413,14 +455,12 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                             if (u0 + k >= ncols) break;
                             const int64_t o = args.swap ? (gc0 + u0 + k) * ldo + gl : gl * ldo + gc0 + u0 + k;
                             args.r2[o] = r2v[k];
-                            if (args.dprime) args.dprime[o] = dpv[k];
+                            if (want_dp) args.dprime[o] = dpv[k];
                             if (args.C) args.C[o] = c[k];
                         }
                     }
                 }
             }
-            __syncwarp();
-            if (lane == 0) ptx::mbar_arrive(&popfree[pbuf]);
         }
     }
 
@@ -499,6 +539,8 @@ bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
 cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     GArgs g{};
     const bool swap = a.m < a.n;     // larger operand on TMEM lanes
+    g.popL = swap ? a.popB : a.popA;
+    g.popC = swap ? a.popA : a.popB;
     const uint32_t *L = swap ? a.B : a.A, *Cn = swap ? a.A : a.B;
     const int64_t ldl32 = swap ? a.ldb32 : a.lda32, ldc32 = swap ? a.lda32 : a.ldb32;
     g.nl = swap ? a.n : a.m;
@@ -514,7 +556,26 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.nlb = (g.nl + BM - 1) / BM;
     g.ncb = (g.nc + BN - 1) / BN;
     g.nst = (int)((a.nbits + KBITS - 1) / KBITS);
+    static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
+    g.trace = trace ? 1 : 0;
+    static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
+    g.debug_skip = skip ? 1 : 0;
     return epi == EPI_LD ? launch_g<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
 }
 
 }  // namespace snp
+
+extern "C" int snp_debug_gemm_trace(long long *host, int n) {
+    if (n > 8 * 2048) n = 8 * 2048;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_gemm_trace, sizeof(long long) * n);
+}
+
+// Debug aid (not in include/snp.h): mode 1 makes a stuck gemm_tc4 pipeline record where
+// it waited and release all waits instead of trapping; returns and clears the record.
+extern "C" int snp_debug_gemm_watchdog(int mode, int *record8) {
+    cudaMemcpyToSymbol(snp::ptx::g_snp_watchdog_mode, &mode, sizeof(int));
+    if (record8) cudaMemcpyFromSymbol(record8, snp::ptx::g_snp_watchdog, 8 * sizeof(int));
+    int zero[8] = {0};
+    cudaMemcpyToSymbol(snp::ptx::g_snp_watchdog, zero, sizeof(zero));
+    return (int)cudaGetLastError();
+}

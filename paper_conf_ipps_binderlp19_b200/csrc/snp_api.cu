@@ -11,6 +11,7 @@
 
 using namespace snp;
 
+
 namespace {
 
 thread_local char g_cuda_err[256] = "";
@@ -100,26 +101,49 @@ int choose_variant(int64_t m, int64_t n, int64_t nbits) {
 
 size_t pops_bytes(int64_t m, int64_t n) { return align256((size_t)m * 4) + align256((size_t)n * 4); }
 
+// Which tensor-core kernel serves a shape (mirrors run_gemm's choice).
+int tc_kernel_for(int64_t m, int64_t n, int64_t nbits, int epi) {
+    const char *kind = std::getenv("SNP_TC_KIND");
+    const bool want_i8 = kind && !std::strcmp(kind, "i8");
+    const char *ff = std::getenv("SNP_FASTID_KERNEL");
+    const bool no_fastid = ff && !std::strcmp(ff, "0");
+    if (!want_i8 && !no_fastid && epi == EPI_COUNTS && fastid_tc4_supported(m, n, nbits)) return SNP_KERNEL_FASTID_MXF4;
+    if (!want_i8 && gemm_tc4_supported(m, n, nbits)) return SNP_KERNEL_TC_MXF4;
+    return SNP_KERNEL_TC_I8;
+}
+
+// ws layout: [popA: align256(4m)][popB: align256(4n)][kernel scratch]
 snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes, cudaStream_t s) {
     cudaError_t e;
     if (variant == SNP_VARIANT_TC) {
         if (!tc_supported(a.m, a.n, a.nbits)) return SNP_E_SHAPE;
         // kind::mxf4 (2x the int8 rate, half the expanded bytes) unless K is too long
         // for exact fp32 accumulation or SNP_TC_KIND=i8 asks for the int8 kernel.
-        const char *kind = std::getenv("SNP_TC_KIND");
-        const bool want_i8 = kind && !std::strcmp(kind, "i8");
-        const char *ff = std::getenv("SNP_FASTID_KERNEL");
-        const bool no_fastid = ff && !std::strcmp(ff, "0");
-        if (!want_i8 && !no_fastid && epi == EPI_COUNTS && fastid_tc4_supported(a.m, a.n, a.nbits)) {
-            e = launch_fastid_tc4(a, epi, s);
-            g_last_kernel = SNP_KERNEL_FASTID_MXF4;
-        } else if (!want_i8 && gemm_tc4_supported(a.m, a.n, a.nbits)) {
+        const int kern = tc_kernel_for(a.m, a.n, a.nbits, epi);
+        if (kern == SNP_KERNEL_FASTID_MXF4) {
+            e = launch_fastid_tc4(a, epi, s);   // derives popcounts from the streamed words
+        } else if (kern == SNP_KERNEL_TC_MXF4) {
+            if (epi == EPI_LD || a.op != SNP_OP_AND) {
+                // the general kernel reads row popcounts: cheap pre-pass if not given
+                if (ws_bytes < pops_bytes(a.m, a.n) || !ws) return SNP_E_WORKSPACE;
+                uint32_t *pa = reinterpret_cast<uint32_t *>(ws);
+                uint32_t *pb = reinterpret_cast<uint32_t *>((char *)ws + align256((size_t)a.m * 4));
+                const uint64_t *A64 = reinterpret_cast<const uint64_t *>(a.A);
+                const uint64_t *B64 = reinterpret_cast<const uint64_t *>(a.B);
+                if (!a.popA) {
+                    if ((e = launch_row_popc(A64, a.m, a.nbits, a.lda32 / 2, pa, s)) != cudaSuccess) return set_cuda_error(e);
+                    a.popA = pa;
+                }
+                if (!a.popB) {
+                    if ((e = launch_row_popc(B64, a.n, a.nbits, a.ldb32 / 2, pb, s)) != cudaSuccess) return set_cuda_error(e);
+                    a.popB = pb;
+                }
+            }
             e = launch_gemm_tc4(a, epi, s);
-            g_last_kernel = SNP_KERNEL_TC_MXF4;
         } else {
             e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
-            g_last_kernel = SNP_KERNEL_TC_I8;
         }
+        g_last_kernel = kern;
     } else {
         e = launch_bitgemm_popc(a, epi, s);
         g_last_kernel = SNP_KERNEL_POPC;
@@ -150,9 +174,10 @@ size_t snp_ld_workspace_bytes(int64_t m, int64_t n, int64_t nbits) {
 }
 
 size_t snp_fastid_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op) {
-    (void)op;
     if (nq <= 0 || nd <= 0 || nbits <= 0) return 0;
     if (choose_variant(nq, nd, nbits) != SNP_VARIANT_TC) return 0;
+    if (op != SNP_OP_AND && tc_kernel_for(nq, nd, nbits, EPI_COUNTS) == SNP_KERNEL_TC_MXF4)
+        return pops_bytes(nq, nd);   // row popcounts for the general kernel's identities
     return tc_workspace_bytes(nq, nd, nbits);
 }
 
@@ -204,9 +229,7 @@ snp_status snp_ld_counts(const uint64_t *A, int64_t m, int64_t lda,
     a.B = reinterpret_cast<const uint32_t *>(B);
     a.m = m; a.n = n; a.lda32 = 2 * lda; a.ldb32 = 2 * ldb; a.nbits = nbits;
     a.op = SNP_OP_AND; a.accumulate = accumulate ? 1 : 0; a.ldc = ldc; a.C = C;
-    void *tcws = variant == SNP_VARIANT_TC ? (char *)ws + pops_bytes(m, n) : nullptr;
-    size_t tcbytes = variant == SNP_VARIANT_TC ? ws_bytes - pops_bytes(m, n) : 0;
-    return run_gemm(a, EPI_COUNTS, variant, tcws, tcbytes, (cudaStream_t)stream);
+    return run_gemm(a, EPI_COUNTS, variant, ws, ws_bytes, (cudaStream_t)stream);
 }
 
 snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *popA,
@@ -232,13 +255,13 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
     uint32_t *pa = reinterpret_cast<uint32_t *>(ws);
     uint32_t *pb = reinterpret_cast<uint32_t *>((char *)ws + align256((size_t)m * 4));
     cudaError_t e;
-    // the CUDA-core variant reads row popcounts; the tensor-core kernels compute them
-    // from the packed words they stream, so no pre-pass is launched for them
-    if (variant != SNP_VARIANT_TC && !popA) {
+    // row popcounts (p_A, p_B of P:L44) for the r2/D' epilogue: one cheap pass over the
+    // packed operands (O(m+n) vs the O(m n) GEMM)
+    if (!popA) {
         if ((e = launch_row_popc(A, m, nbits, lda, pa, s)) != cudaSuccess) return set_cuda_error(e);
         popA = pa;
     }
-    if (variant != SNP_VARIANT_TC && !popB) {
+    if (!popB) {
         if ((e = launch_row_popc(B, n, nbits, ldb, pb, s)) != cudaSuccess) return set_cuda_error(e);
         popB = pb;
     }
@@ -248,9 +271,7 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
     a.m = m; a.n = n; a.lda32 = 2 * lda; a.ldb32 = 2 * ldb; a.nbits = nbits;
     a.op = SNP_OP_AND; a.accumulate = 0; a.ldc = ldc; a.C = counts;
     a.r2 = r2; a.dprime = dprime; a.popA = popA; a.popB = popB;
-    void *tcws = variant == SNP_VARIANT_TC ? (char *)ws + pops_bytes(m, n) : nullptr;
-    size_t tcbytes = variant == SNP_VARIANT_TC ? ws_bytes - pops_bytes(m, n) : 0;
-    return run_gemm(a, EPI_LD, variant, tcws, tcbytes, s);
+    return run_gemm(a, EPI_LD, variant, ws, ws_bytes, s);
 }
 
 snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t *popQ,
@@ -327,6 +348,8 @@ snp_status snp_set_variant(int variant) {
 int snp_last_variant(void) { return g_last_variant; }
 
 int snp_last_kernel(void) { return g_last_kernel; }
+
+
 
 int64_t snp_launch_count(void) { return (int64_t)g_launches.load(); }
 

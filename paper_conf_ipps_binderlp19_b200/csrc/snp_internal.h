@@ -51,9 +51,6 @@ bool tc_supported(int64_t m, int64_t n, int64_t nbits);
 cudaError_t launch_bitgemm_tc(const GemmArgs &a, int epi, void *ws, size_t ws_bytes,
                               cudaStream_t s);
 
-// Tensor-core tcgen05 kind::mxf4 variant (bitgemm_tc4.cu): exact for nbits < 2^24.
-bool tc4_supported(int64_t m, int64_t n, int64_t nbits);
-cudaError_t launch_bitgemm_tc4(const GemmArgs &a, int epi, cudaStream_t s);
 
 // General tcgen05 mxf4 kernel (gemm_tc4.cu): 128x128 tiles, TMA-fed, A in TMEM.
 bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits);

@@ -34,14 +34,38 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+// Watchdog record (debug aid, one copy per translation unit): [0] fired, [1] block,
+// [2] thread, [3] smem address of the barrier, [4] parity.
+static __device__ int g_snp_watchdog[8];
+static __device__ int g_snp_watchdog_mode;   // 0: trap, 1: record and release all waits
+
 // Wait for the phase with the given parity to complete.  A wait longer than ~4 s
 // means a broken pipeline: trap (a launch error) instead of hanging the GPU.
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-    if (mbar_try_wait(bar, parity)) return;
+static __device__ __noinline__ void mbar_wait_slow(uint64_t *bar, uint32_t parity) {
     const uint64_t t0 = globaltimer_ns();
     while (!mbar_try_wait(bar, parity)) {
-        if (globaltimer_ns() - t0 > 4000000000ull) __trap();
+        if (globaltimer_ns() - t0 > 4000000000ull) {
+            if (g_snp_watchdog_mode == 0) __trap();
+            if (atomicCAS(&g_snp_watchdog[0], 0, 1) == 0) {
+                g_snp_watchdog[1] = blockIdx.x;
+                g_snp_watchdog[2] = threadIdx.x;
+                g_snp_watchdog[3] = (int)smem_u32(bar);
+                g_snp_watchdog[4] = (int)parity;
+            }
+            return;
+        }
+        if (g_snp_watchdog_mode && *(volatile int *)&g_snp_watchdog[0]) return;
     }
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    if (mbar_try_wait(bar, parity)) return;
+    mbar_wait_slow(bar, parity);
+}
+// Same, for a whole warp that continues with warp-collective (.sync.aligned) tcgen05
+// instructions: every lane waits, then the warp is re-converged explicitly.
+__device__ __forceinline__ void mbar_wait_warp(uint64_t *bar, uint32_t parity) {
+    mbar_wait(bar, parity);
+    __syncwarp();
 }
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}" ::"r"(smem_u32(bar))
@@ -93,6 +117,7 @@ __device__ __forceinline__ void tmem_dealloc(uint32_t taddr) {      // whole war
 
 // 32 lanes x 32 bit, 8 consecutive columns: thread t of the warp gets lane (base+t).
 __device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
                  : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
                    "=r"(v[7])
@@ -102,6 +127,7 @@ __device__ __forceinline__ void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.
 
 // 32 lanes x 32 bit, 8 consecutive columns written from 8 registers per thread.
 __device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t (&v)[8]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr),
                  "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
                  : "memory");
@@ -146,17 +172,19 @@ __device__ __forceinline__ void mma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, uint
 }
 
 // Four K-steps of tcgen05.mma kind::mxf4 (block32 scales) with A from TMEM, then a
-// commit to `bar`, issued by ONE elected lane of a converged warp (the whole warp
-// must call it).  K-step i uses A columns a0 + 8 i and B descriptor b0 + i * bstep
+// commit to `bar`, issued by lane 0 of a converged warp (the whole warp must call it).
+// All MMAs and commits of a kernel are issued by the same lane: tcgen05.commit only
+// tracks the async operations of the thread that executes it.  K-step i uses A columns a0 + 8 i and B descriptor b0 + i * bstep
 // (descriptor start-address field, 16-byte units).  The first MMA accumulates iff
 // `accumulate`; the other three always accumulate.
 __device__ __forceinline__ void mma4_mxf4_ts_commit(uint32_t d, uint32_t a0, uint64_t b0, uint32_t bstep,
                                                     uint32_t idesc, uint32_t accumulate, uint32_t sfa,
                                                     uint32_t sfb, uint64_t *bar) {
+    __syncwarp();   // warp-collective (.sync.aligned / elect.sync): converge first
     const uint64_t b1 = b0 + bstep, b2 = b0 + 2 * bstep, b3 = b0 + 3 * bstep;
     asm volatile(
         "{\n\t.reg .pred e, p, t;\n\t"
-        "elect.sync _|e, 0xffffffff;\n\t"
+        "{ .reg .b32 ln; mov.u32 ln, %%laneid; setp.eq.u32 e, ln, 0; }\n\t"
         "setp.ne.b32 p, %9, 0;\n\t"
         "setp.eq.b32 t, 0, 0;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %5, %10, [%11], [%12], p;\n\t"
@@ -173,9 +201,10 @@ __device__ __forceinline__ void mma4_mxf4_ts_commit(uint32_t d, uint32_t a0, uin
 __device__ __forceinline__ void mma8_mxf4_ts_commit(uint32_t d, uint32_t a0, uint64_t b0, uint32_t bstep,
                                                     uint32_t idesc, uint32_t accumulate, uint32_t sfa,
                                                     uint32_t sfb, uint64_t *bar) {
+    __syncwarp();   // warp-collective (.sync.aligned / elect.sync): converge first
     asm volatile(
         "{\n\t.reg .pred e, p, t;\n\t.reg .b64 bd;\n\t.reg .b32 ad;\n\t"
-        "elect.sync _|e, 0xffffffff;\n\t"
+        "{ .reg .b32 ln; mov.u32 ln, %%laneid; setp.eq.u32 e, ln, 0; }\n\t"
         "setp.ne.b32 p, %5, 0;\n\t"
         "setp.eq.b32 t, 0, 0;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %4, [%6], [%7], p;\n\t"
@@ -199,10 +228,30 @@ __device__ __forceinline__ void mma8_mxf4_ts_commit(uint32_t d, uint32_t a0, uin
         : "memory");
 }
 
+// Four K-steps of tcgen05.mma kind::mxf4 (A from TMEM) without a commit; one elected lane.
+__device__ __forceinline__ void mma4_mxf4_ts(uint32_t d, uint32_t a0, uint64_t b0, uint32_t bstep, uint32_t idesc,
+                                             uint32_t accumulate, uint32_t sfa, uint32_t sfb) {
+    __syncwarp();   // warp-collective (.sync.aligned / elect.sync): converge first
+    const uint64_t b1 = b0 + bstep, b2 = b0 + 2 * bstep, b3 = b0 + 3 * bstep;
+    asm volatile(
+        "{\n\t.reg .pred e, p, t;\n\t"
+        "{ .reg .b32 ln; mov.u32 ln, %%laneid; setp.eq.u32 e, ln, 0; }\n\t"
+        "setp.ne.b32 p, %9, 0;\n\t"
+        "setp.eq.b32 t, 0, 0;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %5, %10, [%11], [%12], p;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%2], %6, %10, [%11], [%12], t;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%3], %7, %10, [%11], [%12], t;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%4], %8, %10, [%11], [%12], t;\n\t}" ::"r"(d),
+        "r"(a0), "r"(a0 + 8), "r"(a0 + 16), "r"(a0 + 24), "l"(b0), "l"(b1), "l"(b2), "l"(b3), "r"(accumulate),
+        "r"(idesc), "r"(sfa), "r"(sfb)
+        : "memory");
+}
+
 // Commit by one elected lane of a converged warp.
 __device__ __forceinline__ void mma_commit_elect(uint64_t *bar) {
+    __syncwarp();   // warp-collective (.sync.aligned / elect.sync): converge first
     asm volatile(
-        "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "{\n\t.reg .pred e;\n\t{ .reg .b32 ln; mov.u32 ln, %%laneid; setp.eq.u32 e, ln, 0; }\n\t"
         "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
         : "memory");
 }

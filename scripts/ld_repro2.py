@@ -1,0 +1,18 @@
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import snpgen
+import paper_conf_ipps_binderlp19_b200 as snp
+torch.cuda.set_device(0)
+m, nbits = int(os.environ.get("M", 32768)), 16384
+A = torch.empty((m, snp.snp_words(nbits)), dtype=torch.uint64, device="cuda")
+for r0 in range(0, m, 4096):
+    r1 = min(m, r0 + 4096)
+    snp.snp_pack(snpgen.ld_genotypes(1003, torch.arange(r0, r1, device="cuda"), nbits, structure=True, xp="torch", device="cuda"), out=A[r0:r1])
+torch.cuda.synchronize()
+print("packed", flush=True)
+for counts in (False, True):
+    pa = snp.snp_row_popc(A, nbits); torch.cuda.synchronize(); print("popc ok", flush=True)
+    r2, _, c = snp.snp_ld_r2(A, A, nbits, popA=pa, popB=pa, counts=counts)
+    torch.cuda.synchronize()
+    print("ld_r2 ok counts", counts, flush=True)

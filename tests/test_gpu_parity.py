@@ -288,3 +288,49 @@ def test_cfg3_ld_32k_sampled_rows(snp):
     ridx = torch.from_numpy(rows).to(DEV)
     assert np.array_equal(u32(cnt.view(torch.int32)[ridx]), n_ref)
     check_r2(r2[ridx].cpu().numpy(), r2_ref)
+
+
+@pytest.mark.parametrize("mode", ["counts", "r2"])
+def test_cfg3_ld_32k_full_cross_variant(snp, mode):
+    """Race detector at full configs[2] size: every one of the 2^30 LD counts of the
+    tensor-core kernel equals the CUDA-core kernel's (itself oracle-checked above).
+    This is a consistency property over all elements, complementing the sampled
+    oracle parity; repeated three times because pipeline races are intermittent."""
+    m, nbits = 32768, 16384
+    A = torch.empty((m, snp.snp_words(nbits)), dtype=torch.uint64, device=DEV)
+    for r0 in range(0, m, 4096):
+        gg = snpgen.ld_genotypes(1003, torch.arange(r0, r0 + 4096, device=DEV), nbits,
+                                 structure=True, xp="torch", device=DEV)
+        snp.snp_pack(gg, out=A[r0:r0 + 4096])
+    _variant(snp, "popc")
+    ref = snp.snp_ld_counts(A, A, nbits).view(torch.int32)
+    _variant(snp, "tc")
+    try:
+        for _ in range(3):
+            if mode == "counts":
+                got = snp.snp_ld_counts(A, A, nbits)
+            else:
+                _, _, got = snp.snp_ld_r2(A, A, nbits, counts=True)
+            assert snp.snp_last_kernel() == "tc_mxf4"
+            assert int((got.view(torch.int32) != ref).sum().item()) == 0
+            del got
+    finally:
+        _variant(snp, "auto")
+
+
+def test_cfg2_fastid_full_cross_variant(snp):
+    """Same race check for the FastID kernel at configs[1] size, all 6.4e7 outputs, XOR."""
+    nq, nd, nbits, seed = 64, 1_000_000, 4096, 1002
+    D = _gen_dev_fastid(seed, nd, nbits)
+    q, _ = snpgen.fastid_queries(seed, nq, nd, nbits)
+    Q = snp.snp_pack(to_dev(q))
+    _variant(snp, "popc")
+    ref = snp.snp_fastid(Q, D, nbits, "xor").view(torch.int32)
+    _variant(snp, "tc")
+    try:
+        for _ in range(3):
+            got = snp.snp_fastid(Q, D, nbits, "xor")
+            assert snp.snp_last_kernel() == "fastid_mxf4"
+            assert int((got.view(torch.int32) != ref).sum().item()) == 0
+    finally:
+        _variant(snp, "auto")
