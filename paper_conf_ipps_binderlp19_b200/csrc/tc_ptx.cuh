@@ -172,9 +172,9 @@ __device__ __forceinline__ void mma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, uint
 }
 
 // Four K-steps of tcgen05.mma kind::mxf4 (block32 scales) with A from TMEM, then a
-// commit to `bar`, issued by lane 0 of a converged warp (the whole warp must call it).
-// All MMAs and commits of a kernel are issued by the same lane: tcgen05.commit only
-// tracks the async operations of the thread that executes it.  K-step i uses A columns a0 + 8 i and B descriptor b0 + i * bstep
+// commit to `bar`, issued by the elect.sync leader of a converged warp (the whole warp
+// must call it; the wrapper re-converges first, so the leader is always the same lane:
+// tcgen05.commit only tracks the async operations of the thread that executes it).  K-step i uses A columns a0 + 8 i and B descriptor b0 + i * bstep
 // (descriptor start-address field, 16-byte units).  The first MMA accumulates iff
 // `accumulate`; the other three always accumulate.
 __device__ __forceinline__ void mma4_mxf4_ts_commit(uint32_t d, uint32_t a0, uint64_t b0, uint32_t bstep,
@@ -184,7 +184,7 @@ __device__ __forceinline__ void mma4_mxf4_ts_commit(uint32_t d, uint32_t a0, uin
     const uint64_t b1 = b0 + bstep, b2 = b0 + 2 * bstep, b3 = b0 + 3 * bstep;
     asm volatile(
         "{\n\t.reg .pred e, p, t;\n\t"
-        "{ .reg .b32 ln; mov.u32 ln, %%laneid; setp.eq.u32 e, ln, 0; }\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
         "setp.ne.b32 p, %9, 0;\n\t"
         "setp.eq.b32 t, 0, 0;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %5, %10, [%11], [%12], p;\n\t"
@@ -204,7 +204,7 @@ __device__ __forceinline__ void mma8_mxf4_ts_commit(uint32_t d, uint32_t a0, uin
     __syncwarp();   // warp-collective (.sync.aligned / elect.sync): converge first
     asm volatile(
         "{\n\t.reg .pred e, p, t;\n\t.reg .b64 bd;\n\t.reg .b32 ad;\n\t"
-        "{ .reg .b32 ln; mov.u32 ln, %%laneid; setp.eq.u32 e, ln, 0; }\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
         "setp.ne.b32 p, %5, 0;\n\t"
         "setp.eq.b32 t, 0, 0;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %4, [%6], [%7], p;\n\t"
@@ -235,7 +235,7 @@ __device__ __forceinline__ void mma4_mxf4_ts(uint32_t d, uint32_t a0, uint64_t b
     const uint64_t b1 = b0 + bstep, b2 = b0 + 2 * bstep, b3 = b0 + 3 * bstep;
     asm volatile(
         "{\n\t.reg .pred e, p, t;\n\t"
-        "{ .reg .b32 ln; mov.u32 ln, %%laneid; setp.eq.u32 e, ln, 0; }\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
         "setp.ne.b32 p, %9, 0;\n\t"
         "setp.eq.b32 t, 0, 0;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %5, %10, [%11], [%12], p;\n\t"
