@@ -153,11 +153,16 @@ def dist_setup(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    import torch
+    local = local % max(1, torch.cuda.device_count())   # (several ranks per GPU only in logic tests)
     if world > 1:
-        import torch
         import torch.distributed as dist
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")   # gloo: multi-rank logic test on 1 GPU
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     return rank, world, local
 
 
@@ -260,8 +265,9 @@ def setup_fastid(wl, rank, world, dev):
             for op in outs}
     ws = {op: (torch.empty(snp.snp_fastid_workspace_bytes(nq, nd, nbits, op), dtype=torch.uint8, device=dev))
           for op in outs}
-    gathered = {op: (torch.empty(world * nq, dtype=torch.uint32, device=dev),
+    gathered = {op: (torch.empty(world * nq, dtype=torch.int32, device=dev),
                      torch.empty(world * nq, dtype=torch.int64, device=dev)) for op in outs}
+    merged = {}
     res_host = {op: (torch.empty(nq, dtype=torch.uint32).pin_memory(), torch.empty(nq, dtype=torch.int64).pin_memory())
                 for op in outs}
     st = dict(D=D, Q=Q, qbytes=qbytes, qhost=qhost, outs=outs, best=best, ws=ws, lo=lo, nd=nd,
@@ -277,7 +283,7 @@ def setup_fastid(wl, rank, world, dev):
             snp.snp_pack(qbytes, nbits=nbits, out=Q)                       # a1
         if world > 1:
             import torch.distributed as dist
-            dist.broadcast(Q, src=0)                                       # queries -> all ranks
+            dist.broadcast(Q.view(torch.int64), src=0)                     # queries -> all ranks
         for i, op in enumerate(("xor", "andnot")):
             if kev is not None:
                 kev[2 * i].record(s)
@@ -288,9 +294,12 @@ def setup_fastid(wl, rank, world, dev):
             snp.snp_fastid_best(outs[op], index_base=lo, best_count=bc, best_index=bi)          # a6
             if world > 1:
                 import torch.distributed as dist
+                from paper_conf_ipps_binderlp19_b200 import multigpu
                 gc, gi = gathered[op]
-                dist.all_gather_into_tensor(gc, bc)
+                dist.all_gather_into_tensor(gc, bc.view(torch.int32))
                 dist.all_gather_into_tensor(gi, bi)
+                # global best per query, lowest global index on ties
+                merged[op] = multigpu.merge_best(gc.view(world, nq).to(torch.int64), gi.view(world, nq))
             if host:   # e2e: D2H of the step's result (per-query best count and index)
                 res_host[op][0].copy_(bc, non_blocking=True)
                 res_host[op][1].copy_(bi, non_blocking=True)
@@ -348,7 +357,7 @@ def setup_ld(wl, rank, world, dev):
             snp.snp_pack(G, nbits=nbits, out=B)                            # a1
         if world > 1:
             import torch.distributed as dist
-            dist.broadcast(B, src=0)
+            dist.broadcast(B.view(torch.int64), src=0)
         if kev is not None:
             kev[0].record(s)
         snp.snp_ld_r2(B[lo:hi], B, nbits, r2=r2, counts=cnt, ws=ws)       # a2 + a3 + a5

@@ -51,7 +51,7 @@ def fastid_step(Q: torch.Tensor, D_shard: torch.Tensor, nbits: int, op: str, ind
     best = best or (lambda c_, base_: snp_fastid_best(c_, index_base=base_))
     world = dist.get_world_size(group) if dist.is_initialized() else 1
     if world > 1:
-        dist.broadcast(Q, src=0, group=group)
+        dist.broadcast(Q.view(torch.int64) if Q.dtype == torch.uint64 else Q, src=0, group=group)
     counts = compute(Q, D_shard, out)
     bc, bi = best(counts, index_base)
     if world == 1:
@@ -72,5 +72,5 @@ def ld_step(B: torch.Tensor, nbits: int, lo: int, hi: int, compute=None, group=N
     compute = compute or (lambda A_, B_: snp_ld_r2(A_, B_, nbits, counts=True))
     world = dist.get_world_size(group) if dist.is_initialized() else 1
     if world > 1:
-        dist.broadcast(B, src=0, group=group)
+        dist.broadcast(B.view(torch.int64) if B.dtype == torch.uint64 else B, src=0, group=group)
     return compute(B[lo:hi], B)
