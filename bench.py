@@ -6,9 +6,11 @@
 
 A *step* is one pass of the whole hot path over one batch:
   fastid*: a1 pack the query batch -> (N>1: NCCL broadcast of the packed queries)
-           -> a3+a4 snp_fastid XOR (identity search, Eq. 2) and ANDNOT (mixture
-           analysis, Eq. 3) over the resident packed database -> a6 best match per
-           query for both (N>1: all-gather of the per-shard bests).
+           -> a3+a4+a6 ONE snp_fastid_search pass over the resident packed database
+           giving XOR (identity search, Eq. 2) and ANDNOT (mixture analysis, Eq. 3)
+           count matrices and the best match per query for both (N>1: all-gather of
+           the per-shard bests).  --fastid-step separate runs snp_fastid +
+           snp_fastid_best per op instead (two database passes + two count re-reads).
   ld*:     a1 pack the genotype matrix -> (N>1: NCCL broadcast of the packed
            matrix) -> a2 row popcounts + a3 AND-count GEMM + a5 r2 epilogue
            (counts and r2 written) for this rank's row block.
@@ -56,6 +58,9 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-graph", dest="graph", action="store_false",
                    help="run the timed steps eagerly instead of replaying a captured CUDA graph")
+    p.add_argument("--fastid-step", default="fused", choices=["fused", "separate"],
+                   help="fused: one snp_fastid_search pass for XOR+ANDNOT counts and best matches; "
+                        "separate: snp_fastid + snp_fastid_best per op")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target oracle CPU time")
     a = p.parse_args()
     if a.warmup < 3:
@@ -229,6 +234,8 @@ def cpu_baseline(wl, seconds, cores=None):
 
 # ----------------------------------------------------------------------------- workloads
 
+FASTID_STEP = "fused"
+
 def _gen_fastid_db(snp, snpgen, torch, seed, row0, rows, nbits, dev, chunk=32768):
     D = torch.empty((rows, snp.snp_words(nbits)), dtype=torch.uint64, device=dev)
     for r0 in range(0, rows, chunk):
@@ -260,20 +267,37 @@ def setup_fastid(wl, rank, world, dev):
     qbytes = torch.from_numpy(np.ascontiguousarray(q)).to(dev)
     qhost = torch.from_numpy(np.ascontiguousarray(q)).pin_memory()
     Q = torch.empty((nq, snp.snp_words(nbits)), dtype=torch.uint64, device=dev)
-    outs = {op: torch.empty((nq, nd), dtype=torch.uint32, device=dev) for op in ("xor", "andnot")}
+    OPS = ("xor", "andnot")
+    fused = FASTID_STEP == "fused"
+    outs = {op: torch.empty((nq, nd), dtype=torch.uint32, device=dev) for op in OPS}
     best = {op: (torch.empty(nq, dtype=torch.uint32, device=dev), torch.empty(nq, dtype=torch.int64, device=dev))
-            for op in outs}
-    ws = {op: (torch.empty(snp.snp_fastid_workspace_bytes(nq, nd, nbits, op), dtype=torch.uint8, device=dev))
-          for op in outs}
+            for op in OPS}
+    if fused:
+        ws = torch.empty(snp.snp_fastid_search_workspace_bytes(nq, nd, nbits, len(OPS)), dtype=torch.uint8,
+                         device=dev)
+    else:
+        ws = {op: (torch.empty(snp.snp_fastid_workspace_bytes(nq, nd, nbits, op), dtype=torch.uint8, device=dev))
+              for op in OPS}
     gathered = {op: (torch.empty(world * nq, dtype=torch.int32, device=dev),
-                     torch.empty(world * nq, dtype=torch.int64, device=dev)) for op in outs}
+                     torch.empty(world * nq, dtype=torch.int64, device=dev)) for op in OPS}
     merged = {}
     res_host = {op: (torch.empty(nq, dtype=torch.uint32).pin_memory(), torch.empty(nq, dtype=torch.int64).pin_memory())
-                for op in outs}
+                for op in OPS}
     st = dict(D=D, Q=Q, qbytes=qbytes, qhost=qhost, outs=outs, best=best, ws=ws, lo=lo, nd=nd,
               gathered=gathered, res_host=res_host)
     cmp_rank = 2 * nq * nd * nbits
     cmp_all = 2 * nq * (nd_total if wl["scaling"] == "strong" else wl["nd"] * world) * nbits
+
+    def _search():
+        # a3 + a4 + a6 for both ops in ONE pass over the resident database (f1)
+        snp.snp_fastid_search(Q, D, nbits, OPS, counts=[outs[op] for op in OPS],
+                              best=[best[op] for op in OPS], index_base=lo, ws=ws)
+
+    def _fast(op):
+        return lambda: snp.snp_fastid(Q, D, nbits, op, out=outs[op], ws=ws[op] if ws[op].numel() else None)
+
+    def _best(op):
+        return lambda: snp.snp_fastid_best(outs[op], index_base=lo, best_count=best[op][0], best_index=best[op][1])
 
     def step(kev=None, host=False):
         s = torch.cuda.current_stream()
@@ -284,14 +308,22 @@ def setup_fastid(wl, rank, world, dev):
         if world > 1:
             import torch.distributed as dist
             dist.broadcast(Q.view(torch.int64), src=0)                     # queries -> all ranks
-        for i, op in enumerate(("xor", "andnot")):
+        if fused:
             if kev is not None:
-                kev[2 * i].record(s)
-            snp.snp_fastid(Q, D, nbits, op, out=outs[op], ws=ws[op] if ws[op].numel() else None)  # a3+a4
+                kev[0].record(s)
+            _search()
             if kev is not None:
-                kev[2 * i + 1].record(s)
+                kev[1].record(s)
+        else:   # one snp_fastid + snp_fastid_best per op (two database passes)
+            for i, op in enumerate(OPS):
+                if kev is not None:
+                    kev[2 * i].record(s)
+                _fast(op)()                                                # a3+a4
+                if kev is not None:
+                    kev[2 * i + 1].record(s)
+                _best(op)()                                                # a6
+        for op in OPS:
             bc, bi = best[op]
-            snp.snp_fastid_best(outs[op], index_base=lo, best_count=bc, best_index=bi)          # a6
             if world > 1:
                 import torch.distributed as dist
                 from paper_conf_ipps_binderlp19_b200 import multigpu
@@ -305,18 +337,19 @@ def setup_fastid(wl, rank, world, dev):
                 res_host[op][1].copy_(bi, non_blocking=True)
 
     # the same device-resident step as separately capturable parts (N=1 graph mode)
-    def _fast(op):
-        return lambda: snp.snp_fastid(Q, D, nbits, op, out=outs[op], ws=ws[op] if ws[op].numel() else None)
-
-    def _best(op):
-        return lambda: snp.snp_fastid_best(outs[op], index_base=lo, best_count=best[op][0], best_index=best[op][1])
-    parts = [(lambda: snp.snp_pack(qbytes, nbits=nbits, out=Q), False),
-             (_fast("xor"), True), (_best("xor"), False), (_fast("andnot"), True), (_best("andnot"), False)]
+    pack_part = (lambda: snp.snp_pack(qbytes, nbits=nbits, out=Q), False)
+    if fused:
+        parts = [pack_part, (_search, True)]
+    else:
+        parts = [pack_part, (_fast("xor"), True), (_best("xor"), False), (_fast("andnot"), True),
+                 (_best("andnot"), False)]
 
     # algorithmic bytes of the dominant kernel per launch: DB + queries read, counts written
     words = (nbits + 63) // 64
-    alg_bytes = (nd + nq) * words * 8 + nq * nd * 4
-    return dict(step=step, parts=parts, cmp_rank=cmp_rank, cmp_all=cmp_all, kernel_launches_per_step=2,
+    nout = len(OPS) if fused else 1
+    alg_bytes = (nd + nq) * words * 8 + nout * nq * nd * 4
+    return dict(step=step, parts=parts, cmp_rank=cmp_rank, cmp_all=cmp_all,
+                kernel_launches_per_step=1 if fused else 2, step_mode=FASTID_STEP,
                 kernel_cmp=nq * nd * nbits, kernel_bytes=alg_bytes,
                 h2d=nq * nbits, d2h=2 * nq * 12, l2_flush=False,
                 l2_note=f"inputs larger than L2 ({nd * snp.snp_words(nbits) * 8 / 1e6:.0f} MB database per rank)",
@@ -470,6 +503,8 @@ def run_ours(args):
     import paper_conf_ipps_binderlp19_b200 as snp
     snp.snp_set_variant(args.variant)
     steps = args.steps or (200 if wl["kind"] == "fastid" else 20)
+    global FASTID_STEP
+    FASTID_STEP = args.fastid_step
     wlrun = (setup_fastid if wl["kind"] == "fastid" else setup_ld)(wl, rank, world, dev)
     torch.cuda.synchronize()
 
@@ -555,6 +590,7 @@ def run_ours(args):
             "config": {"workload": args.workload, "desc": wl["desc"],
                        **{k: v for k, v in wl.items() if k in ("nq", "nd", "m", "nbits")},
                        "variant": variant, "kernel": kernel, "l2": wlrun["l2_note"],
+                       **({"step": wlrun["step_mode"]} if "step_mode" in wlrun else {}),
                        "launch": "cuda-graph replay per step" if use_graph else "eager",
                        "parallelism": f"{'db' if wl['kind'] == 'fastid' else 'row'}-shard x{world}"},
             "word_ops_per_s": value / 64, "tops_eq": 2 * value / 1e12,

@@ -145,6 +145,30 @@ snp_status snp_fastid_best(const uint32_t *counts, int64_t nq, int64_t nd, int64
                            int64_t index_base, uint32_t *best_count, int64_t *best_index,
                            void *stream);
 
+/* f1 — fused FastID search (P:L54-78 for the ops, P:L58/L62 for the
+ * decision): ONE pass over the database computes, for each of the nops (1..4) ops in
+ * ops[] (a HOST array of snp_op), the count matrix of snp_fastid and/or the per-query
+ * best match of snp_fastid_best, without the counts being re-read (or written at all
+ * when only best matches are wanted).  All ops derive from the one AND count of a
+ * (query, row) pair, so XOR and ANDNOT together cost one database pass, not two.
+ *   counts:     HOST array of nops device pointers (or NULL = none); counts[j] is
+ *               uint32 [nq][ldo] for ops[j] as in snp_fastid (overwritten), or NULL.
+ *   best_count, best_index: HOST arrays of nops device pointers (both arrays NULL =
+ *               no best matches); entry j is uint32 [nq] / int64 [nq] (both NULL or
+ *               both set): min count over the nd rows and index_base + lowest row
+ *               attaining it (R4); nd == 0 gives 0xFFFFFFFF / -1.
+ * nd < 2^32 - 1.  ws: snp_fastid_search_workspace_bytes(nq, nd, nbits, nops) bytes
+ * (never 0 when nq > 0).  Kernels: the fused tcgen05 kernel for nq <= 64 (two or three
+ * launches: key init + search [+ pack by the caller]); other shapes / a forced
+ * SNP_VARIANT_POPC compose snp_fastid's kernels with best.cu per op, chunking the
+ * database through workspace counts when counts[j] is NULL. */
+size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int nops);
+snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
+                             const uint64_t *D, int64_t nd, int64_t ldd, int64_t nbits,
+                             int nops, const int *ops, uint32_t *const *counts, int64_t ldo,
+                             uint32_t *const *best_count, int64_t *const *best_index,
+                             int64_t index_base, void *ws, size_t ws_bytes, void *stream);
+
 /* e — multi-GPU row partition (host only, no device access): rows [0, rows)
  * split into `world` contiguous ranges bounds[r] .. bounds[r+1] (bounds is a
  * HOST array of world+1 int64), each boundary a multiple of `align` (except

@@ -20,7 +20,8 @@ from ._lib import SnpError, check, lib, status_string  # noqa: F401
 __all__ = [
     "SnpError", "OPS", "VARIANTS", "snp_words", "snp_ld_workspace_bytes",
     "snp_fastid_workspace_bytes", "snp_pack", "snp_row_popc", "snp_ld_counts",
-    "snp_ld_r2", "snp_fastid", "snp_fastid_best", "snp_shard_plan", "snp_set_variant",
+    "snp_ld_r2", "snp_fastid", "snp_fastid_best", "snp_fastid_search",
+    "snp_fastid_search_workspace_bytes", "snp_shard_plan", "snp_set_variant",
     "snp_last_variant", "snp_last_kernel", "snp_launch_count", "status_string",
 ]
 
@@ -199,6 +200,63 @@ def snp_fastid_best(counts: torch.Tensor, index_base: int = 0, nd: int | None = 
     check(lib().snp_fastid_best(_ptr(counts), nq, nd, _ld(counts), int(index_base), _ptr(best_count),
                                 _ptr(best_index), _stream(stream)), "snp_fastid_best")
     return best_count, best_index
+
+
+def snp_fastid_search_workspace_bytes(nq: int, nd: int, nbits: int, nops: int) -> int:
+    return int(lib().snp_fastid_search_workspace_bytes(int(nq), int(nd), int(nbits), int(nops)))
+
+
+def snp_fastid_search(Q: torch.Tensor, D: torch.Tensor, nbits: int, ops=("xor", "andnot"),
+                      counts=True, best=True, index_base: int = 0, ldo: int | None = None,
+                      ws: torch.Tensor | None = None, stream=None):
+    """f1: one pass over D for every op in ops -> (counts list, best list).
+
+    counts: True (allocate [nq][nd] uint32 per op), False (none) or a list of
+    tensors/None per op.  best: True/False or a list of (best_count, best_index)
+    pairs / None per op.  Returns (counts_list, best_list), entries None where not
+    requested."""
+    _dev_tensor(Q, "Q", _WORD_DTYPES)
+    _dev_tensor(D, "D", _WORD_DTYPES)
+    if isinstance(ops, (str, int)):
+        ops = (ops,)
+    opi = [_op(o) for o in ops]
+    k = len(opi)
+    nq, nd = Q.shape[0], D.shape[0]
+    dev = Q.device
+    if counts is True:
+        counts = [torch.empty((nq, nd if ldo is None else ldo), dtype=torch.uint32, device=dev) for _ in opi]
+    elif counts is False or counts is None:
+        counts = [None] * k
+    if best is True:
+        best = [(torch.empty(nq, dtype=torch.uint32, device=dev), torch.empty(nq, dtype=torch.int64, device=dev))
+                for _ in opi]
+    elif best is False or best is None:
+        best = [None] * k
+    if len(counts) != k or len(best) != k:
+        raise ValueError("counts / best must have one entry per op")
+    for c in counts:
+        _dev_tensor(c, "counts", _U32)
+    for b in best:
+        if b is not None:
+            _dev_tensor(b[0], "best_count", _U32)
+            _dev_tensor(b[1], "best_index", (torch.int64,))
+    ld = next((_ld(c) for c in counts if c is not None), nd if ldo is None else int(ldo))
+    P = ctypes.c_void_p * k
+    ops_arr = (ctypes.c_int * k)(*opi)
+    c_arr = P(*[_ptr(c) for c in counts])
+    bc_arr = P(*[_ptr(None if b is None else b[0]) for b in best])
+    bi_arr = P(*[_ptr(None if b is None else b[1]) for b in best])
+    need = snp_fastid_search_workspace_bytes(nq, nd, nbits, k)
+    if ws is None:
+        ws = _workspace(need, dev)
+    any_best = any(b is not None for b in best)
+    check(lib().snp_fastid_search(_ptr(Q), nq, _ld(Q), _ptr(D), nd, _ld(D), int(nbits), k,
+                                  ctypes.cast(ops_arr, ctypes.c_void_p), ctypes.cast(c_arr, ctypes.c_void_p), ld,
+                                  ctypes.cast(bc_arr, ctypes.c_void_p) if any_best else None,
+                                  ctypes.cast(bi_arr, ctypes.c_void_p) if any_best else None,
+                                  int(index_base), _ptr(ws), 0 if ws is None else ws.numel(), _stream(stream)),
+          "snp_fastid_search")
+    return counts, best
 
 
 def snp_shard_plan(rows: int, world: int, align: int = 128) -> list[int]:

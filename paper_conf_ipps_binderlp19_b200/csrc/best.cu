@@ -27,7 +27,7 @@ __device__ __forceinline__ unsigned long long kmin(unsigned long long a, unsigne
 }
 
 __global__ void __launch_bounds__(BT) best_reduce(const uint32_t *__restrict__ c, int64_t nd,
-                                                  int64_t ldo, unsigned long long *keys) {
+                                                  int64_t ldo, int64_t jbase, unsigned long long *keys) {
     const int64_t i = blockIdx.y;
     const int64_t j0 = (int64_t)blockIdx.x * PER_BLOCK;
     const int64_t j1 = j0 + PER_BLOCK < nd ? j0 + PER_BLOCK : nd;
@@ -39,17 +39,17 @@ __global__ void __launch_bounds__(BT) best_reduce(const uint32_t *__restrict__ c
         const uint4 *p = reinterpret_cast<const uint4 *>(row + j0);
         for (int64_t v = threadIdx.x; v < nv; v += BT) {
             const uint4 x = __ldg(p + v);
-            const unsigned long long j = (unsigned long long)(j0 + 4 * v);
+            const unsigned long long j = (unsigned long long)(jbase + j0 + 4 * v);
             best = kmin(best, ((unsigned long long)x.x << 32) | j);
             best = kmin(best, ((unsigned long long)x.y << 32) | (j + 1));
             best = kmin(best, ((unsigned long long)x.z << 32) | (j + 2));
             best = kmin(best, ((unsigned long long)x.w << 32) | (j + 3));
         }
         for (int64_t j = j0 + 4 * nv + threadIdx.x; j < j1; j += BT)
-            best = kmin(best, ((unsigned long long)row[j] << 32) | (unsigned long long)j);
+            best = kmin(best, ((unsigned long long)row[j] << 32) | (unsigned long long)(jbase + j));
     } else {
         for (int64_t j = j0 + threadIdx.x; j < j1; j += BT)
-            best = kmin(best, ((unsigned long long)row[j] << 32) | (unsigned long long)j);
+            best = kmin(best, ((unsigned long long)row[j] << 32) | (unsigned long long)(jbase + j));
     }
 #pragma unroll
     for (int o = 16; o; o >>= 1) best = kmin(best, __shfl_xor_sync(0xffffffffu, best, o));
@@ -62,11 +62,11 @@ __global__ void __launch_bounds__(BT) best_reduce(const uint32_t *__restrict__ c
     }
 }
 
-__global__ void best_finalize(int64_t nq, int64_t index_base, uint32_t *best_count,
-                              int64_t *best_index) {
+__global__ void best_finalize(const unsigned long long *keys, int64_t nq, int64_t index_base,
+                              uint32_t *best_count, int64_t *best_index) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nq;
          i += (int64_t)gridDim.x * blockDim.x) {
-        const unsigned long long k = reinterpret_cast<unsigned long long *>(best_index)[i];
+        const unsigned long long k = keys[i];   // read before best_index (may alias keys) is written
         if (k == ~0ULL) {
             best_count[i] = 0xffffffffu;
             best_index[i] = -1;
@@ -77,33 +77,49 @@ __global__ void best_finalize(int64_t nq, int64_t index_base, uint32_t *best_cou
     }
 }
 
+int small_grid(int64_t n) { return (int)((n + 255) / 256 < 1024 ? (n + 255) / 256 : 1024); }
+
 }  // namespace
 
+cudaError_t launch_best_init(unsigned long long *keys, int64_t n, cudaStream_t s) {
+    best_init<<<small_grid(n), 256, 0, s>>>(n, keys);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_best_reduce(const uint32_t *counts, int64_t nq, int64_t nd, int64_t ldo, int64_t jbase,
+                               unsigned long long *keys, cudaStream_t s) {
+    if (nd <= 0) return cudaSuccess;
+    const int64_t gx = (nd + PER_BLOCK - 1) / PER_BLOCK;
+    int64_t done = 0;
+    while (done < nq) {   // gridDim.y <= 65535
+        const int64_t chunk = nq - done < 65535 ? nq - done : 65535;
+        dim3 grid((unsigned)gx, (unsigned)chunk);
+        best_reduce<<<grid, BT, 0, s>>>(counts + done * ldo, nd, ldo, jbase, keys + done);
+        count_launches(1);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        done += chunk;
+    }
+    return cudaSuccess;
+}
+
+cudaError_t launch_best_finalize(const unsigned long long *keys, int64_t nq, int64_t index_base,
+                                 uint32_t *best_count, int64_t *best_index, cudaStream_t s) {
+    best_finalize<<<small_grid(nq), 256, 0, s>>>(keys, nq, index_base, best_count, best_index);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+// snp_fastid_best: best_index doubles as the key scratch, so nothing is allocated.
 cudaError_t launch_best(const uint32_t *counts, int64_t nq, int64_t nd, int64_t ldo,
                         int64_t index_base, uint32_t *best_count, int64_t *best_index,
                         cudaStream_t s) {
     unsigned long long *keys = reinterpret_cast<unsigned long long *>(best_index);
-    const int sb = (int)((nq + 255) / 256 < 1024 ? (nq + 255) / 256 : 1024);
-    best_init<<<sb, 256, 0, s>>>(nq, keys);
-    count_launches(1);
-    cudaError_t e = cudaGetLastError();
+    cudaError_t e = launch_best_init(keys, nq, s);
     if (e != cudaSuccess) return e;
-    if (nd > 0) {
-        int64_t gx = (nd + PER_BLOCK - 1) / PER_BLOCK;
-        int64_t done = 0;
-        while (done < nq) {   // gridDim.y <= 65535
-            const int64_t chunk = nq - done < 65535 ? nq - done : 65535;
-            dim3 grid((unsigned)gx, (unsigned)chunk);
-            best_reduce<<<grid, BT, 0, s>>>(counts + done * ldo, nd, ldo, keys + done);
-            count_launches(1);
-            e = cudaGetLastError();
-            if (e != cudaSuccess) return e;
-            done += chunk;
-        }
-    }
-    best_finalize<<<sb, 256, 0, s>>>(nq, index_base, best_count, best_index);
-    count_launches(1);
-    return cudaGetLastError();
+    if ((e = launch_best_reduce(counts, nq, nd, ldo, 0, keys, s)) != cudaSuccess) return e;
+    return launch_best_finalize(keys, nq, index_base, best_count, best_index, s);
 }
 
 }  // namespace snp

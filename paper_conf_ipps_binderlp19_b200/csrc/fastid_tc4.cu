@@ -63,14 +63,30 @@ struct FCfg {
     static_assert(SF_COL + 32 <= 512, "TMEM budget");
 };
 
+// Epilogue of one launch: up to 4 comparison ops, all derived from the one AND count c of
+// a (query, database row) pair by  x = cq * pQ + cd * pD + cc * c:
+//   AND (0,0,1), XOR (1,1,-2), ANDNOT (1,0,-1), NOTAND (0,1,-1)   [uint32 wrap-around].
+// Per op, the counts are stored (outs[j] != NULL) and/or the per-query best match is
+// kept (best bit j): running (min count, lowest row) per query column in registers,
+// merged across warps and CTAs by a 64-bit atomicMin on (count << 32 | row) keys.
+constexpr int MAXOPS = 4;
+
 struct FArgs {
     const uint32_t *Q;   // queries (column side), packed u32 view
     int64_t nq, ldq32;
     int64_t nd;          // database rows (lane side)
     int64_t nbits;
-    int op, accumulate;
+    int nops;
+    uint32_t cq[MAXOPS], cd[MAXOPS], cc[MAXOPS];
+    uint32_t *outs[MAXOPS];
+    int accumulate;
     int64_t ldo;
-    uint32_t *out;
+    int best_mask;                       // bit j: keep the best match of op j
+    unsigned long long *keys;            // [nops][nq] (count << 32 | local row), pre-set to ~0
+    unsigned int *done;                  // CTA completion counter, pre-set to 0
+    uint32_t *best_count[MAXOPS];        // [nq] per op with a best bit
+    int64_t *best_index[MAXOPS];
+    int64_t index_base;
     int64_t ntiles;
     int nst;
     size_t qbytes;       // expanded query bytes in shared memory
@@ -132,7 +148,19 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
         : "r"(taddr));
 }
 
-template <int BN, int OP>
+// NOPS: ops per launch; BEST: keep best matches; ACC: accumulate into the counts.
+// Everything uniform that would otherwise be tested inside the 32-column epilogue loop
+// is a template parameter or folded into per-lane predicates: loop unswitching on
+// runtime flags multiplied the code size (214 KB) and the instruction-cache misses
+// slowed every warp role 3x.
+// OPS >= 0: the ops are compile-time (op j in bits 2j..2j+1), so the epilogue key is two
+// shift/add instructions per (column, op) instead of two IMADs by runtime coefficients.
+// OPS = -1: coefficients from FArgs (any combination).
+__host__ __device__ constexpr uint32_t op_cq(int op) { return (op == 1 || op == 2) ? 1u : 0u; }
+__host__ __device__ constexpr uint32_t op_cd(int op) { return (op == 1 || op == 3) ? 1u : 0u; }
+__host__ __device__ constexpr uint32_t op_cc(int op) { return op == 0 ? 1u : op == 1 ? (uint32_t)-2 : (uint32_t)-1; }
+
+template <int BN, int NOPS, bool BEST, bool ACC, int OPS>
 __global__ void __launch_bounds__(NTHREADS, 1)
 fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     using C = FCfg<BN>;
@@ -151,6 +179,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popf + 2);
     uint32_t *popQ = tmem_slot + 4;          // [BN]
     uint32_t *popD = popQ + BN;              // [2 acc][G][BM]
+    uint32_t *popQ32 = popD + 2 * G * BM;    // [BN] 32 * popQ (epilogue key term)
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     __shared__ unsigned int launch_k;
@@ -217,6 +246,10 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     ptx::tc_fence_before();
     __syncthreads();
     ptx::tc_fence_after();
+    if (warp >= EPI_WARP0 && warp < EPI_WARP0 + NEPI) {   // only the epilogue warps read it
+        for (int r = tid - EPI_WARP0 * 32; r < BN; r += NEPI * 32) popQ32[r] = 32u * popQ[r];
+        asm volatile("bar.sync 1, %0;" ::"r"(NEPI * 32) : "memory");
+    }
 
     if (args.trace && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 1] = (long long)ptx::globaltimer_ns();
     if (warp == TMA_WARP) {
@@ -307,36 +340,40 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         publish_until(my_tiles);
     } else if (warp == MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
-        // The whole warp runs the loop (converged, uniform values); one elected lane issues
-        // the 4 MMAs of a stage and the commit in a single asm block.  Descriptors are
-        // precomputed: stepping K only adds to the start-address field.
+        // The whole warp runs the loop (converged, uniform values); the elected lane issues.
+        // Descriptors are precomputed: stepping K only adds to the start-address field.
+        // tmem was read from shared memory (a per-thread value to ptxas); a warp reduction
+        // lands it in a uniform register so everything derived from it stays uniform.
         constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
-        const uint32_t sfa = tmem + C::SF_COL, sfb = tmem + C::SF_COL + 16;
+        const uint32_t tmu = __reduce_or_sync(0xffffffffu, tmem);
+        const uint32_t sfa = tmu + C::SF_COL, sfb = tmu + C::SF_COL + 16;
         const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(qsm), BN * 16, 128);
         constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;           // one K-step = 2 chunks
         constexpr uint32_t SSTEP = ((KBITS / 32) * BN * 16) >> 4; // one stage = 16 chunks
+        // Waits are warp votes, so every loop value below is warp-uniform and lives in
+        // uniform registers: ~7 uniform instructions per MMA instead of ~16 with R2URs.
         int b = 0;
         uint32_t bround = 0;
         int64_t itm = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
-            if (tl >= 2) ptx::mbar_wait_warp(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            if (tl >= 2) ptx::mbar_wait_uniform(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
             ptx::tc_fence_after();
-            const uint32_t d = tmem + (uint32_t)(acc * C::ACC_COLS);
+            const uint32_t d = tmu + (uint32_t)(acc * C::ACC_COLS);
             uint64_t bd = bdesc0;
             for (int s = 0; s < nst; ++s, ++itm) {
-                ptx::mbar_wait_warp(&full[b], bround & 1);
-                const bool trm = args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024;
-                if (trm) g_fastid_trace[8 * itm + 3] = clock64();
+                ptx::mbar_wait_uniform(&full[b], bround & 1);
                 ptx::tc_fence_after();
-
-                ptx::mma8_mxf4_ts_commit(d, tmem + (uint32_t)(C::A_COL0 + 64 * b), bd, BSTEP, IDESC,
-                                         s != 0 ? 1u : 0u, sfa, sfb, &empty[b]);
-
+                const uint32_t a0 = tmu + (uint32_t)(C::A_COL0 + 64 * b);
+#pragma unroll
+                for (int k = 0; k < KBITS / 64; ++k)
+                    ptx::mma_mxf4_ts(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa,
+                                     sfb);
+                ptx::mma_commit_uniform(&empty[b]);
                 bd += SSTEP;
                 if (++b == NS) { b = 0; ++bround; }
             }
-            ptx::mma_commit_elect(&accf[acc]);
+            ptx::mma_commit_uniform(&accf[acc]);
         }
         __syncwarp();
     } else {
@@ -348,6 +385,10 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         const int c0 = 32 * h;
         const int ncols = (int)(args.nq - c0 < 32 ? (args.nq - c0 > 0 ? args.nq - c0 : 0) : 32);
         const int64_t ldo = args.ldo;
+        // running best of column c0 + lane, per op (held by that lane only)
+        uint32_t bc[NOPS], bi[NOPS];
+#pragma unroll
+        for (int j = 0; j < NOPS; ++j) { bc[j] = 0xffffffffu; bi[j] = 0xffffffffu; }
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
@@ -364,33 +405,104 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             ptx::tc_fence_before();
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&acce[acc]);   // accumulator + pops drained: reusable
-            const int64_t gd = t * BM + li;
-            if (gd < args.nd && ncols > 0 && !args.nostore) {
-                uint32_t *o = args.out + (int64_t)c0 * ldo + gd;
-                if (ncols == 32 && !args.accumulate) {
+            if (ncols == 0) continue;                      // nq <= 32: this column half is idle
+            const int64_t row0 = t * BM + q * 32;          // local database row of lane 0
+            const int64_t gd = row0 + lane;
+            const bool valid = gd < args.nd;
+            // Everything is computed as the 32x-scaled key of the best-match reduction:
+            //   key = 32 x + lane,  x = cq pQ + cd pD + cc c  (op identity)
+            // and the count c comes out of the fp32 accumulator by the 2^23 magic add
+            // (fb = bits(v + 2^23) = 0x4B000000 + c for 0 <= c < 2^23; FMA pipe, no F2I):
+            //   key = 32cc fb + cq (32 pQ) + [32 cd pD - 32 cc 0x4B000000 + lane]   (mod 2^32).
+            // Invalid rows (past nd) get +0xF0000000 instead of lane: larger than every real
+            // key (< 2^28), so they never win a reduction and are never stored.
+            const uint32_t laneterm = valid ? (uint32_t)lane : 0xF0000000u;
+            uint32_t L[NOPS], C32[NOPS];
+            bool sv[NOPS];
+            uint32_t *op_[NOPS];
 #pragma unroll
-                    for (int u = 0; u < 32; ++u) {
-                        const uint32_t c = __float2uint_rn(__uint_as_float(v[u]));
-                        uint32_t x;   // exact: every result is a count in [0, 2^31)
-                        if (OP == 0) x = c;
-                        else if (OP == 1) x = popQ[c0 + u] + pd - 2u * c;
-                        else if (OP == 2) x = popQ[c0 + u] - c;
-                        else x = pd - c;
-                        __stcs(o, x);          // streaming store: written once, never re-read here
-                        o += ldo;
-                    }
+            for (int j = 0; j < NOPS; ++j) {
+                if (OPS >= 0) {
+                    const int op = (OPS >> (2 * j)) & 3;
+                    C32[j] = 32u * op_cc(op);
+                    L[j] = 32u * op_cd(op) * pd - C32[j] * 0x4B000000u + laneterm;
                 } else {
+                    C32[j] = 32u * args.cc[j];
+                    L[j] = 32u * args.cd[j] * pd - C32[j] * 0x4B000000u + laneterm;
+                }
+                sv[j] = valid && args.outs[j] != nullptr && !args.nostore;
+                op_[j] = sv[j] ? args.outs[j] + (int64_t)c0 * ldo + gd : nullptr;
+            }
+            // best match: key = count << 5 | lane, so ONE redux.sync.min gives the tile
+            // quarter's minimum count and, among equal counts, its lowest row; lane u keeps
+            // column u's tile minimum and folds it into its running best once per tile
+            uint32_t mk[NOPS];
 #pragma unroll
-                    for (int u = 0; u < 32; ++u) {
-                        if (u >= ncols) break;
-                        const uint32_t c = __float2uint_rn(__uint_as_float(v[u]));
-                        uint32_t x;
-                        if (OP == 0) x = c;
-                        else if (OP == 1) x = popQ[c0 + u] + pd - 2u * c;
-                        else if (OP == 2) x = popQ[c0 + u] - c;
-                        else x = pd - c;
-                        *o = args.accumulate ? *o + x : x;
-                        o += ldo;
+            for (int j = 0; j < NOPS; ++j) mk[j] = 0xffffffffu;
+#pragma unroll
+            for (int u = 0; u < 32; ++u) {
+                const uint32_t fb = __float_as_uint(__fadd_rn(__uint_as_float(v[u]), 8388608.0f));
+                const uint32_t pq32 = popQ32[c0 + u];
+                const bool colok = u < ncols;
+#pragma unroll
+                for (int j = 0; j < NOPS; ++j) {
+                    uint32_t key;
+                    if (OPS >= 0) {
+                        const int op = (OPS >> (2 * j)) & 3;
+                        const uint32_t f32 = fb << 5;
+                        key = op == 0 ? f32 + L[j]                       // AND
+                            : op == 1 ? pq32 + L[j] - (f32 << 1)         // XOR
+                            : op == 2 ? pq32 + L[j] - f32                // ANDNOT
+                                      : L[j] - f32;                      // NOTAND
+                    } else {
+                        key = C32[j] * fb + (args.cq[j] * pq32 + L[j]);
+                    }
+                    if (sv[j] && colok) {
+                        const uint32_t x = key >> 5;   // valid rows: laneterm = lane < 32
+                        uint32_t *o = op_[j] + (int64_t)u * ldo;
+                        if (ACC) *o += x;
+                        else __stcs(o, x);   // streaming store: written once, never re-read here
+                    }
+                    if (BEST) {
+                        const uint32_t m = __reduce_min_sync(0xffffffffu, key);
+                        mk[j] = lane == u ? m : mk[j];
+                    }
+                }
+            }
+            if (BEST) {
+#pragma unroll
+                for (int j = 0; j < NOPS; ++j) {
+                    // tiles arrive in increasing row order: strict < keeps the lowest row
+                    if (mk[j] < 0xF0000000u && (mk[j] >> 5) < bc[j]) {
+                        bc[j] = mk[j] >> 5;
+                        bi[j] = (uint32_t)row0 + (mk[j] & 31u);
+                    }
+                }
+            }
+        }
+        if (BEST) {
+#pragma unroll
+            for (int j = 0; j < NOPS; ++j) {
+                if (((args.best_mask >> j) & 1) && lane < ncols && bc[j] != 0xffffffffu)
+                    atomicMin(args.keys + (int64_t)j * args.nq + c0 + lane,
+                              ((unsigned long long)bc[j] << 32) | bi[j]);
+            }
+            // the last epilogue warp of the grid to finish turns the merged keys into
+            // (best_count, best_index) (kept inside this role: a CTA-wide finalize after
+            // the role branches de-uniformised the MMA issue loop)
+            __threadfence();
+            uint32_t last = 0;
+            if (lane == 0) last = atomicAdd(args.done, 1u) == gridDim.x * NEPI - 1 ? 1u : 0u;
+            if (__shfl_sync(0xffffffffu, last, 0)) {
+                __threadfence();
+                const int nq = (int)args.nq;   // <= 64 (fastid_tc4_supported)
+#pragma unroll
+                for (int j = 0; j < NOPS; ++j) {
+                    if (!((args.best_mask >> j) & 1)) continue;
+                    for (int i = lane; i < nq; i += 32) {
+                        const unsigned long long k = __ldcg(args.keys + j * nq + i);
+                        args.best_count[j][i] = k == ~0ULL ? 0xffffffffu : (uint32_t)(k >> 32);
+                        args.best_index[j][i] = k == ~0ULL ? -1 : (int64_t)(k & 0xffffffffULL) + args.index_base;
                     }
                 }
             }
@@ -405,6 +517,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         ptx::tc_fence_after();
         ptx::tmem_dealloc<512>(tmem);
     }
+}
+
+__global__ void fastid_search_init(unsigned long long *keys, int64_t n, unsigned int *done) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        keys[i] = ~0ULL;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *done = 0u;
 }
 
 typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
@@ -439,20 +557,41 @@ size_t smem_bytes(int bn, int64_t nbits) {
     return (size_t)bn * (size_t)nst * (KBITS / 32) * 16 + NP * PSTAGE + 8192;   // + barriers, pops (~5 KB)
 }
 
+void op_coefs(int op, uint32_t &cq, uint32_t &cd, uint32_t &cc) {
+    // x = cq pQ + cd pD + cc AND  (uint32 wrap-around for the negatives)
+    switch (op) {
+    case 0: cq = 0; cd = 0; cc = 1; break;                   // AND      Eq. (1)
+    case 1: cq = 1; cd = 1; cc = (uint32_t)-2; break;        // XOR      Eq. (2)
+    case 2: cq = 1; cd = 0; cc = (uint32_t)-1; break;        // ANDNOT   Eq. (3), r = query
+    default: cq = 0; cd = 1; cc = (uint32_t)-1; break;       // NOTAND   Eq. (3), r = DB row
+    }
+}
+
 template <int BN>
-cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
+cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     // the database is the B operand of the user call (Q op D), on TMEM lanes here
     FArgs f{};
-    f.Q = a.A;
-    f.nq = a.m;
-    f.ldq32 = a.lda32;
-    f.nd = a.n;
+    f.Q = a.Q;
+    f.nq = a.nq;
+    f.ldq32 = a.ldq32;
+    f.nd = a.nd;
     f.nbits = a.nbits;
-    f.op = a.op;
+    f.nops = a.nops;
     f.accumulate = a.accumulate;
-    f.ldo = a.ldc;
-    f.out = a.C;
-    f.ntiles = (a.n + BM - 1) / BM;
+    f.ldo = a.ldo;
+    for (int j = 0; j < a.nops; ++j) {
+        op_coefs(a.ops[j], f.cq[j], f.cd[j], f.cc[j]);
+        f.outs[j] = a.counts[j];
+        if (a.best_count[j]) {
+            f.best_mask |= 1 << j;
+            f.best_count[j] = a.best_count[j];
+            f.best_index[j] = a.best_index[j];
+        }
+    }
+    f.keys = a.keys;
+    f.done = a.done;
+    f.index_base = a.index_base;
+    f.ntiles = (a.nd + BM - 1) / BM;
     f.nst = (int)((a.nbits + KBITS - 1) / KBITS);
     f.qbytes = (size_t)BN * f.nst * (KBITS / 32) * 16;
     static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
@@ -464,27 +603,59 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
     EncodeTiledFn enc = encode_fn();
     if (!enc) return cudaErrorNotSupported;
     CUtensorMap tm;
-    const cuuint64_t dims[2] = {(cuuint64_t)a.ldb32, (cuuint64_t)a.n};
-    const cuuint64_t strides[1] = {(cuuint64_t)a.ldb32 * 4};
+    const cuuint64_t dims[2] = {(cuuint64_t)a.ldd32, (cuuint64_t)a.nd};
+    const cuuint64_t strides[1] = {(cuuint64_t)a.ldd32 * 4};
     const cuuint32_t box[2] = {KBITS / 32, BM};
     const cuuint32_t estr[2] = {1, 1};
-    CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(a.B), dims, strides, box, estr,
+    CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(a.D), dims, strides, box, estr,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
 
-    void (*kern)(const CUtensorMap, const FArgs) = a.op == 0   ? fastid_tc4_kernel<BN, 0>
-                                                   : a.op == 1 ? fastid_tc4_kernel<BN, 1>
-                                                   : a.op == 2 ? fastid_tc4_kernel<BN, 2>
-                                                               : fastid_tc4_kernel<BN, 3>;
-    static size_t attr_set[4] = {0, 0, 0, 0};   // max dynamic smem already granted, per op kernel
-    if (attr_set[a.op & 3] < smem) {
+    using KernFn = void (*)(const CUtensorMap, const FArgs);
+    const bool best = f.best_mask != 0;
+    KernFn kern = nullptr;
+    int ki = 0;
+    if (a.accumulate) {
+        if (a.nops != 1 || best) return cudaErrorInvalidValue;
+        kern = fastid_tc4_kernel<BN, 1, false, true, -1>; ki = 0;
+    } else if (a.nops == 1) {   // compile-time op
+        static KernFn k1[2][4] = {{fastid_tc4_kernel<BN, 1, false, false, 0>, fastid_tc4_kernel<BN, 1, false, false, 1>,
+                                   fastid_tc4_kernel<BN, 1, false, false, 2>, fastid_tc4_kernel<BN, 1, false, false, 3>},
+                                  {fastid_tc4_kernel<BN, 1, true, false, 0>, fastid_tc4_kernel<BN, 1, true, false, 1>,
+                                   fastid_tc4_kernel<BN, 1, true, false, 2>, fastid_tc4_kernel<BN, 1, true, false, 3>}};
+        kern = k1[best][a.ops[0] & 3];
+        ki = 1 + 4 * best + (a.ops[0] & 3);
+    } else if (a.nops == 2 && a.ops[0] == 1 && a.ops[1] == 2) {   // XOR + ANDNOT (identity + mixture)
+        kern = best ? fastid_tc4_kernel<BN, 2, true, false, 1 | (2 << 2)>
+                    : fastid_tc4_kernel<BN, 2, false, false, 1 | (2 << 2)>;
+        ki = 9 + best;
+    } else {
+        switch (a.nops * 2 + (best ? 1 : 0)) {
+        case 4: kern = fastid_tc4_kernel<BN, 2, false, false, -1>; ki = 11; break;
+        case 5: kern = fastid_tc4_kernel<BN, 2, true, false, -1>; ki = 12; break;
+        case 6: kern = fastid_tc4_kernel<BN, 3, false, false, -1>; ki = 13; break;
+        case 7: kern = fastid_tc4_kernel<BN, 3, true, false, -1>; ki = 14; break;
+        case 8: kern = fastid_tc4_kernel<BN, 4, false, false, -1>; ki = 15; break;
+        case 9: kern = fastid_tc4_kernel<BN, 4, true, false, -1>; ki = 16; break;
+        default: return cudaErrorInvalidValue;
+        }
+    }
+    static size_t attr_set[17] = {};   // max dynamic smem already granted, per instantiation
+    if (attr_set[ki] < smem) {
         const size_t grant = MAX_SMEM - 1024;   // leave room for the kernel's static shared memory
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)grant);
         if (e != cudaSuccess) return e;
-        attr_set[a.op & 3] = grant;
+        attr_set[ki] = grant;
     }
     const int grid = (int)(f.ntiles < num_sms() ? f.ntiles : num_sms());
+    if (f.best_mask) {
+        const int64_t nk = (int64_t)a.nops * a.nq;
+        fastid_search_init<<<(int)((nk + 255) / 256), 256, 0, s>>>(a.keys, nk, a.done);
+        count_launches(1);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+    }
     kern<<<grid, NTHREADS, smem, s>>>(tm, f);
     count_launches(1);
     return cudaGetLastError();
@@ -495,7 +666,8 @@ cudaError_t launch_f(const GemmArgs &a, cudaStream_t s) {
 // Shape filter: queries on the column side (<= 128 rows, the user's first operand),
 // their whole expanded K range resident in shared memory, exact fp32 range.
 bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
-    if (m < 1 || m > 64 || n < 1 || nbits < 1 || nbits >= (1LL << 24)) return false;
+    // nbits < 2^23: counts leave the fp32 accumulator by the 2^23 magic add
+    if (m < 1 || m > 64 || n < 1 || nbits < 1 || nbits >= (1LL << 23)) return false;
     if (n < 4 * m) return false;
     if (n > (int64_t)0x7fffffff - BM) return false;
     return smem_bytes(64, nbits) <= MAX_SMEM - 1024;
@@ -503,7 +675,21 @@ bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
 
 cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     if (epi != EPI_COUNTS) return cudaErrorNotSupported;
-    return launch_f<64>(a, s);   // queries <= 64 (fastid_tc4_supported)
+    SearchArgs sa{};
+    sa.Q = a.A; sa.nq = a.m; sa.ldq32 = a.lda32;
+    sa.D = a.B; sa.nd = a.n; sa.ldd32 = a.ldb32;
+    sa.nbits = a.nbits;
+    sa.nops = 1; sa.ops[0] = a.op; sa.counts[0] = a.C;
+    sa.ldo = a.ldc; sa.accumulate = a.accumulate;
+    return launch_f<64>(sa, s);   // queries <= 64 (fastid_tc4_supported)
+}
+
+size_t fastid_search_tc4_ws_bytes(int64_t nq, int nops) {
+    return (((size_t)nops * nq * 8 + 255) & ~(size_t)255) + 256;
+}
+
+cudaError_t launch_fastid_search_tc4(const SearchArgs &a, cudaStream_t s) {
+    return launch_f<64>(a, s);
 }
 
 }  // namespace snp

@@ -323,6 +323,156 @@ snp_status snp_fastid_best(const uint32_t *counts, int64_t nq, int64_t nd, int64
     return e == cudaSuccess ? SNP_OK : set_cuda_error(e);
 }
 
+}  // extern "C"
+
+// ---------------------------------------------------------------- f1: fused search
+namespace {
+
+// Database rows per chunk of the composed (non-fused) search path when best matches are
+// wanted without stored counts: <= 64 MiB of chunk counts, a multiple of 128 rows.
+int64_t search_chunk_rows(int64_t nq, int64_t nd) {
+    int64_t ch = ((int64_t)(64 << 20) / (4 * (nq > 0 ? nq : 1))) / 128 * 128;
+    const char *e = std::getenv("SNP_SEARCH_CHUNK_ROWS");   // test hook: force small chunks
+    if (e && std::atoll(e) > 0) ch = std::atoll(e);
+    if (ch < 128) ch = 128;
+    return ch < nd ? ch : nd;
+}
+
+bool search_fused(int64_t nq, int64_t nd, int64_t nbits) {
+    return nd > 0 && choose_variant(nq, nd, nbits) == SNP_VARIANT_TC &&
+           tc_kernel_for(nq, nd, nbits, EPI_COUNTS) == SNP_KERNEL_FASTID_MXF4;
+}
+
+}  // namespace
+
+extern "C" {
+
+size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int nops) {
+    if (nq <= 0 || nbits <= 0 || nops < 1 || nops > 4) return 0;
+    if (nd < 0) return 0;
+    if (search_fused(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(nq, nops);
+    size_t b = align256((size_t)nops * nq * 8);
+    if (nd == 0) return b;
+    b += align256((size_t)nq * search_chunk_rows(nq, nd) * 4);
+    size_t g = 0;
+    for (int op = SNP_OP_AND; op <= SNP_OP_NOTAND; ++op) {
+        const size_t x = snp_fastid_workspace_bytes(nq, nd, nbits, op);
+        if (x > g) g = x;
+    }
+    return b + g;
+}
+
+snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
+                             const uint64_t *D, int64_t nd, int64_t ldd, int64_t nbits,
+                             int nops, const int *ops, uint32_t *const *counts, int64_t ldo,
+                             uint32_t *const *best_count, int64_t *const *best_index,
+                             int64_t index_base, void *ws, size_t ws_bytes, void *stream) {
+    snp_status st;
+    if (nq < 0 || nd < 0) return SNP_E_SHAPE;
+    if (nops < 1 || nops > 4) return SNP_E_OP;
+    if (!ops) return SNP_E_NULL;
+    for (int j = 0; j < nops; ++j)
+        if (ops[j] < SNP_OP_AND || ops[j] > SNP_OP_NOTAND) return SNP_E_OP;
+    if ((st = check_nbits(nbits)) != SNP_OK) return st;
+    if ((st = check_packed(Q, nq, ldq, nbits)) != SNP_OK) return st;
+    if ((st = check_packed(D, nd, ldd, nbits)) != SNP_OK) return st;
+    if ((best_count == nullptr) != (best_index == nullptr)) return SNP_E_NULL;
+    if (nd > 0xfffffffeLL) return SNP_E_RANGE;
+    if (nq == 0) return SNP_OK;
+    bool any_counts = false, any_best = false;
+    for (int j = 0; j < nops; ++j) {
+        uint32_t *c = counts ? counts[j] : nullptr;
+        if (c) {
+            any_counts = true;
+            if (!aligned16(c)) return SNP_E_ALIGN;
+        }
+        if (best_count) {
+            if ((best_count[j] == nullptr) != (best_index[j] == nullptr)) return SNP_E_NULL;
+            if (best_count[j]) {
+                any_best = true;
+                if (((uintptr_t)best_count[j] & 3u) || ((uintptr_t)best_index[j] & 7u)) return SNP_E_ALIGN;
+            }
+        }
+    }
+    if (any_counts && ldo < nd) return SNP_E_SHAPE;
+    if (!any_counts && !any_best) return SNP_OK;
+    const size_t need = snp_fastid_search_workspace_bytes(nq, nd, nbits, nops);
+    if (ws_bytes < need || !ws) return SNP_E_WORKSPACE;
+    if ((st = check_arch()) != SNP_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+
+    SearchArgs a{};
+    a.Q = reinterpret_cast<const uint32_t *>(Q);
+    a.nq = nq; a.ldq32 = 2 * ldq;
+    a.D = reinterpret_cast<const uint32_t *>(D);
+    a.nd = nd; a.ldd32 = 2 * ldd;
+    a.nbits = nbits;
+    a.nops = nops;
+    a.ldo = ldo;
+    a.index_base = index_base;
+    for (int j = 0; j < nops; ++j) {
+        a.ops[j] = ops[j];
+        a.counts[j] = counts ? counts[j] : nullptr;
+        a.best_count[j] = best_count ? best_count[j] : nullptr;
+        a.best_index[j] = best_index ? best_index[j] : nullptr;
+    }
+    if (search_fused(nq, nd, nbits)) {
+        // one pass over the database for every op (fastid_tc4.cu)
+        a.keys = reinterpret_cast<unsigned long long *>(ws);
+        a.done = reinterpret_cast<unsigned int *>((char *)ws + align256((size_t)nops * nq * 8));
+        if ((e = launch_fastid_search_tc4(a, s)) != cudaSuccess) return set_cuda_error(e);
+        g_last_variant = SNP_VARIANT_TC;
+        g_last_kernel = SNP_KERNEL_FASTID_MXF4;
+        return SNP_OK;
+    }
+
+    // Composed path (shapes the fused kernel does not take, or a forced variant): per op,
+    // counts by snp_fastid's kernels, best by best.cu; without stored counts the database
+    // is processed in chunks into workspace counts (nothing nq x nd is allocated).
+    unsigned long long *keys = reinterpret_cast<unsigned long long *>(ws);
+    char *p = (char *)ws + align256((size_t)nops * nq * 8);
+    const int64_t ch = nd > 0 ? search_chunk_rows(nq, nd) : 0;
+    uint32_t *chunk = reinterpret_cast<uint32_t *>(p);
+    if (nd > 0) p += align256((size_t)nq * ch * 4);
+    void *gws = p;
+    const size_t gws_bytes = ws_bytes - (size_t)(p - (char *)ws);
+    for (int j = 0; j < nops; ++j) {
+        const bool best = a.best_count[j] != nullptr;
+        unsigned long long *kj = keys + (int64_t)j * nq;
+        if (best && (e = launch_best_init(kj, nq, s)) != cudaSuccess) return set_cuda_error(e);
+        const int variant = choose_variant(nq, nd, nbits);
+        if (a.counts[j] && nd > 0) {
+            GemmArgs g{};
+            g.A = a.Q; g.B = a.D; g.m = nq; g.n = nd; g.lda32 = a.ldq32; g.ldb32 = a.ldd32;
+            g.nbits = nbits; g.op = ops[j]; g.ldc = ldo; g.C = a.counts[j];
+            if ((st = run_gemm(g, EPI_COUNTS, variant, gws, gws_bytes, s)) != SNP_OK) return st;
+            if (best && (e = launch_best_reduce(a.counts[j], nq, nd, ldo, 0, kj, s)) != cudaSuccess)
+                return set_cuda_error(e);
+        } else if (best) {
+            for (int64_t j0 = 0; j0 < nd; j0 += ch) {
+                const int64_t rows = nd - j0 < ch ? nd - j0 : ch;
+                const int cv = choose_variant(nq, rows, nbits);
+                GemmArgs g{};
+                g.A = a.Q; g.B = a.D + j0 * a.ldd32; g.m = nq; g.n = rows;
+                g.lda32 = a.ldq32; g.ldb32 = a.ldd32;
+                g.nbits = nbits; g.op = ops[j]; g.ldc = ch; g.C = chunk;
+                if ((st = run_gemm(g, EPI_COUNTS, cv, gws, gws_bytes, s)) != SNP_OK) return st;
+                if ((e = launch_best_reduce(chunk, nq, rows, ch, j0, kj, s)) != cudaSuccess)
+                    return set_cuda_error(e);
+            }
+        }
+        if (best && (e = launch_best_finalize(kj, nq, index_base, a.best_count[j], a.best_index[j], s)) !=
+                        cudaSuccess)
+            return set_cuda_error(e);
+    }
+    return SNP_OK;
+}
+
+}  // extern "C"
+
+extern "C" {
+
 snp_status snp_shard_plan(int64_t rows, int world, int64_t align, int64_t *bounds) {
     if (world < 1 || align < 1 || rows < 0) return SNP_E_RANGE;
     if (!bounds) return SNP_E_NULL;

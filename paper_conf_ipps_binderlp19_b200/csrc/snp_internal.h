@@ -45,6 +45,26 @@ cudaError_t launch_best(const uint32_t *counts, int64_t nq, int64_t nd, int64_t 
                         int64_t index_base, uint32_t *best_count, int64_t *best_index,
                         cudaStream_t s);
 
+// f1 fused FastID search (snp_fastid_search): one pass over the database, up to 4 ops
+// derived from one AND count, each with optional counts and optional best match.
+struct SearchArgs {
+    const uint32_t *Q;   // [nq][ldq32] queries, packed u32 view
+    int64_t nq, ldq32;
+    const uint32_t *D;   // [nd][ldd32] database
+    int64_t nd, ldd32;
+    int64_t nbits;
+    int nops;
+    int ops[4];
+    uint32_t *counts[4];      // per op [nq][ldo] or NULL
+    int64_t ldo;
+    int accumulate;
+    uint32_t *best_count[4];  // per op [nq] or NULL (then best_index[j] is NULL too)
+    int64_t *best_index[4];
+    int64_t index_base;
+    unsigned long long *keys; // workspace: [nops][nq] merge keys
+    unsigned int *done;       // workspace: CTA completion counter
+};
+
 // Tensor-core tcgen05 variant (bitgemm_tc.cu).  ws: expanded operands.
 size_t tc_workspace_bytes(int64_t m, int64_t n, int64_t nbits);
 bool tc_supported(int64_t m, int64_t n, int64_t nbits);
@@ -60,5 +80,15 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s);
 // memory, database streamed by TMA.  The queries are the user's first operand.
 bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits);
 cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s);
+size_t fastid_search_tc4_ws_bytes(int64_t nq, int nops);
+cudaError_t launch_fastid_search_tc4(const SearchArgs &a, cudaStream_t s);
+
+// best.cu building blocks for the chunked search path: keys (count << 32 | j) are
+// initialised to ~0, min-merged per count block (j offset by jbase), then finalised.
+cudaError_t launch_best_init(unsigned long long *keys, int64_t n, cudaStream_t s);
+cudaError_t launch_best_reduce(const uint32_t *counts, int64_t nq, int64_t nd, int64_t ldo, int64_t jbase,
+                               unsigned long long *keys, cudaStream_t s);
+cudaError_t launch_best_finalize(const unsigned long long *keys, int64_t nq, int64_t index_base,
+                                 uint32_t *best_count, int64_t *best_index, cudaStream_t s);
 
 }  // namespace snp

@@ -67,6 +67,19 @@ __device__ __forceinline__ void mbar_wait_warp(uint64_t *bar, uint32_t parity) {
     mbar_wait(bar, parity);
     __syncwarp();
 }
+// Warp-uniform wait for MMA-issuing warps: the exit condition is a warp vote, so ptxas
+// keeps the issuing loop's counters, TMEM addresses and descriptors in uniform registers
+// (no per-MMA R2UR conversions; the tcgen05.mma issue path stays on the uniform datapath).
+static __device__ __noinline__ void mbar_wait_uniform_slow(uint64_t *bar, uint32_t parity) {
+    const uint64_t t0 = globaltimer_ns();
+    while (!__all_sync(0xffffffffu, mbar_try_wait(bar, parity))) {
+        if (__any_sync(0xffffffffu, globaltimer_ns() - t0 > 4000000000ull)) __trap();
+    }
+}
+__device__ __forceinline__ void mbar_wait_uniform(uint64_t *bar, uint32_t parity) {
+    if (__all_sync(0xffffffffu, mbar_try_wait(bar, parity))) return;
+    mbar_wait_uniform_slow(bar, parity);
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}" ::"r"(smem_u32(bar))
                  : "memory");
@@ -244,6 +257,25 @@ __device__ __forceinline__ void mma4_mxf4_ts(uint32_t d, uint32_t a0, uint64_t b
         "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%4], %8, %10, [%11], [%12], t;\n\t}" ::"r"(d),
         "r"(a0), "r"(a0 + 8), "r"(a0 + 16), "r"(a0 + 24), "l"(b0), "l"(b1), "l"(b2), "l"(b3), "r"(accumulate),
         "r"(idesc), "r"(sfa), "r"(sfb)
+        : "memory");
+}
+
+// One tcgen05.mma kind::mxf4 (block32 scales, A from TMEM) issued by the elect.sync
+// leader of a converged warp; with warp-uniform operands ptxas emits a single uniform
+// UTCOMMA.  accumulate = 0 overwrites D.
+__device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a, uint64_t b, uint32_t idesc, uint32_t accumulate,
+                                            uint32_t sfa, uint32_t sfb) {
+    asm volatile(
+        "{\n\t.reg .pred e, p;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}" ::"r"(d),
+        "r"(a), "l"(b), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb)
+        : "memory");
+}
+// tcgen05.commit to an mbarrier by the elect.sync leader (uniform UTCBAR).
+__device__ __forceinline__ void mma_commit_uniform(uint64_t *bar) {
+    asm volatile(
+        "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
         : "memory");
 }
 

@@ -334,3 +334,126 @@ def test_cfg2_fastid_full_cross_variant(snp):
             assert int((got.view(torch.int32) != ref).sum().item()) == 0
     finally:
         _variant(snp, "auto")
+
+
+# ------------------------------------------------------------------ f1 fused search
+
+ALL_OPS = ("and", "xor", "andnot", "notand")
+SEARCH_SHAPES = [(1, 4, 1), (3, 700, 129), (33, 1000, 4096), (64, 2000, 777), (64, 300, 100),
+                 (70, 513, 1000), (130, 300, 2049)]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("nq,nd,nbits", SEARCH_SHAPES)
+def test_search_all_ops_counts_and_best(snp, variant, nq, nd, nbits):
+    db = snpgen.fastid_db(31, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(31, nq, nd, nbits)
+    D = pack_dev(snp, db, garbage_seed=5)
+    Q = pack_dev(snp, q, garbage_seed=6)
+    _variant(snp, variant)
+    try:
+        counts, best = snp.snp_fastid_search(Q, D, nbits, ALL_OPS, counts=True, best=True, index_base=7)
+        for j, op in enumerate(ALL_OPS):
+            ref = oracle.counts(q, db, op)
+            assert np.array_equal(u32(counts[j]), ref), (op, variant)
+            rb, ri = oracle.best(ref, 7)
+            assert np.array_equal(u32(best[j][0]), rb), op
+            assert np.array_equal(best[j][1].cpu().numpy(), ri), op
+        # best only (no count matrix written), two ops, chunked composition for big nq
+        _, best2 = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False, best=True)
+        for j, op in enumerate(("xor", "andnot")):
+            rb, ri = oracle.best(oracle.counts(q, db, op))
+            assert np.array_equal(u32(best2[j][0]), rb) and np.array_equal(best2[j][1].cpu().numpy(), ri)
+    finally:
+        _variant(snp, "auto")
+
+
+def test_search_kernel_choice(snp):
+    nbits, nd = 4096, 4096
+    db = snpgen.fastid_db(3, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(3, 64, nd, nbits)
+    snp.snp_fastid_search(pack_dev(snp, q), pack_dev(snp, db), nbits)
+    assert snp.snp_last_kernel() == "fastid_mxf4"
+
+
+def test_search_ties_lowest_index_across_ctas(snp):
+    """Many exact ties spread over every CTA, warp and lane quarter: the merged best
+    must be the lowest database index (reading R4), for counts and best-only."""
+    nbits, nd, nq = 1000, 200_000, 40
+    base = snpgen.fastid_db(41, np.arange(13), nbits)
+    idx = (np.arange(nd) * 7 + 3) % 13                # row j = base[idx[j]]
+    db = base[idx]
+    q = base[np.arange(nq) % 13].copy()
+    q[::5, :3] ^= 1                                   # some queries have no exact copy
+    D = pack_dev(snp, db)
+    Q = pack_dev(snp, q)
+    for variant in ("auto", "popc"):
+        _variant(snp, variant)
+        try:
+            for counts in (True, False):
+                c, best = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot", "and"), counts=counts,
+                                                index_base=1 << 33)
+                for j, op in enumerate(("xor", "andnot", "and")):
+                    ref = oracle.counts(q, base, op)[:, idx]     # = counts vs every db row
+                    rb, ri = oracle.best(ref, 1 << 33)
+                    assert np.array_equal(u32(best[j][0]), rb), (variant, op)
+                    assert np.array_equal(best[j][1].cpu().numpy(), ri), (variant, op)
+        finally:
+            _variant(snp, "auto")
+
+
+def test_search_chunked_composition(snp, monkeypatch):
+    """Best-only search for shapes the fused kernel does not take runs in database
+    chunks through workspace counts; force small ragged chunks."""
+    monkeypatch.setenv("SNP_SEARCH_CHUNK_ROWS", "384")
+    nq, nd, nbits = 100, 2000, 300
+    db = snpgen.fastid_db(43, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(43, nq, nd, nbits)
+    _, best = snp.snp_fastid_search(pack_dev(snp, q), pack_dev(snp, db), nbits, ALL_OPS, counts=False,
+                                    index_base=5)
+    for j, op in enumerate(ALL_OPS):
+        rb, ri = oracle.best(oracle.counts(q, db, op), 5)
+        assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), op
+
+
+def test_search_empty_database(snp):
+    nbits = 256
+    q = snpgen.fastid_db(44, np.arange(5), nbits)
+    Q = pack_dev(snp, q)
+    D = torch.empty((0, snp.snp_words(nbits)), dtype=torch.uint64, device=DEV)
+    _, best = snp.snp_fastid_search(Q, D, nbits, ("xor",), counts=False)
+    assert (u32(best[0][0]) == 0xFFFFFFFF).all() and (best[0][1].cpu().numpy() == -1).all()
+
+
+@pytest.mark.parametrize("variant", ["auto", "popc"])
+def test_cfg2_search_1m(snp, variant):
+    """configs[1] in the launch configuration bench.py times: ONE search call for XOR +
+    ANDNOT with counts and best matches.  Sampled DB columns (every tile-boundary
+    neighbourhood included) vs the oracle; best == numpy min/argmin over the full
+    count matrices; planted identity copies found."""
+    nq, nd, nbits, seed = 64, 1_000_000, 4096, 1002
+    D = _gen_dev_fastid(seed, nd, nbits)
+    q, plan = snpgen.fastid_queries(seed, nq, nd, nbits)
+    Q = snp.snp_pack(to_dev(q))
+    cols = _sample_cols(nd, 128, 600, 10)
+    dbs = snpgen.fastid_db(seed, cols, nbits)
+    _variant(snp, variant)
+    try:
+        counts, best = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"))
+        if variant == "auto":
+            assert snp.snp_last_kernel() == "fastid_mxf4"
+        for j, op in enumerate(("xor", "andnot")):
+            got = u32(counts[j].view(torch.int32)[:, torch.from_numpy(cols).to(DEV)])
+            assert np.array_equal(got, oracle.counts(q, dbs, op)), op
+            full = counts[j].cpu().numpy().astype(np.uint32)
+            assert np.array_equal(u32(best[j][0]), full.min(1)), op
+            assert np.array_equal(best[j][1].cpu().numpy(), full.argmin(1)), op
+            if op == "xor":
+                for qi, (kind, js, flips) in enumerate(plan):
+                    if kind == "copy":
+                        assert u32(best[j][0])[qi] <= len(flips)
+        _, bonly = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False)
+        for j in range(2):
+            assert torch.equal(bonly[j][0], best[j][0]) and torch.equal(bonly[j][1], best[j][1])
+    finally:
+        _variant(snp, "auto")
