@@ -101,12 +101,26 @@ __device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
     return (1u << (uint32_t)(nbits - lo)) - 1u;
 }
 
-__device__ __forceinline__ void expand4(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
-    const uint32_t M = 0x22222222u;   // e2m1 1.0 = 0b0010 in every nibble where the bit is set
-    o0 = (x << 1) & M;
-    o1 = x & M;
-    o2 = (x >> 1) & M;
-    o3 = (x >> 2) & M;
+// Bits -> e2m1 nibbles for kind::mxf4 (scale factors all 2^0).  Output word t of input
+// word x holds bit 4n + t in nibble n (a fixed K permutation shared by both operands).
+// The two operands use complementary nibble positions so every product of set bits is
+// exactly 1.0 with as few shifts as possible (e2m1: bit0 = 0.5, bit1 = 1.0, bit2 = 2.0):
+//   t:        0            1           2            3
+//   A (TMEM)  bit0 = 0.5   bit1 = 1.0  bit2 = 2.0   bit1 = 1.0 (x >> 2)
+//   B (smem)  bit2 = 2.0   bit1 = 1.0  bit0 = 0.5   bit1 = 1.0 (x >> 2)
+// A: 4 LOP3 + 1 shift, B: 4 LOP3 + 2 shifts (was 4 LOP3 + 3 shifts for 1.0 everywhere).
+__device__ __forceinline__ void expandA(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
+    o0 = x & 0x11111111u;
+    o1 = x & 0x22222222u;
+    o2 = x & 0x44444444u;
+    o3 = __umulhi(x, 0x40000000u) & 0x22222222u;   // (x >> 2) on the FMA pipe
+}
+__device__ __forceinline__ void expandB(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
+    const uint32_t y = __umulhi(x, 0x40000000u);    // x >> 2
+    o0 = (x * 4u) & 0x44444444u;
+    o1 = x & 0x22222222u;
+    o2 = y & 0x11111111u;
+    o3 = y & 0x22222222u;
 }
 
 __host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
@@ -229,7 +243,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             if (row < args.nq && w < nw32) x = __ldg(args.Q + row * args.ldq32 + w) & word_mask(w, nbits);
             if (x) atomicAdd(&popQ[row], (uint32_t)__popc(x));
             uint4 o;
-            expand4(x, o.x, o.y, o.z, o.w);
+            expandB(x, o.x, o.y, o.z, o.w);   // queries: MMA B operand
             *reinterpret_cast<uint4 *>(qsm + (size_t)w * BN * 16 + row * 16) = o;
         }
     }
@@ -322,7 +336,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 uint32_t v[32];
 #pragma unroll
                 for (int i = 0; i < 8; ++i)
-                    expand4(wv[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+                    expandA(wv[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
                 tmem_st32(tbase + 32 * h, v);
             }
             ptx::tmem_st_wait();

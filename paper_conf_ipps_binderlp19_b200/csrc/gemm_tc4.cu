@@ -38,7 +38,12 @@ namespace {
 constexpr int BM = 128, BN = 128;
 constexpr int KBITS = 512;
 constexpr int KW = KBITS / 32;                 // 16 packed words per row per stage
-constexpr int NS = 3;                          // pipeline slots (packed ring, TMEM A, smem B)
+constexpr int NS = 3;                          // expanded slots (TMEM A stage + smem B stage)
+#ifndef GEMM_NP
+#define GEMM_NP 6
+#endif
+constexpr int NP = GEMM_NP;                    // packed TMA ring: NP x 16 KB in flight per SM
+                                               // (3 slots left the expanders waiting on L2)
 #ifndef GEMM_G
 #define GEMM_G 2
 #endif
@@ -56,7 +61,7 @@ constexpr int ACC_COLS = BN;
 constexpr int A_COL0 = 2 * ACC_COLS;           // 256
 constexpr int SF_COL = A_COL0 + NS * 64;       // 448
 static_assert(SF_COL + 32 <= 512, "TMEM budget");
-constexpr size_t SMEM = (size_t)NS * PSLOT + (size_t)NS * BSLOT + 1024;
+constexpr size_t SMEM = (size_t)NP * PSLOT + (size_t)NS * BSLOT + 1024;
 
 struct GArgs {
     int64_t nl, nc, nbits;
@@ -78,14 +83,26 @@ __device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
     return (1u << (uint32_t)(nbits - lo)) - 1u;
 }
 
-// 32 bits -> 4 words of 8 e2m1 nibbles (1.0 = 0b0010 where the bit is set); nibble n of
-// output t holds bit 4n + t.  The two right shifts run on the FMA pipe (IMAD.HI).
-__device__ __forceinline__ void expand4(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
-    const uint32_t M = 0x22222222u;
-    o0 = (x << 1) & M;
-    o1 = x & M;
-    o2 = __umulhi(x, 0x80000000u) & M;   // x >> 1
-    o3 = __umulhi(x, 0x40000000u) & M;   // x >> 2
+// Bits -> e2m1 nibbles for kind::mxf4 (scale factors all 2^0).  Output word t of input
+// word x holds bit 4n + t in nibble n (a fixed K permutation shared by both operands).
+// The two operands use complementary nibble positions so every product of set bits is
+// exactly 1.0 with as few shifts as possible (e2m1: bit0 = 0.5, bit1 = 1.0, bit2 = 2.0):
+//   t:        0            1           2            3
+//   A (TMEM)  bit0 = 0.5   bit1 = 1.0  bit2 = 2.0   bit1 = 1.0 (x >> 2)
+//   B (smem)  bit2 = 2.0   bit1 = 1.0  bit0 = 0.5   bit1 = 1.0 (x >> 2)
+// A: 4 LOP3 + 1 shift, B: 4 LOP3 + 2 shifts (was 4 LOP3 + 3 shifts for 1.0 everywhere).
+__device__ __forceinline__ void expandA(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
+    o0 = x & 0x11111111u;
+    o1 = x & 0x22222222u;
+    o2 = x & 0x44444444u;
+    o3 = __umulhi(x, 0x40000000u) & 0x22222222u;   // (x >> 2) on the FMA pipe
+}
+__device__ __forceinline__ void expandB(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
+    const uint32_t y = __umulhi(x, 0x40000000u);    // x >> 2
+    o0 = (x * 4u) & 0x44444444u;
+    o1 = x & 0x22222222u;
+    o2 = y & 0x11111111u;
+    o3 = y & 0x22222222u;
 }
 
 __host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
@@ -146,12 +163,12 @@ __global__ void __launch_bounds__(NTHREADS, 1)
 gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
                 const GArgs args) {
     extern __shared__ __align__(1024) uint8_t smem[];
-    uint8_t *ring = smem;                                        // [NS][PSLOT]
-    uint8_t *bexp = smem + (size_t)NS * PSLOT;                   // [NS][BSLOT]
+    uint8_t *ring = smem;                                        // [NP][PSLOT]
+    uint8_t *bexp = smem + (size_t)NP * PSLOT;                   // [NS][BSLOT]
     uint64_t *bars = reinterpret_cast<uint64_t *>(bexp + (size_t)NS * BSLOT);
-    uint64_t *pfull = bars;            // [NS] TMA -> expanders
-    uint64_t *pempty = pfull + NS;     // [NS] expanders -> TMA
-    uint64_t *full = pempty + NS;      // [NS] expanders -> MMA
+    uint64_t *pfull = bars;            // [NP] TMA -> expanders
+    uint64_t *pempty = pfull + NP;     // [NP] expanders -> TMA
+    uint64_t *full = pempty + NP;      // [NS] expanders -> MMA
     uint64_t *empty = full + NS;       // [NS] MMA -> expanders
     uint64_t *accf = empty + NS;       // [2]
     uint64_t *acce = accf + 2;         // [2]
@@ -161,14 +178,20 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     const int64_t nbits = args.nbits;
     const int nst = args.nst;
     const int64_t ntiles = args.nlb * args.ncb;
-    const int64_t my_tiles = ntiles > blockIdx.x ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    // 32-bit tile arithmetic (ntiles < 2^31): a 64-bit division is a subroutine CALL, and
+    // any call in the kernel made ptxas drop the MMA issue loop out of uniform registers
+    const uint32_t nlb32 = (uint32_t)args.nlb;
+    const int64_t my_tiles =
+        ntiles > blockIdx.x ? (int64_t)(((uint32_t)ntiles - 1u - blockIdx.x) / gridDim.x + 1u) : 0;
     const int64_t total_it = my_tiles * nst;
     const int64_t full32 = nbits / 32;
 
     if (tid == 0) {
-        for (int i = 0; i < NS; ++i) {
+        for (int i = 0; i < NP; ++i) {
             ptx::mbar_init(&pfull[i], 1);
             ptx::mbar_init(&pempty[i], 8);
+        }
+        for (int i = 0; i < NS; ++i) {
             ptx::mbar_init(&full[i], 8);
             ptx::mbar_init(&empty[i], 1);
         }
@@ -206,13 +229,14 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             uint32_t round = 0;
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
                 const int64_t t = blockIdx.x + tl * gridDim.x;
-                const int32_t rl = (int32_t)((t % args.nlb) * BM), rc = (int32_t)((t / args.nlb) * BN);
+                const uint32_t t32 = (uint32_t)t;
+                const int32_t rl = (int32_t)((t32 % nlb32) * BM), rc = (int32_t)((t32 / nlb32) * BN);
                 for (int s = 0; s < nst; ++s) {
                     if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
                     ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
                     ptx::tma_load_2d(ring + p * PSLOT, &tmL, &pfull[p], s * KW, rl);
                     ptx::tma_load_2d(ring + p * PSLOT + BM * PROW, &tmC, &pfull[p], s * KW, rc);
-                    if (++p == NS) { p = 0; ++round; }
+                    if (++p == NP) { p = 0; ++round; }
                 }
             }
         }
@@ -231,6 +255,9 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         int s = g % nst;
         int slot = g % NS;
         uint32_t use = (uint32_t)(g / NS);              // how often `slot` was used before
+        static_assert(NP % G == 0, "each packed slot belongs to one expander group");
+        int pk = g;                                     // packed slot (group g: g, g + G, ...)
+        uint32_t pround = 0;
         for (int64_t it = g; it < total_it; it += G) {
             const bool tr = args.trace && blockIdx.x == 0 && r8 == 0 && lane == 0 && it < 2048;
             if (tr) g_gemm_trace[8 * it + 0] = clock64();
@@ -238,18 +265,20 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             // a slot while its pfull barrier is only at phase u+1; waiting for the MMA to
             // release use u+1 first rules out parity aliasing on pfull (same parity as u)
             if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
-            ptx::mbar_wait_warp(&pfull[slot], use & 1);
+            ptx::mbar_wait_warp(&pfull[pk], pround & 1);
             if (tr) g_gemm_trace[8 * it + 1] = clock64();
             if (args.debug_skip) {
                 __syncwarp();
-                if (lane == 0) { ptx::mbar_arrive(&pempty[slot]); ptx::mbar_arrive(&full[slot]); }
+                if (lane == 0) { ptx::mbar_arrive(&pempty[pk]); ptx::mbar_arrive(&full[slot]); }
                 s += G;
                 while (s >= nst) { s -= nst; ++tl; }
                 slot += G;
                 if (slot >= NS) { slot -= NS; ++use; }
+                pk += G;
+                if (pk >= NP) { pk -= NP; ++pround; }
                 continue;
             }
-            const uint8_t *src = ring + slot * PSLOT + (is_a ? 0 : BM * PROW) + row * PROW;
+            const uint8_t *src = ring + pk * PSLOT + (is_a ? 0 : BM * PROW) + row * PROW;
             uint32_t w[KW];
 #pragma unroll
             for (int c = 0; c < 4; ++c) {
@@ -269,7 +298,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                     uint32_t v[32];
 #pragma unroll
                     for (int i = 0; i < 8; ++i)
-                        expand4(w[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+                        expandA(w[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
                     tmem_st32(tA + 32 * h, v);
                 }
                 ptx::tmem_st_wait();
@@ -279,7 +308,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
 #pragma unroll
                 for (int i = 0; i < KW; ++i) {          // chunk i of the K-major operand = word i
                     uint4 o;
-                    expand4(w[i], o.x, o.y, o.z, o.w);
+                    expandB(w[i], o.x, o.y, o.z, o.w);
                     *reinterpret_cast<uint4 *>(dstB + (size_t)i * BN * 16) = o;
                 }
                 ptx::fence_proxy_async_smem();
@@ -289,7 +318,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 // release the packed slot only now: every lane has consumed its LDS results
                 // (an arrive right after the loads could let the next TMA overwrite data
                 // that is still in flight to registers)
-                ptx::mbar_arrive(&pempty[slot]);
+                ptx::mbar_arrive(&pempty[pk]);
                 ptx::mbar_arrive(&full[slot]);
             }
             if (tr) g_gemm_trace[8 * it + 3] = clock64();
@@ -297,33 +326,37 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             while (s >= nst) { s -= nst; ++tl; }
             slot += G;
             if (slot >= NS) { slot -= NS; ++use; }
+            pk += G;
+            if (pk >= NP) { pk -= NP; ++pround; }
         }
     } else if (warp == MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
+        // Warp-uniform loop (votes for the waits, tmem via a warp reduction): the TMEM
+        // addresses and descriptors stay in uniform registers and each MMA is one UTCOMMA.
         constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
-        const uint32_t sfa = tmem + SF_COL, sfb = tmem + SF_COL + 16;
+        const uint32_t tmu = __reduce_or_sync(0xffffffffu, tmem);
+        const uint32_t sfa = tmu + SF_COL, sfb = tmu + SF_COL + 16;
         const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(bexp), BN * 16, 128);
         constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;
         int b = 0;
         uint32_t round = 0;
-        int64_t itm = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
-            if (tl >= 2) ptx::mbar_wait_warp(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            if (tl >= 2) ptx::mbar_wait_uniform(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
             ptx::tc_fence_after();
-            const uint32_t d = tmem + (uint32_t)(acc * ACC_COLS);
-            for (int s = 0; s < nst; ++s, ++itm) {
-                const bool trm = args.trace && blockIdx.x == 0 && lane == 0 && itm < 2048;
-                ptx::mbar_wait_warp(&full[b], round & 1);
-                if (trm) g_gemm_trace[8 * itm + 5] = clock64();
+            const uint32_t d = tmu + (uint32_t)(acc * ACC_COLS);
+            for (int s = 0; s < nst; ++s) {
+                ptx::mbar_wait_uniform(&full[b], round & 1);
                 ptx::tc_fence_after();
-                ptx::mma8_mxf4_ts_commit(d, tmem + (uint32_t)(A_COL0 + 64 * b),
-                                         bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4), BSTEP, IDESC,
-                                         s != 0 ? 1u : 0u, sfa, sfb, &empty[b]);
-                if (trm) g_gemm_trace[8 * itm + 7] = clock64();
+                const uint32_t a0 = tmu + (uint32_t)(A_COL0 + 64 * b);
+                const uint64_t b0 = bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4);
+#pragma unroll
+                for (int k = 0; k < KBITS / 64; ++k)
+                    ptx::mma_mxf4_ts(d, a0 + 8 * k, b0 + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                ptx::mma_commit_uniform(&empty[b]);
                 if (++b == NS) { b = 0; ++round; }
             }
-            ptx::mma_commit_elect(&accf[acc]);
+            ptx::mma_commit_uniform(&accf[acc]);
         }
         __syncwarp();
     } else {
@@ -342,8 +375,9 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             const int acc = (int)(tl & 1);
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
             const int64_t t = blockIdx.x + tl * gridDim.x;
-            const int64_t gl = (t % args.nlb) * BM + li;
-            const int64_t gc0 = (t / args.nlb) * BN + c0;
+            const uint32_t t32 = (uint32_t)t;
+            const int64_t gl = (int64_t)(t32 % nlb32) * BM + li;
+            const int64_t gc0 = (int64_t)(t32 / nlb32) * BN + c0;
             const bool rows_ok = gl < args.nl && gc0 < args.nc;
             const int ncols = gc0 < args.nc ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
             // popcounts: lane j holds the column popcounts of columns c0 + j and c0 + 32 + j
