@@ -61,7 +61,9 @@ constexpr int ACC_COLS = BN;
 constexpr int A_COL0 = 2 * ACC_COLS;           // 256
 constexpr int SF_COL = A_COL0 + NS * 64;       // 448
 static_assert(SF_COL + 32 <= 512, "TMEM budget");
-constexpr size_t SMEM = (size_t)NP * PSLOT + (size_t)NS * BSLOT + 1024;
+constexpr int TRW = 32 * 32 * 4;                // per epilogue warp: 32 x 32 count transpose
+constexpr size_t SMEM = (size_t)NP * PSLOT + (size_t)NS * BSLOT + (size_t)NEPI * TRW + 1024;
+static_assert(SMEM <= 232448, "227 KB opt-in shared memory");
 
 struct GArgs {
     int64_t nl, nc, nbits;
@@ -73,6 +75,7 @@ struct GArgs {
     int nst;
     int trace;
     int debug_skip;   // profiling experiment: expanders only pass tokens (results invalid)
+    int order;        // tile raster: 1 lane-block-major, 0 column-block-major
     const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
 };
 
@@ -158,6 +161,122 @@ __device__ __forceinline__ void ld_stats_f32(int64_t n, int64_t na, int64_t nb, 
     dp = __fdiv_rn(fn, (float)dmax);
 }
 
+
+// 1/d rounded once to fp32 (d exact in fp64); 0 for d = 0 (monomorphic SNP: r2 = 0).
+__device__ __forceinline__ float inv_exact(int64_t d) { return d ? (float)(1.0 / (double)d) : 0.f; }
+
+// Exact count from the fp32 accumulator (an integer < 2^24): the 2^23 magic add below
+// 2^23 (FMA pipe, no F2I), F2I above.
+__device__ __forceinline__ uint32_t acc_count(uint32_t v, bool small) {
+    return small ? __float_as_uint(__fadd_rn(__uint_as_float(v), 8388608.0f)) - 0x4B000000u
+                 : __float2uint_rn(__uint_as_float(v));
+}
+
+// Epilogue of a 32-row x 32-column block when the output's row index is the TMEM lane
+// (no operand swap): c[j] holds (row = this lane, column j) as fp32 accumulator bits.  The block is transposed
+// through the warp's 4 KB of shared memory (16-byte chunks XOR-swizzled by row: 4
+// wavefronts per STS.128, conflict-free LDS.32) so that afterwards lane = output column
+// and every store of a row is one coalesced 128-byte line.  Row quantities (nA, 1/da)
+// are broadcast from their lane by shuffles.
+//   counts: x = op identity of SURVEY §8a a4 with (pQ, pD) = (row, column) popcounts
+//   LD:     reading R3 from exact integers: num = n nAB - nA nB (int32 for n <= 46340),
+//           r2 = min(1, (num / da) (num / db)) with 1/da, 1/db rounded once: 7 fp32
+//           roundings in total, relative error <= 7 * 2^-24 = 4.2e-7;
+//           exactly 0 where num = 0.  D' = num / Dmax (correctly rounded division).
+template <int EPI>
+__device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[32], uint32_t *tw, int lane,
+                                               int64_t row0, int64_t col0, uint32_t pl, uint32_t pcol, float ia,
+                                               bool small_n, bool want_dp) {
+    const bool small = args.nbits < (1LL << 23);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) c[i] = acc_count(c[i], small);   // in place: c is the TMEM load
+    __syncwarp();   // the previous block's reads of tw are done
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        const uint32_t a = ptx::smem_u32(tw + lane * 32 + ((k ^ (lane & 7)) << 2));
+        asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(c[4 * k]), "r"(c[4 * k + 1]),
+                     "r"(c[4 * k + 2]), "r"(c[4 * k + 3])
+                     : "memory");
+    }
+    __syncwarp();
+    const int64_t gc = col0 + lane;
+    const bool colok = gc < args.nc;
+    const int64_t ldo = args.ldo;
+    const int64_t n = args.nbits;
+    const int32_t n32 = (int32_t)n;
+    const int32_t pb = (int32_t)pcol;
+    const int rows = (int)(args.nl - row0 < 32 ? args.nl - row0 : 32);   // warp-uniform
+    const int64_t o0 = row0 * ldo + gc;
+    if (EPI == EPI_COUNTS) {
+        uint32_t *cp = args.C + o0;
+        const int op = args.op;
+        const bool acc = args.accumulate != 0;
+#pragma unroll 4
+        for (int r = 0; r < 32; ++r) {
+            const uint32_t plr = __shfl_sync(0xffffffffu, pl, r);
+            if (r >= rows) break;
+            const uint32_t c = tw[r * 32 + ((((lane >> 2) ^ (r & 7))) << 2) + (lane & 3)];
+            const uint32_t x = op == 0 ? c : op == 1 ? plr + pcol - 2u * c : op == 2 ? plr - c : pcol - c;
+            if (colok) {
+                if (acc) *cp += x;
+                else __stcs(cp, x);
+            }
+            cp += ldo;
+        }
+        return;
+    }
+    float *rp = args.r2 + o0;
+    if (small_n && !want_dp) {
+        // the benchmarked LD path: per element 2 IMAD, I2F, 3 FMUL, FMNMX, 1-2 STG
+        const float ib = inv_exact((int64_t)pb * (n - (int64_t)pb));
+        const int32_t npb = -pb;
+        uint32_t *cp = args.C ? args.C + o0 : nullptr;
+#pragma unroll 4
+        for (int r = 0; r < 32; ++r) {
+            const int32_t plr = (int32_t)__shfl_sync(0xffffffffu, pl, r);
+            const float iar = __shfl_sync(0xffffffffu, ia, r);
+            if (r >= rows) break;
+            const int32_t c = (int32_t)tw[r * 32 + ((((lane >> 2) ^ (r & 7))) << 2) + (lane & 3)];
+            const int32_t num = n32 * c + plr * npb;
+            const float fn = (float)num;
+            const float r2v = fminf(__fmul_rn(__fmul_rn(fn, iar), __fmul_rn(fn, ib)), 1.0f);
+            if (colok) {
+                __stcs(rp, r2v);   // outputs are written once: evict-first keeps the packed
+                if (cp) __stcs(cp, (uint32_t)c);   // operands resident in L2
+            }
+            rp += ldo;
+            if (cp) cp += ldo;
+        }
+        return;
+    }
+    const float ib = inv_exact((int64_t)pb * (n - (int64_t)pb));
+#pragma unroll 1
+    for (int r = 0; r < rows; ++r) {
+        const uint32_t plr = __shfl_sync(0xffffffffu, pl, r);
+        const float iar = __shfl_sync(0xffffffffu, ia, r);
+        const uint32_t cr = tw[r * 32 + ((((lane >> 2) ^ (r & 7))) << 2) + (lane & 3)];
+        if (!colok) continue;
+        const int64_t o = o0 + (int64_t)r * ldo;
+        float r2v, dpv = 0.f;
+        if (small_n) {
+            const int32_t num = n32 * (int32_t)cr - (int32_t)plr * pb;
+            const float fn = (float)num;
+            r2v = fminf(__fmul_rn(__fmul_rn(fn, iar), __fmul_rn(fn, ib)), 1.0f);
+            if (num != 0) {
+                const int32_t pa_ = (int32_t)plr;
+                const int32_t dmax = num > 0 ? min(pa_ * (n32 - pb), (n32 - pa_) * pb)
+                                             : min(pa_ * pb, (n32 - pa_) * (n32 - pb));
+                dpv = __fdiv_rn(fn, (float)dmax);
+            }
+        } else {
+            ld_stats_f32(n, (int64_t)plr, (int64_t)pb, (int64_t)cr, r2v, dpv);
+        }
+        __stcs(args.r2 + o, r2v);
+        if (want_dp) __stcs(args.dprime + o, dpv);
+        if (args.C) __stcs(args.C + o, cr);
+    }
+}
+
 template <int EPI>
 __global__ void __launch_bounds__(NTHREADS, 1)
 gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
@@ -165,7 +284,8 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t *ring = smem;                                        // [NP][PSLOT]
     uint8_t *bexp = smem + (size_t)NP * PSLOT;                   // [NS][BSLOT]
-    uint64_t *bars = reinterpret_cast<uint64_t *>(bexp + (size_t)NS * BSLOT);
+    uint32_t *trs = reinterpret_cast<uint32_t *>(bexp + (size_t)NS * BSLOT);   // [NEPI][32][32]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(trs + NEPI * 32 * 32);
     uint64_t *pfull = bars;            // [NP] TMA -> expanders
     uint64_t *pempty = pfull + NP;     // [NP] expanders -> TMA
     uint64_t *full = pempty + NP;      // [NS] expanders -> MMA
@@ -180,7 +300,12 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     const int64_t ntiles = args.nlb * args.ncb;
     // 32-bit tile arithmetic (ntiles < 2^31): a 64-bit division is a subroutine CALL, and
     // any call in the kernel made ptxas drop the MMA issue loop out of uniform registers
-    const uint32_t nlb32 = (uint32_t)args.nlb;
+    const uint32_t nlb32 = (uint32_t)args.nlb, ncb32 = (uint32_t)args.ncb;
+    // tile t -> (lane block, column block): lane-block-major (the 148 tiles in flight share
+    // one lane block and write 148 adjacent column blocks of the same output rows) or
+    // column-block-major
+    auto tile_lb = [&](uint32_t t) { return args.order ? t / ncb32 : t % nlb32; };
+    auto tile_cb = [&](uint32_t t) { return args.order ? t % ncb32 : t / nlb32; };
     const int64_t my_tiles =
         ntiles > blockIdx.x ? (int64_t)(((uint32_t)ntiles - 1u - blockIdx.x) / gridDim.x + 1u) : 0;
     const int64_t total_it = my_tiles * nst;
@@ -230,7 +355,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
                 const int64_t t = blockIdx.x + tl * gridDim.x;
                 const uint32_t t32 = (uint32_t)t;
-                const int32_t rl = (int32_t)((t32 % nlb32) * BM), rc = (int32_t)((t32 / nlb32) * BN);
+                const int32_t rl = (int32_t)(tile_lb(t32) * BM), rc = (int32_t)(tile_cb(t32) * BN);
                 for (int s = 0; s < nst; ++s) {
                     if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
                     ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
@@ -376,8 +501,8 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
             const int64_t t = blockIdx.x + tl * gridDim.x;
             const uint32_t t32 = (uint32_t)t;
-            const int64_t gl = (int64_t)(t32 % nlb32) * BM + li;
-            const int64_t gc0 = (int64_t)(t32 / nlb32) * BN + c0;
+            const int64_t gl = (int64_t)tile_lb(t32) * BM + li;
+            const int64_t gc0 = (int64_t)tile_cb(t32) * BN + c0;
             const bool rows_ok = gl < args.nl && gc0 < args.nc;
             const int ncols = gc0 < args.nc ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
             // popcounts: lane j holds the column popcounts of columns c0 + j and c0 + 32 + j
@@ -393,6 +518,8 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * ACC_COLS + c0);
             const int32_t n32 = (int32_t)n, pl32 = (int32_t)pl;
             const int32_t da32 = pl32 * (n32 - pl32);
+            // 1 / (nA (n - nA)) of this lane's row, one rounding (0 for a monomorphic SNP)
+            const float ia = (EPI == EPI_LD && !args.swap) ? inv_exact((int64_t)pl * (n - (int64_t)pl)) : 0.f;
             // two halves of 32 accumulator columns; the accumulator is released right after
             // the second TMEM load, before that half is processed
 #pragma unroll 1
@@ -407,6 +534,11 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                     if (lane == 0) ptx::mbar_arrive(&acce[acc]);   // accumulator drained
                 }
                 const uint32_t pcol = hh ? pcol1 : pcol0;
+                if (!args.swap) {
+                    epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, gl - lane, gc0 + 32 * hh, pl, pcol,
+                                        ia, small_n, want_dp);
+                    continue;
+                }
                 if (!__any_sync(0xffffffffu, rows_ok)) continue;   // warp-uniform skip only:
                 // the column popcounts are shuffled across the warp, so every lane runs the
                 // loop and only rows_ok lanes store
@@ -594,6 +726,8 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.trace = trace ? 1 : 0;
     static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
     g.debug_skip = skip ? 1 : 0;
+    static const char *ord = std::getenv("SNP_GEMM_ORDER");
+    g.order = ord ? (ord[0] == '1') : 1;
     return epi == EPI_LD ? launch_g<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
 }
 

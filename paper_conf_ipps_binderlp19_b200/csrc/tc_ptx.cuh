@@ -29,6 +29,19 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t parity) {
         : "memory");
     return ok != 0;
 }
+// try_wait with a suspend-time hint: the thread sleeps (issuing nothing) until the phase
+// completes or ~hint_ns pass, so waiting warps do not steal issue slots from working ones.
+__device__ __forceinline__ bool mbar_try_wait_sleep(uint64_t *bar, uint32_t parity, uint32_t hint_ns) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity), "r"(hint_ns)
+        : "memory");
+    return ok != 0;
+}
 __device__ __forceinline__ uint64_t globaltimer_ns() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -43,9 +56,13 @@ static __device__ int g_snp_watchdog_mode;   // 0: trap, 1: record and release a
 // means a broken pipeline: trap (a launch error) instead of hanging the GPU.
 static __device__ __noinline__ void mbar_wait_slow(uint64_t *bar, uint32_t parity) {
     const uint64_t t0 = globaltimer_ns();
-    while (!mbar_try_wait(bar, parity)) {
+    const int mode = g_snp_watchdog_mode;   // read once: no global load per poll
+    for (;;) {
+#pragma unroll 1
+        for (int i = 0; i < 16; ++i)
+            if (mbar_try_wait_sleep(bar, parity, 100000u)) return;
         if (globaltimer_ns() - t0 > 4000000000ull) {
-            if (g_snp_watchdog_mode == 0) __trap();
+            if (mode == 0) __trap();
             if (atomicCAS(&g_snp_watchdog[0], 0, 1) == 0) {
                 g_snp_watchdog[1] = blockIdx.x;
                 g_snp_watchdog[2] = threadIdx.x;
@@ -54,7 +71,7 @@ static __device__ __noinline__ void mbar_wait_slow(uint64_t *bar, uint32_t parit
             }
             return;
         }
-        if (g_snp_watchdog_mode && *(volatile int *)&g_snp_watchdog[0]) return;
+        if (mode && *(volatile int *)&g_snp_watchdog[0]) return;
     }
 }
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
@@ -72,7 +89,10 @@ __device__ __forceinline__ void mbar_wait_warp(uint64_t *bar, uint32_t parity) {
 // (no per-MMA R2UR conversions; the tcgen05.mma issue path stays on the uniform datapath).
 static __device__ __noinline__ void mbar_wait_uniform_slow(uint64_t *bar, uint32_t parity) {
     const uint64_t t0 = globaltimer_ns();
-    while (!__all_sync(0xffffffffu, mbar_try_wait(bar, parity))) {
+    for (;;) {
+#pragma unroll 1
+        for (int i = 0; i < 16; ++i)
+            if (__all_sync(0xffffffffu, mbar_try_wait_sleep(bar, parity, 100000u))) return;
         if (__any_sync(0xffffffffu, globaltimer_ns() - t0 > 4000000000ull)) __trap();
     }
 }

@@ -1,0 +1,4 @@
+set -x
+mkdir -p gpurun_out/prof
+SNP_DEBUG_SKIP_EXPAND=1 timeout 600 ncu --set full --clock-control none --import-source on -k regex:gemm_tc4 -s 1 -c 1 -o gpurun_out/prof/ld_r2_skip python scripts/ld_one.py > gpurun_out/ncu_ld1.log 2>&1; echo $?
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:gemm_tc4 -s 1 -c 1 -o gpurun_out/prof/ld_r2 python scripts/ld_one.py > gpurun_out/ncu_ld2.log 2>&1; echo $?
