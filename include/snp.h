@@ -126,10 +126,12 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
 /* a3 + a4 — FastID comparison counts (Eqs. 2-3):
  *   out[i*ldo + j] (=|+=) sum_k op(Q_ik, D_jk)   for queries i < nq, DB rows j < nd.
  * Q: [nq][ldq] packed query profiles over SNPs, D: [nd][ldd] database profiles.
- * popQ/popD: optional row popcounts; may be NULL.  Every current variant derives
- * the popcounts it needs itself (the tensor-core kernels accumulate them from the
- * packed words they already stream for the identities XOR = pQ + pD - 2 AND,
- * ANDNOT = pQ - AND, NOTAND = pD - AND), so they are accepted but not read.
+ * popQ/popD: optional exact row popcounts over nbits (snp_row_popc); may be NULL.
+ * The tensor-core kernels need them for the identities XOR = pQ + pD - 2 AND,
+ * ANDNOT = pQ - AND, NOTAND = pD - AND: given ones are read as they are (the FastID
+ * kernel then skips counting the streamed database words), NULL ones are derived
+ * in-kernel from the packed words or by a pre-pass.  The CUDA-core variant ignores
+ * them (one LOP3 per op).
  * out: uint32 [nq][ldo], ldo >= nd. */
 snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t *popQ,
                       const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD,
@@ -157,6 +159,10 @@ snp_status snp_fastid_best(const uint32_t *counts, int64_t nq, int64_t nd, int64
  *               no best matches); entry j is uint32 [nq] / int64 [nq] (both NULL or
  *               both set): min count over the nd rows and index_base + lowest row
  *               attaining it (R4); nd == 0 gives 0xFFFFFFFF / -1.
+ *   popD:       uint32 [nd] database row popcounts over nbits (snp_row_popc), or NULL.
+ *               A database is resident and prepared once, so its popcounts
+ *               can be too; given, the kernel skips counting every streamed word.
+ *               They must be exact: wrong popcounts give wrong XOR/ANDNOT/NOTAND counts.
  * nd < 2^32 - 1.  ws: snp_fastid_search_workspace_bytes(nq, nd, nbits, nops) bytes
  * (never 0 when nq > 0).  Kernels: the fused tcgen05 kernel for nq <= 64 (two or three
  * launches: key init + search [+ pack by the caller]); other shapes / a forced
@@ -164,7 +170,8 @@ snp_status snp_fastid_best(const uint32_t *counts, int64_t nq, int64_t nd, int64
  * database through workspace counts when counts[j] is NULL. */
 size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int nops);
 snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
-                             const uint64_t *D, int64_t nd, int64_t ldd, int64_t nbits,
+                             const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD,
+                             int64_t nbits,
                              int nops, const int *ops, uint32_t *const *counts, int64_t ldo,
                              uint32_t *const *best_count, int64_t *const *best_index,
                              int64_t index_base, void *ws, size_t ws_bytes, void *stream);

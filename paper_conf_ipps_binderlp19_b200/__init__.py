@@ -208,7 +208,7 @@ def snp_fastid_search_workspace_bytes(nq: int, nd: int, nbits: int, nops: int) -
 
 def snp_fastid_search(Q: torch.Tensor, D: torch.Tensor, nbits: int, ops=("xor", "andnot"),
                       counts=True, best=True, index_base: int = 0, ldo: int | None = None,
-                      ws: torch.Tensor | None = None, stream=None):
+                      ws: torch.Tensor | None = None, popD: torch.Tensor | None = None, stream=None):
     """f1: one pass over D for every op in ops -> (counts list, best list).
 
     counts: True (allocate [nq][nd] uint32 per op), False (none) or a list of
@@ -250,7 +250,10 @@ def snp_fastid_search(Q: torch.Tensor, D: torch.Tensor, nbits: int, ops=("xor", 
     if ws is None:
         ws = _workspace(need, dev)
     any_best = any(b is not None for b in best)
-    check(lib().snp_fastid_search(_ptr(Q), nq, _ld(Q), _ptr(D), nd, _ld(D), int(nbits), k,
+    _dev_tensor(popD, "popD", _U32)
+    if popD is not None and popD.numel() < nd:
+        raise ValueError("popD needs one popcount per database row")
+    check(lib().snp_fastid_search(_ptr(Q), nq, _ld(Q), _ptr(D), nd, _ld(D), _ptr(popD), int(nbits), k,
                                   ctypes.cast(ops_arr, ctypes.c_void_p), ctypes.cast(c_arr, ctypes.c_void_p), ld,
                                   ctypes.cast(bc_arr, ctypes.c_void_p) if any_best else None,
                                   ctypes.cast(bi_arr, ctypes.c_void_p) if any_best else None,

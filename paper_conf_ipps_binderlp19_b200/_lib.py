@@ -25,7 +25,7 @@ SIGNATURES = {
     "snp_fastid": (_int, [_p, _i64, _i64, _p, _p, _i64, _i64, _p, _i64, _int, _p, _i64, _int, _p, _sz, _p]),
     "snp_fastid_best": (_int, [_p, _i64, _i64, _i64, _i64, _p, _p, _p]),
     "snp_fastid_search_workspace_bytes": (_sz, [_i64, _i64, _i64, _int]),
-    "snp_fastid_search": (_int, [_p, _i64, _i64, _p, _i64, _i64, _i64, _int, _p, _p, _i64, _p, _p, _i64,
+    "snp_fastid_search": (_int, [_p, _i64, _i64, _p, _i64, _i64, _p, _i64, _int, _p, _p, _i64, _p, _p, _i64,
                                  _p, _sz, _p]),
     "snp_shard_plan": (_int, [_i64, _int, _i64, _p]),
     "snp_set_variant": (_int, [_int]),

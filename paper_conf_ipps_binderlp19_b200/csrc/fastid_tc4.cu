@@ -31,6 +31,7 @@ namespace snp {
 // clock64 stamps per iteration: [0] expander before waits, [1] after pfull+empty,
 // [2] before full arrive, [3] MMA after full wait.  Enabled by SNP_TRACE=1.
 __device__ long long g_fastid_trace[8 * 1024];
+__device__ long long g_fastid_etrace[4 * 256];   // FASTID_TRACE2: per tile, CTA 0
 __device__ long long g_fastid_cta_time[3 * 1024];
 __device__ long long g_fastid_launch_time[2 * 64];   // CTA 0: start / end globaltimer per launch
 __device__ unsigned int g_fastid_launch_ctr;   // per CTA: start, main loop start, end (globaltimer ns)
@@ -40,23 +41,42 @@ namespace {
 constexpr int BM = 128;
 constexpr int KBITS = 512;
 static_assert(KBITS == 512, "a stage is exactly the 8 K=64 MMAs of mma8_mxf4_ts_commit");
-constexpr int NP = 8;                   // packed TMA ring depth (64 KB in flight per SM)
+#ifndef FASTID_NP
+#define FASTID_NP 8
+#endif
+#ifndef FASTID_NS
+#define FASTID_NS 4
+#endif
+constexpr int NP = FASTID_NP;           // packed TMA ring depth (64 KB in flight per SM)
 constexpr int PSTAGE = BM * KBITS / 8;  // 8 KB packed per stage, 64-byte rows, 64B-swizzled
-constexpr int G = 4;                    // expander groups (group g takes stages it = g mod G)
-constexpr int NEXP = 4 * G;             // expander warps: group g = warps 4g..4g+3 (one per lane quarter)
+#ifndef FASTID_G
+#define FASTID_G 4
+#endif
+#ifndef FASTID_NEPI
+#define FASTID_NEPI 8
+#endif
+// Warp roles for GG expander groups (group g takes stages it = g mod GG; 4 warps each, one
+// per TMEM lane quarter).  GG = 4 when the expanders also count the database popcounts;
+// GG = 2 when the caller gives them (fewer warps competing for issue slots: measured
+// 203 vs 220 us on FastID-1M).
 // The warp scheduler favours higher warp ids, so the latency-critical single-thread
 // roles get the highest ids: MMA issuer last, TMA producer next, epilogue below them.
-constexpr int NEPI = 8;                 // epilogue warps 16..23: lane quarter w % 4, column half
-constexpr int EPI_WARP0 = NEXP;
-constexpr int TMA_WARP = NEXP + NEPI;   // 24
-constexpr int MMA_WARP = NEXP + NEPI + 1;   // 25
-constexpr int NTHREADS = (NEXP + NEPI + 2) * 32;
+constexpr int NEPI = FASTID_NEPI;       // epilogue warps: lane quarter w % 4, column block w / 4
+template <int GG>
+struct Roles {
+    static constexpr int G = GG;
+    static constexpr int NEXP = 4 * GG;
+    static constexpr int EPI_WARP0 = NEXP;
+    static constexpr int TMA_WARP = NEXP + NEPI;
+    static constexpr int MMA_WARP = NEXP + NEPI + 1;
+    static constexpr int NTHREADS = (NEXP + NEPI + 2) * 32;
+};
 constexpr size_t MAX_SMEM = 232448;     // 227 KB opt-in
 
 template <int BN>
 struct FCfg {
-    static constexpr int NS = 4;                    // TMEM A stages of 64 columns (multiple of G)
-    static_assert(NS % G == 0 && NP % G == 0, "rings must be multiples of the group count");
+    static constexpr int NS = FASTID_NS;            // TMEM A stages of 64 columns (multiple of G)
+    static_assert(NS % 4 == 0 && NP % 4 == 0, "rings must be multiples of the group count");
     static constexpr int ACC_COLS = BN;
     static constexpr int A_COL0 = 2 * ACC_COLS;
     static constexpr int SF_COL = A_COL0 + NS * 64;
@@ -92,6 +112,8 @@ struct FArgs {
     size_t qbytes;       // expanded query bytes in shared memory
     int trace;
     int nostore;         // profiling experiment: skip the output stores
+    const uint32_t *popDg;   // database row popcounts (resident with the database), or NULL:
+                             // then the expanders count them from the streamed words
 };
 
 __device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
@@ -150,6 +172,15 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32
         : "memory");
 }
 
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
+    __syncwarp();   // warp-collective (.sync.aligned): converge first
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+        : "r"(taddr));
+}
+
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
     __syncwarp();   // warp-collective (.sync.aligned): converge first
     asm volatile(
@@ -174,9 +205,12 @@ __host__ __device__ constexpr uint32_t op_cq(int op) { return (op == 1 || op == 
 __host__ __device__ constexpr uint32_t op_cd(int op) { return (op == 1 || op == 3) ? 1u : 0u; }
 __host__ __device__ constexpr uint32_t op_cc(int op) { return op == 0 ? 1u : op == 1 ? (uint32_t)-2 : (uint32_t)-1; }
 
-template <int BN, int NOPS, bool BEST, bool ACC, int OPS>
-__global__ void __launch_bounds__(NTHREADS, 1)
+template <int BN, int NOPS, bool BEST, bool ACC, int OPS, int GG>
+__global__ void __launch_bounds__(Roles<GG>::NTHREADS, 1)
 fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
+    constexpr int G = GG, NEXP = Roles<GG>::NEXP, EPI_WARP0 = Roles<GG>::EPI_WARP0;
+    constexpr int TMA_WARP = Roles<GG>::TMA_WARP, MMA_WARP = Roles<GG>::MMA_WARP;
+    constexpr int NTHREADS = Roles<GG>::NTHREADS;
     using C = FCfg<BN>;
     constexpr int NS = C::NS;
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -232,20 +266,33 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     ptx::tc_fence_after();
     const uint32_t tmem = *tmem_slot;
 
-    // ---- prologue: expand the whole query batch once (resident MMA B operand)
+    // ---- prologue: expand the whole query batch once (resident MMA B operand).  Warp w
+    // takes words w, w + 26, ...; lane = query row (BN / 32 rows per lane), so the 16-byte
+    // stores of a warp are contiguous (conflict-free) and the loads of consecutive words are
+    // independent (unrolled); row popcounts: one shared atomic per thread and row.
     {
-        const int64_t nchunks = (int64_t)nst * (KBITS / 32);
+        constexpr int RPL = BN / 32;
+        const int64_t nchunks = (int64_t)nst * (KBITS / 32);   // 32-bit words per row
         const int64_t nw32 = ((nbits + 127) / 128) * 4;
-        for (int64_t idx = tid; idx < (int64_t)BN * nchunks; idx += NTHREADS) {
-            const int row = (int)(idx % BN);
-            const int64_t w = idx / BN;
-            uint32_t x = 0;
-            if (row < args.nq && w < nw32) x = __ldg(args.Q + row * args.ldq32 + w) & word_mask(w, nbits);
-            if (x) atomicAdd(&popQ[row], (uint32_t)__popc(x));
-            uint4 o;
-            expandB(x, o.x, o.y, o.z, o.w);   // queries: MMA B operand
-            *reinterpret_cast<uint4 *>(qsm + (size_t)w * BN * 16 + row * 16) = o;
+        uint32_t pc[RPL];
+#pragma unroll
+        for (int h = 0; h < RPL; ++h) pc[h] = 0;
+#pragma unroll 4
+        for (int64_t w = warp; w < nchunks; w += NTHREADS / 32) {
+#pragma unroll
+            for (int h = 0; h < RPL; ++h) {
+                const int row = 32 * h + lane;
+                uint32_t x = 0;
+                if (row < args.nq && w < nw32) x = __ldg(args.Q + row * args.ldq32 + w) & word_mask(w, nbits);
+                pc[h] += __popc(x);
+                uint4 o;
+                expandB(x, o.x, o.y, o.z, o.w);   // queries: MMA B operand
+                *reinterpret_cast<uint4 *>(qsm + (size_t)w * BN * 16 + row * 16) = o;
+            }
         }
+#pragma unroll
+        for (int h = 0; h < RPL; ++h)
+            if (pc[h]) atomicAdd(&popQ[32 * h + lane], pc[h]);
     }
     if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {   // one warp per lane quarter
         const int q = warp & 3;
@@ -290,7 +337,9 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         const int arow = qa * 32 + lane;
         uint32_t popa = 0;
         int64_t cur_tl = 0;   // tile whose popcount partial is being accumulated
+        const bool pre = args.popDg != nullptr;
         auto publish_until = [&](int64_t upto) {
+            if (pre) return;
             for (; cur_tl < upto; ++cur_tl) {
                 const int acc = (int)(cur_tl & 1);
                 if (cur_tl >= 2) ptx::mbar_wait_warp(&acce[acc], (uint32_t)(((cur_tl >> 1) - 1) & 1));
@@ -309,6 +358,9 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             const bool tr = args.trace && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
             if (tr) g_fastid_trace[8 * it + 0] = clock64();
             ptx::mbar_wait_warp(&pfull[p], pround & 1);
+#ifdef FASTID_TRACE2
+            if (tr) g_fastid_trace[8 * it + 4] = clock64();
+#endif
             if (bround > 0) ptx::mbar_wait_warp(&empty[b], (bround - 1) & 1);
             if (tr) g_fastid_trace[8 * it + 1] = clock64();
             // 64-byte row of the stage; TMA 64B swizzle: 16-byte chunk c of row r sits at
@@ -326,8 +378,10 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #pragma unroll
                 for (int i = 0; i < 16; ++i) wv[i] &= word_mask(w0 + i, nbits);
             }
+            if (!pre) {
 #pragma unroll
-            for (int i = 0; i < 16; ++i) popa += __popc(wv[i]);
+                for (int i = 0; i < 16; ++i) popa += __popc(wv[i]);
+            }
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&pempty[p]);
             const uint32_t tbase = tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + 64 * b);
@@ -371,13 +425,25 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         int64_t itm = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
+#ifdef FASTID_TRACE2
+            if (args.trace && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 0] = clock64();
+#endif
             if (tl >= 2) ptx::mbar_wait_uniform(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+#ifdef FASTID_TRACE2
+            if (args.trace && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 1] = clock64();
+#endif
             ptx::tc_fence_after();
             const uint32_t d = tmu + (uint32_t)(acc * C::ACC_COLS);
             uint64_t bd = bdesc0;
             for (int s = 0; s < nst; ++s, ++itm) {
+#ifdef FASTID_TRACE2
+                if (args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 3] = clock64();
+#endif
                 ptx::mbar_wait_uniform(&full[b], bround & 1);
                 ptx::tc_fence_after();
+#ifdef FASTID_TRACE2
+                if (args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 5] = clock64();
+#endif
                 const uint32_t a0 = tmu + (uint32_t)(C::A_COL0 + 64 * b);
 #pragma unroll
                 for (int k = 0; k < KBITS / 64; ++k)
@@ -392,12 +458,14 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         __syncwarp();
     } else {
         // ------------------------------------------------------------ epilogue (8 warps)
-        // warp e: TMEM lane quarter e % 4 (database rows), query columns [32 h, 32 h + 32)
+        // warp e: TMEM lane quarter e % 4 (database rows), query columns [EC h, EC h + EC)
+        constexpr int EC = BN * 4 / NEPI;   // 32 (8 epilogue warps) or 16 (16 warps)
+        static_assert(EC == 16 || EC == 32, "epilogue column block");
         const int e = warp - EPI_WARP0;
         const int q = e & 3, h = e >> 2;
         const int li = q * 32 + lane;
-        const int c0 = 32 * h;
-        const int ncols = (int)(args.nq - c0 < 32 ? (args.nq - c0 > 0 ? args.nq - c0 : 0) : 32);
+        const int c0 = EC * h;
+        const int ncols = (int)(args.nq - c0 < EC ? (args.nq - c0 > 0 ? args.nq - c0 : 0) : EC);
         const int64_t ldo = args.ldo;
         // running best of column c0 + lane, per op (held by that lane only)
         uint32_t bc[NOPS], bi[NOPS];
@@ -407,14 +475,23 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             const int acc = (int)(tl & 1);
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
             const int64_t t = blockIdx.x + tl * gridDim.x;
-            ptx::mbar_wait_warp(&popf[acc], ph);
+            const bool pre = args.popDg != nullptr;
+            const int64_t gd_l = t * BM + li;   // this lane's local database row
+            uint32_t pd = 0;
+            if (pre) pd = gd_l < args.nd ? __ldg(args.popDg + gd_l) : 0u;   // before the wait
+            else ptx::mbar_wait_warp(&popf[acc], ph);
             ptx::mbar_wait_warp(&accf[acc], ph);
+#ifdef FASTID_TRACE2
+            if (args.trace && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 2] = clock64();
+#endif
             ptx::tc_fence_after();
-            uint32_t v[32];
-            tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
-            uint32_t pd = 0;   // read the popcount partials BEFORE releasing the buffer pair
+            uint32_t v[EC];
+            if constexpr (EC == 32) tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
+            else tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
+            if (!pre) {   // read the popcount partials BEFORE releasing the buffer pair
 #pragma unroll
-            for (int gg = 0; gg < G; ++gg) pd += popD[(acc * G + gg) * BM + li];
+                for (int gg = 0; gg < G; ++gg) pd += popD[(acc * G + gg) * BM + li];
+            }
             ptx::tmem_ld_wait();
             ptx::tc_fence_before();
             __syncwarp();
@@ -454,7 +531,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #pragma unroll
             for (int j = 0; j < NOPS; ++j) mk[j] = 0xffffffffu;
 #pragma unroll
-            for (int u = 0; u < 32; ++u) {
+            for (int u = 0; u < EC; ++u) {
                 const uint32_t fb = __float_as_uint(__fadd_rn(__uint_as_float(v[u]), 8388608.0f));
                 const uint32_t pq32 = popQ32[c0 + u];
                 const bool colok = u < ncols;
@@ -493,6 +570,9 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                     }
                 }
             }
+#ifdef FASTID_TRACE2
+            if (args.trace && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 3] = clock64();
+#endif
         }
         if (BEST) {
 #pragma unroll
@@ -581,7 +661,7 @@ void op_coefs(int op, uint32_t &cq, uint32_t &cd, uint32_t &cc) {
     }
 }
 
-template <int BN>
+template <int BN, int GG>
 cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     // the database is the B operand of the user call (Q op D), on TMEM lanes here
     FArgs f{};
@@ -589,6 +669,7 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     f.nq = a.nq;
     f.ldq32 = a.ldq32;
     f.nd = a.nd;
+    f.popDg = a.popD;
     f.nbits = a.nbits;
     f.nops = a.nops;
     f.accumulate = a.accumulate;
@@ -630,28 +711,31 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     const bool best = f.best_mask != 0;
     KernFn kern = nullptr;
     int ki = 0;
+    int nthreads = Roles<GG>::NTHREADS;   // the runtime-coefficient kernels are GG = 4 only
     if (a.accumulate) {
+        nthreads = Roles<4>::NTHREADS;
         if (a.nops != 1 || best) return cudaErrorInvalidValue;
-        kern = fastid_tc4_kernel<BN, 1, false, true, -1>; ki = 0;
+        kern = fastid_tc4_kernel<BN, 1, false, true, -1, 4>; ki = 0;
     } else if (a.nops == 1) {   // compile-time op
-        static KernFn k1[2][4] = {{fastid_tc4_kernel<BN, 1, false, false, 0>, fastid_tc4_kernel<BN, 1, false, false, 1>,
-                                   fastid_tc4_kernel<BN, 1, false, false, 2>, fastid_tc4_kernel<BN, 1, false, false, 3>},
-                                  {fastid_tc4_kernel<BN, 1, true, false, 0>, fastid_tc4_kernel<BN, 1, true, false, 1>,
-                                   fastid_tc4_kernel<BN, 1, true, false, 2>, fastid_tc4_kernel<BN, 1, true, false, 3>}};
+        static KernFn k1[2][4] = {{fastid_tc4_kernel<BN, 1, false, false, 0, GG>, fastid_tc4_kernel<BN, 1, false, false, 1, GG>,
+                                   fastid_tc4_kernel<BN, 1, false, false, 2, GG>, fastid_tc4_kernel<BN, 1, false, false, 3, GG>},
+                                  {fastid_tc4_kernel<BN, 1, true, false, 0, GG>, fastid_tc4_kernel<BN, 1, true, false, 1, GG>,
+                                   fastid_tc4_kernel<BN, 1, true, false, 2, GG>, fastid_tc4_kernel<BN, 1, true, false, 3, GG>}};
         kern = k1[best][a.ops[0] & 3];
         ki = 1 + 4 * best + (a.ops[0] & 3);
     } else if (a.nops == 2 && a.ops[0] == 1 && a.ops[1] == 2) {   // XOR + ANDNOT (identity + mixture)
-        kern = best ? fastid_tc4_kernel<BN, 2, true, false, 1 | (2 << 2)>
-                    : fastid_tc4_kernel<BN, 2, false, false, 1 | (2 << 2)>;
+        kern = best ? fastid_tc4_kernel<BN, 2, true, false, 1 | (2 << 2), GG>
+                    : fastid_tc4_kernel<BN, 2, false, false, 1 | (2 << 2), GG>;
         ki = 9 + best;
     } else {
+        nthreads = Roles<4>::NTHREADS;
         switch (a.nops * 2 + (best ? 1 : 0)) {
-        case 4: kern = fastid_tc4_kernel<BN, 2, false, false, -1>; ki = 11; break;
-        case 5: kern = fastid_tc4_kernel<BN, 2, true, false, -1>; ki = 12; break;
-        case 6: kern = fastid_tc4_kernel<BN, 3, false, false, -1>; ki = 13; break;
-        case 7: kern = fastid_tc4_kernel<BN, 3, true, false, -1>; ki = 14; break;
-        case 8: kern = fastid_tc4_kernel<BN, 4, false, false, -1>; ki = 15; break;
-        case 9: kern = fastid_tc4_kernel<BN, 4, true, false, -1>; ki = 16; break;
+        case 4: kern = fastid_tc4_kernel<BN, 2, false, false, -1, 4>; ki = 11; break;
+        case 5: kern = fastid_tc4_kernel<BN, 2, true, false, -1, 4>; ki = 12; break;
+        case 6: kern = fastid_tc4_kernel<BN, 3, false, false, -1, 4>; ki = 13; break;
+        case 7: kern = fastid_tc4_kernel<BN, 3, true, false, -1, 4>; ki = 14; break;
+        case 8: kern = fastid_tc4_kernel<BN, 4, false, false, -1, 4>; ki = 15; break;
+        case 9: kern = fastid_tc4_kernel<BN, 4, true, false, -1, 4>; ki = 16; break;
         default: return cudaErrorInvalidValue;
         }
     }
@@ -670,7 +754,7 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }
-    kern<<<grid, NTHREADS, smem, s>>>(tm, f);
+    kern<<<grid, nthreads, smem, s>>>(tm, f);
     count_launches(1);
     return cudaGetLastError();
 }
@@ -692,10 +776,12 @@ cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     SearchArgs sa{};
     sa.Q = a.A; sa.nq = a.m; sa.ldq32 = a.lda32;
     sa.D = a.B; sa.nd = a.n; sa.ldd32 = a.ldb32;
+    sa.popD = a.popB;   // the user's popD (NULL: counted in-kernel)
     sa.nbits = a.nbits;
     sa.nops = 1; sa.ops[0] = a.op; sa.counts[0] = a.C;
     sa.ldo = a.ldc; sa.accumulate = a.accumulate;
-    return launch_f<64>(sa, s);   // queries <= 64 (fastid_tc4_supported)
+    // queries <= 64 (fastid_tc4_supported)
+    return sa.popD ? launch_f<64, 2>(sa, s) : launch_f<64, 4>(sa, s);
 }
 
 size_t fastid_search_tc4_ws_bytes(int64_t nq, int nops) {
@@ -703,7 +789,7 @@ size_t fastid_search_tc4_ws_bytes(int64_t nq, int nops) {
 }
 
 cudaError_t launch_fastid_search_tc4(const SearchArgs &a, cudaStream_t s) {
-    return launch_f<64>(a, s);
+    return a.popD ? launch_f<64, 2>(a, s) : launch_f<64, 4>(a, s);
 }
 
 }  // namespace snp
@@ -718,6 +804,11 @@ extern "C" int snp_debug_fastid_launch_times(long long *host, int n) {
 extern "C" int snp_debug_fastid_cta_times(long long *host, int n) {
     if (n > 3 * 1024) n = 3 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_cta_time, sizeof(long long) * n);
+}
+
+extern "C" int snp_debug_fastid_etrace(long long *host, int n) {
+    if (n > 4 * 256) n = 4 * 256;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_etrace, sizeof(long long) * n);
 }
 
 extern "C" int snp_debug_fastid_trace(long long *host, int n) {

@@ -162,8 +162,10 @@ __device__ __forceinline__ void ld_stats_f32(int64_t n, int64_t na, int64_t nb, 
 }
 
 
-// 1/d rounded once to fp32 (d exact in fp64); 0 for d = 0 (monomorphic SNP: r2 = 0).
-__device__ __forceinline__ float inv_exact(int64_t d) { return d ? (float)(1.0 / (double)d) : 0.f; }
+// 1/d in fp32: d rounded to fp32, then a correctly rounded reciprocal (2 roundings; FP64
+// division is avoided: the DFMA pipe throttled the epilogue); 0 for d = 0 (monomorphic
+// SNP: r2 = 0).
+__device__ __forceinline__ float inv_exact(int64_t d) { return d ? __frcp_rn((float)d) : 0.f; }
 
 // Exact count from the fp32 accumulator (an integer < 2^24): the 2^23 magic add below
 // 2^23 (FMA pipe, no F2I), F2I above.
@@ -180,8 +182,8 @@ __device__ __forceinline__ uint32_t acc_count(uint32_t v, bool small) {
 // are broadcast from their lane by shuffles.
 //   counts: x = op identity of SURVEY §8a a4 with (pQ, pD) = (row, column) popcounts
 //   LD:     reading R3 from exact integers: num = n nAB - nA nB (int32 for n <= 46340),
-//           r2 = min(1, (num / da) (num / db)) with 1/da, 1/db rounded once: 7 fp32
-//           roundings in total, relative error <= 7 * 2^-24 = 4.2e-7;
+//           r2 = min(1, (num / da) (num / db)) with 1/da, 1/db from 2 roundings each: 9
+//           fp32 roundings in total, relative error <= 9 * 2^-24 = 5.4e-7;
 //           exactly 0 where num = 0.  D' = num / Dmax (correctly rounded division).
 template <int EPI>
 __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[32], uint32_t *tw, int lane,

@@ -298,9 +298,10 @@ snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t
     a.B = reinterpret_cast<const uint32_t *>(D);
     a.m = nq; a.n = nd; a.lda32 = 2 * ldq; a.ldb32 = 2 * ldd; a.nbits = nbits;
     a.op = op; a.accumulate = accumulate ? 1 : 0; a.ldc = ldo; a.C = out;
+    a.popA = popQ; a.popB = popD;
     if (variant == SNP_VARIANT_TC) {
-        // every tensor-core kernel accumulates both operands' popcounts from the packed
-        // words it streams (no extra pass over the database); popQ/popD are not needed
+        // given popcounts are used as they are (the FastID kernel skips counting the
+        // streamed database words); NULL ones are derived in-kernel or by a pre-pass
         return run_gemm(a, EPI_COUNTS, variant, ws, ws_bytes, s);
     }
     return run_gemm(a, EPI_COUNTS, variant, nullptr, 0, s);
@@ -363,7 +364,7 @@ size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, 
 }
 
 snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
-                             const uint64_t *D, int64_t nd, int64_t ldd, int64_t nbits,
+                             const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD, int64_t nbits,
                              int nops, const int *ops, uint32_t *const *counts, int64_t ldo,
                              uint32_t *const *best_count, int64_t *const *best_index,
                              int64_t index_base, void *ws, size_t ws_bytes, void *stream) {
@@ -407,6 +408,7 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
     a.nq = nq; a.ldq32 = 2 * ldq;
     a.D = reinterpret_cast<const uint32_t *>(D);
     a.nd = nd; a.ldd32 = 2 * ldd;
+    a.popD = popD;
     a.nbits = nbits;
     a.nops = nops;
     a.ldo = ldo;
@@ -445,7 +447,7 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
         if (a.counts[j] && nd > 0) {
             GemmArgs g{};
             g.A = a.Q; g.B = a.D; g.m = nq; g.n = nd; g.lda32 = a.ldq32; g.ldb32 = a.ldd32;
-            g.nbits = nbits; g.op = ops[j]; g.ldc = ldo; g.C = a.counts[j];
+            g.nbits = nbits; g.op = ops[j]; g.ldc = ldo; g.C = a.counts[j]; g.popB = popD;
             if ((st = run_gemm(g, EPI_COUNTS, variant, gws, gws_bytes, s)) != SNP_OK) return st;
             if (best && (e = launch_best_reduce(a.counts[j], nq, nd, ldo, 0, kj, s)) != cudaSuccess)
                 return set_cuda_error(e);
@@ -456,6 +458,7 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
                 GemmArgs g{};
                 g.A = a.Q; g.B = a.D + j0 * a.ldd32; g.m = nq; g.n = rows;
                 g.lda32 = a.ldq32; g.ldb32 = a.ldd32;
+                g.popB = popD ? popD + j0 : nullptr;
                 g.nbits = nbits; g.op = ops[j]; g.ldc = ch; g.C = chunk;
                 if ((st = run_gemm(g, EPI_COUNTS, cv, gws, gws_bytes, s)) != SNP_OK) return st;
                 if ((e = launch_best_reduce(chunk, nq, rows, ch, j0, kj, s)) != cudaSuccess)

@@ -52,6 +52,7 @@ struct SearchArgs {
     int64_t nq, ldq32;
     const uint32_t *D;   // [nd][ldd32] database
     int64_t nd, ldd32;
+    const uint32_t *popD;     // [nd] database row popcounts or NULL (derived in-kernel)
     int64_t nbits;
     int nops;
     int ops[4];

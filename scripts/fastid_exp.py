@@ -17,10 +17,14 @@ def t(fn, n=20):
     e.record(); torch.cuda.synchronize()
     return s.elapsed_time(e) / n
 res = {}
+pd = snp.snp_row_popc(D, nbits)
+res["2ops counts+best popD"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=outs, best=True, popD=pd))
+res["2ops best only popD"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False, best=True, popD=pd))
 res["2ops counts+best"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=outs, best=True))
 res["2ops best only"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False, best=True))
 res["1op counts+best"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor",), counts=outs[:1], best=True))
 res["1op counts"] = t(lambda: snp.snp_fastid(Q, D, nbits, "xor", out=outs[0]))
+res["1op counts popD"] = t(lambda: snp.snp_fastid(Q, D, nbits, "xor", out=outs[0], popD=pd))
 res["1op best only"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor",), counts=False, best=True))
 rd = nd * w * 8
 print(json.dumps({k: {"us": 1e3 * v, "GBps_read_only": rd / v / 1e6} for k, v in res.items()}), flush=True)

@@ -1,0 +1,46 @@
+"""Pipeline trace of CTA 0 of the fused FastID search (build with -DFASTID_TRACE2):
+per stage it: expander [0] start, [4] after pfull wait, [1] after empty wait, [2] before
+full arrive; MMA warp [3] before full wait, [5] after it."""
+import ctypes, os, sys
+os.environ["SNP_TRACE"] = "1"
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import paper_conf_ipps_binderlp19_b200 as snp
+torch.cuda.set_device(0)
+nq, nd, nbits = 64, 1_000_000, 4096
+w = snp.snp_words(nbits)
+D = torch.randint(-2**62, 2**62, (nd, w), dtype=torch.int64, device="cuda").view(torch.uint64)
+Q = torch.randint(-2**62, 2**62, (nq, w), dtype=torch.int64, device="cuda").view(torch.uint64)
+pd = snp.snp_row_popc(D, nbits)
+outs = [torch.empty((nq, nd), dtype=torch.uint32, device="cuda") for _ in range(2)]
+mode = os.environ.get("MODE", "search")
+for _ in range(3):
+    if mode == "search":
+        snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=outs, best=True, popD=pd)
+    else:
+        snp.snp_fastid(Q, D, nbits, "xor", out=outs[0])
+torch.cuda.synchronize()
+buf = (ctypes.c_longlong * 8192)()
+snp.lib().snp_debug_fastid_trace(buf, 8192)
+t = np.array(buf, dtype=np.int64).reshape(1024, 8)
+nit = 53 * 8
+t = t[:nit]
+v = slice(16, nit - 8)
+def med(x): return float(np.median(x))
+print("mode", mode)
+print("expander: pfull wait", med(t[v, 4] - t[v, 0]), " empty wait", med(t[v, 1] - t[v, 4]),
+      " produce", med(t[v, 2] - t[v, 1]), " iteration", med(np.diff(t[16:nit:4, 0])) if False else "")
+print("MMA: wait for full", med(t[v, 5] - t[v, 3]), " full-arrive->MMA got", med(t[v, 5] - t[v, 2]),
+      " MMA stage interval", med(np.diff(t[16:nit - 8, 5])), " mean", float(np.diff(t[16:nit - 8, 5]).mean()))
+print("stage throughput (cycles/stage) over CTA:", (t[nit - 1, 5] - t[8, 5]) / (nit - 9))
+for it in range(40, 56):
+    r = t[it] - t[0, 0]
+    print(it, r[0], r[4], r[1], r[2], "| mma", r[3], r[5])
+
+eb = (ctypes.c_longlong * 1024)()
+snp.lib().snp_debug_fastid_etrace(eb, 1024)
+e = np.array(eb, dtype=np.int64).reshape(256, 4)[:53]
+print("tile: MMA acce wait", med(e[2:50, 1] - e[2:50, 0]), "mean", float((e[2:50, 1] - e[2:50, 0]).mean()),
+      " epilogue busy (accf->done)", med(e[2:50, 3] - e[2:50, 2]), " tile interval (MMA)", med(np.diff(e[2:50, 1])))
+for k in range(10, 16):
+    print(k, e[k] - e[0, 0])

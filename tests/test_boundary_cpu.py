@@ -152,29 +152,29 @@ def test_search_validation_before_launch(snplib):
     half = P2(FAKE, None)
     cast = lambda a: ctypes.cast(a, ctypes.c_void_p)   # noqa: E731
     # (Q, nq, ldq, D, nd, ldd, nbits, nops, ops, counts, ldo, best_count, best_index, base, ws, ws_bytes, stream)
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 0, cast(ops), null, 9, null, null, 0, p, 1 << 20, null) == E_OP
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 5, cast(ops), null, 9, null, null, 0, p, 1 << 20, null) == E_OP
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 2, cast(badops), null, 9, null, null, 0, p, 1 << 20,
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 0, cast(ops), null, 9, null, null, 0, p, 1 << 20, null) == E_OP
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 5, cast(ops), null, 9, null, null, 0, p, 1 << 20, null) == E_OP
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 2, cast(badops), null, 9, null, null, 0, p, 1 << 20,
                                null) == E_OP
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 2, null, null, 9, null, null, 0, p, 1 << 20, null) == E_NULL
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 2, null, null, 9, null, null, 0, p, 1 << 20, null) == E_NULL
     # best_count array without best_index array, and a half-set (count, index) pair
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 2, cast(ops), null, 9, cast(outs), null, 0, p, 1 << 20,
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 2, cast(ops), null, 9, cast(outs), null, 0, p, 1 << 20,
                                null) == E_NULL
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 2, cast(ops), null, 9, cast(outs), cast(half), 0, p,
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 2, cast(ops), null, 9, cast(outs), cast(half), 0, p,
                                1 << 20, null) == E_NULL
     # counts need ldo >= nd; packed operands validated like snp_fastid
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 2, cast(ops), cast(outs), 8, null, null, 0, p, 1 << 20,
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 2, cast(ops), cast(outs), 8, null, null, 0, p, 1 << 20,
                                null) == E_SHAPE
-    assert L.snp_fastid_search(p, 4, 1, p, 9, 2, 100, 2, cast(ops), cast(outs), 9, null, null, 0, p, 1 << 20,
+    assert L.snp_fastid_search(p, 4, 1, p, 9, 2, null, 100, 2, cast(ops), cast(outs), 9, null, null, 0, p, 1 << 20,
                                null) == E_SHAPE
-    assert L.snp_fastid_search(p, 4, 2, p, 1 << 32, 2, 100, 2, cast(ops), cast(outs), 1 << 32, null, null, 0, p,
+    assert L.snp_fastid_search(p, 4, 2, p, 1 << 32, 2, null, 100, 2, cast(ops), cast(outs), 1 << 32, null, null, 0, p,
                                1 << 20, null) == E_RANGE
     # nothing requested / nq == 0: valid no-ops
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 2, cast(ops), null, 9, null, null, 0, null, 0, null) == OK
-    assert L.snp_fastid_search(p, 0, 2, p, 9, 2, 100, 2, cast(ops), cast(outs), 9, null, null, 0, null, 0,
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 2, cast(ops), null, 9, null, null, 0, null, 0, null) == OK
+    assert L.snp_fastid_search(p, 0, 2, p, 9, 2, null, 100, 2, cast(ops), cast(outs), 9, null, null, 0, null, 0,
                                null) == OK
     # the workspace is always required when there is work
-    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, 100, 2, cast(ops), cast(outs), 9, null, null, 0, null, 0,
+    assert L.snp_fastid_search(p, 4, 2, p, 9, 2, null, 100, 2, cast(ops), cast(outs), 9, null, null, 0, null, 0,
                                null) == E_WORKSPACE
     assert snplib.snp_fastid_search_workspace_bytes(4, 9, 100, 2) >= 2 * 4 * 8
     assert snplib.snp_fastid_search_workspace_bytes(4, 0, 100, 2) >= 2 * 4 * 8

@@ -345,14 +345,17 @@ SEARCH_SHAPES = [(1, 4, 1), (3, 700, 129), (33, 1000, 4096), (64, 2000, 777), (6
 
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("nq,nd,nbits", SEARCH_SHAPES)
-def test_search_all_ops_counts_and_best(snp, variant, nq, nd, nbits):
+@pytest.mark.parametrize("pre", [False, True], ids=["popD_inkernel", "popD_given"])
+def test_search_all_ops_counts_and_best(snp, variant, nq, nd, nbits, pre):
     db = snpgen.fastid_db(31, np.arange(nd), nbits)
     q, _ = snpgen.fastid_queries(31, nq, nd, nbits)
     D = pack_dev(snp, db, garbage_seed=5)
     Q = pack_dev(snp, q, garbage_seed=6)
+    popD = snp.snp_row_popc(D, nbits) if pre else None
     _variant(snp, variant)
     try:
-        counts, best = snp.snp_fastid_search(Q, D, nbits, ALL_OPS, counts=True, best=True, index_base=7)
+        counts, best = snp.snp_fastid_search(Q, D, nbits, ALL_OPS, counts=True, best=True, index_base=7,
+                                             popD=popD)
         for j, op in enumerate(ALL_OPS):
             ref = oracle.counts(q, db, op)
             assert np.array_equal(u32(counts[j]), ref), (op, variant)
@@ -360,7 +363,7 @@ def test_search_all_ops_counts_and_best(snp, variant, nq, nd, nbits):
             assert np.array_equal(u32(best[j][0]), rb), op
             assert np.array_equal(best[j][1].cpu().numpy(), ri), op
         # best only (no count matrix written), two ops, chunked composition for big nq
-        _, best2 = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False, best=True)
+        _, best2 = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False, best=True, popD=popD)
         for j, op in enumerate(("xor", "andnot")):
             rb, ri = oracle.best(oracle.counts(q, db, op))
             assert np.array_equal(u32(best2[j][0]), rb) and np.array_equal(best2[j][1].cpu().numpy(), ri)
@@ -438,22 +441,25 @@ def test_cfg2_search_1m(snp, variant):
     cols = _sample_cols(nd, 128, 600, 10)
     dbs = snpgen.fastid_db(seed, cols, nbits)
     _variant(snp, variant)
+    popD = snp.snp_row_popc(D, nbits)   # resident with the database, as bench.py prepares it
     try:
-        counts, best = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"))
-        if variant == "auto":
-            assert snp.snp_last_kernel() == "fastid_mxf4"
-        for j, op in enumerate(("xor", "andnot")):
-            got = u32(counts[j].view(torch.int32)[:, torch.from_numpy(cols).to(DEV)])
-            assert np.array_equal(got, oracle.counts(q, dbs, op)), op
-            full = counts[j].cpu().numpy().astype(np.uint32)
-            assert np.array_equal(u32(best[j][0]), full.min(1)), op
-            assert np.array_equal(best[j][1].cpu().numpy(), full.argmin(1)), op
-            if op == "xor":
-                for qi, (kind, js, flips) in enumerate(plan):
-                    if kind == "copy":
-                        assert u32(best[j][0])[qi] <= len(flips)
-        _, bonly = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False)
-        for j in range(2):
-            assert torch.equal(bonly[j][0], best[j][0]) and torch.equal(bonly[j][1], best[j][1])
+        for pd in (None, popD):
+            counts, best = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), popD=pd)
+            if variant == "auto":
+                assert snp.snp_last_kernel() == "fastid_mxf4"
+            for j, op in enumerate(("xor", "andnot")):
+                got = u32(counts[j].view(torch.int32)[:, torch.from_numpy(cols).to(DEV)])
+                assert np.array_equal(got, oracle.counts(q, dbs, op)), op
+                full = counts[j].cpu().numpy().astype(np.uint32)
+                assert np.array_equal(u32(best[j][0]), full.min(1)), op
+                assert np.array_equal(best[j][1].cpu().numpy(), full.argmin(1)), op
+                if op == "xor":
+                    for qi, (kind, js, flips) in enumerate(plan):
+                        if kind == "copy":
+                            assert u32(best[j][0])[qi] <= len(flips)
+            _, bonly = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False, popD=pd)
+            for j in range(2):
+                assert torch.equal(bonly[j][0], best[j][0]) and torch.equal(bonly[j][1], best[j][1])
+            del counts
     finally:
         _variant(snp, "auto")
