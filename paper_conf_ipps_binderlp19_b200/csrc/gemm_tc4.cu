@@ -75,7 +75,7 @@ struct GArgs {
     int nst;
     int trace;
     int debug_skip;   // profiling experiment: expanders only pass tokens (results invalid)
-    int order;        // tile raster: 1 lane-block-major, 0 column-block-major
+    int order;        // tile raster: 2 grouped (default), 1 lane-block-major, 0 column-block-major
     const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
 };
 
@@ -303,11 +303,29 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     // 32-bit tile arithmetic (ntiles < 2^31): a 64-bit division is a subroutine CALL, and
     // any call in the kernel made ptxas drop the MMA issue loop out of uniform registers
     const uint32_t nlb32 = (uint32_t)args.nlb, ncb32 = (uint32_t)args.ncb;
-    // tile t -> (lane block, column block): lane-block-major (the 148 tiles in flight share
-    // one lane block and write 148 adjacent column blocks of the same output rows) or
-    // column-block-major
-    auto tile_lb = [&](uint32_t t) { return args.order ? t / ncb32 : t % nlb32; };
-    auto tile_cb = [&](uint32_t t) { return args.order ? t % ncb32 : t / nlb32; };
+    // tile t -> (lane block, column block).  order 2 (default): groups of RG lane blocks;
+    // inside a group the lane block varies fastest, so the ~148 tiles in flight cover RG
+    // lane blocks x ~148/RG column blocks: each packed column block is read from DRAM once
+    // per group and reused RG times from L2, the group's lane blocks stay L2-resident for
+    // its whole column sweep (DRAM reads ~ nlb/RG x the column operand instead of ~nlb x).
+    // order 1: lane-block-major; order 0: column-block-major.
+    constexpr uint32_t RG = 16;
+    auto tile_lb = [&](uint32_t t) -> uint32_t {
+        if (args.order == 2) {
+            const uint32_t g = t / (RG * ncb32), w = t - g * RG * ncb32;
+            const uint32_t rows = nlb32 - g * RG < RG ? nlb32 - g * RG : RG;
+            return g * RG + w % rows;
+        }
+        return args.order ? t / ncb32 : t % nlb32;
+    };
+    auto tile_cb = [&](uint32_t t) -> uint32_t {
+        if (args.order == 2) {
+            const uint32_t g = t / (RG * ncb32), w = t - g * RG * ncb32;
+            const uint32_t rows = nlb32 - g * RG < RG ? nlb32 - g * RG : RG;
+            return w / rows;
+        }
+        return args.order ? t % ncb32 : t / nlb32;
+    };
     const int64_t my_tiles =
         ntiles > blockIdx.x ? (int64_t)(((uint32_t)ntiles - 1u - blockIdx.x) / gridDim.x + 1u) : 0;
     const int64_t total_it = my_tiles * nst;
@@ -729,7 +747,7 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
     g.debug_skip = skip ? 1 : 0;
     static const char *ord = std::getenv("SNP_GEMM_ORDER");
-    g.order = ord ? (ord[0] == '1') : 1;
+    g.order = ord ? (ord[0] - '0') : 2;
     return epi == EPI_LD ? launch_g<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
 }
 
