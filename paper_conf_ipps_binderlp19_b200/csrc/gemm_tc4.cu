@@ -658,6 +658,388 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     }
 }
 
+
+// ============================================================================ CTA-pair kernel
+// gemm_tc4x2_kernel: the same bit-GEMM with tcgen05.mma.cta_group::2 on a cluster of two
+// CTAs (one TPC).  A pair tile is 256 lane rows x 128 columns: each CTA expands its own
+// 128 lane rows into its TMEM (MMA operand A from TMEM) and only 64 of the 128 column
+// rows into its shared memory (the pair's B operand is split N/2 per CTA); the leader
+// CTA's single thread issues M = 256, N = 128, K = 64 MMAs that read both CTAs' halves.
+// Per CTA and stage this halves the B-side nibble writes to shared memory (16 KB instead
+// of 32 KB) and cuts packed loads and expansion ALU work by a quarter — the shared-memory
+// pipe and the ALU were the binding resources of the 1-CTA kernel.
+// Cross-CTA protocol:
+//   full[s]   (leader)  12 arrivals: the 6 expander warps of the stage's group in BOTH CTAs,
+//                       remote arrive.release.cluster after their TMEM / shared writes;
+//   empty[s]  (both)    tcgen05.commit multicast from the leader's MMA thread;
+//   accf[a]   (both)    tcgen05.commit multicast at the end of a pair tile;
+//   acce[a]   (leader)  16 arrivals: 8 epilogue warps of each CTA after draining TMEM.
+namespace x2 {
+constexpr int BNP = 128;                       // pair tile columns
+constexpr int BNH = BNP / 2;                   // column rows per CTA
+constexpr int NS = 3;                          // TMEM A / smem B stages
+#ifndef X2_NP
+#define X2_NP 8
+#endif
+#ifndef X2_G
+#define X2_G 2
+#endif
+constexpr int NP = X2_NP;                      // packed TMA ring
+constexpr int G = X2_G;                        // expander groups
+constexpr int GW = 6;                          // warps per group: 4 A (lane quarters) + 2 B
+constexpr int NEXP = G * GW;                   // 12
+constexpr int NEPI = 8;
+constexpr int EPI_WARP0 = NEXP;                // 12..19
+constexpr int TMA_WARP = NEXP + NEPI;          // 20
+constexpr int MMA_WARP = NEXP + NEPI + 1;      // 21
+constexpr int NTHREADS = (NEXP + NEPI + 2) * 32;
+constexpr int PSLOT = (BM + BNH) * PROW;       // 12 KB packed per slot (128 A rows, 64 C rows)
+constexpr int BSLOT = BNH * KBITS / 2;         // 16 KB expanded B per slot
+constexpr int ACC_COLS = BNP;                  // 128
+constexpr int A_COL0 = 2 * ACC_COLS;           // 256
+constexpr int SF_COL = A_COL0 + NS * 64;       // 448
+static_assert(SF_COL + 32 <= 512, "TMEM budget");
+constexpr size_t SMEM = (size_t)NP * PSLOT + (size_t)NS * BSLOT + (size_t)NEPI * TRW + 1024;
+static_assert(SMEM <= 232448, "227 KB opt-in shared memory");
+
+__device__ __forceinline__ uint32_t cta_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_id() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t num_clusters() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%nclusterid.x;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// arrive on the barrier at the same shared-memory offset in CTA `rank` of the cluster
+__device__ __forceinline__ void arrive_remote(uint64_t *bar, uint32_t rank) {
+    uint32_t ra;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(ptx::smem_u32(bar)), "r"(rank));
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
+}
+__device__ __forceinline__ bool try_wait_cluster(uint64_t *bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(ptx::smem_u32(bar)), "r"(parity), "r"(100000u)
+        : "memory");
+    return ok != 0;
+}
+// warp-uniform wait with cluster-scope acquire (the arrivals come from both CTAs)
+__device__ __forceinline__ bool try_wait_cluster_now(uint64_t *bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(ptx::smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void wait_cluster_uniform(uint64_t *bar, uint32_t parity) {
+    if (__all_sync(0xffffffffu, try_wait_cluster_now(bar, parity))) return;
+    const uint64_t t0 = ptx::globaltimer_ns();
+    while (!__all_sync(0xffffffffu, try_wait_cluster(bar, parity))) {
+        if (__any_sync(0xffffffffu, ptx::globaltimer_ns() - t0 > 4000000000ull)) __trap();
+    }
+}
+__device__ __forceinline__ void mma_mxf4_ts2(uint32_t d, uint32_t a, uint64_t b, uint32_t idesc, uint32_t accumulate,
+                                             uint32_t sfa, uint32_t sfb) {
+    asm volatile(
+        "{\n\t.reg .pred e, p;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "@e tcgen05.mma.cta_group::2.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}" ::"r"(d),
+        "r"(a), "l"(b), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb)
+        : "memory");
+}
+// commit the leader's outstanding MMAs to the barrier at this offset in BOTH CTAs
+__device__ __forceinline__ void commit_both(uint64_t *bar) {
+    asm volatile(
+        "{\n\t.reg .pred e;\n\t.reg .b16 m;\n\tmov.b16 m, 3;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], m;\n\t}" ::"r"(
+            ptx::smem_u32(bar))
+        : "memory");
+}
+}  // namespace x2
+
+template <int EPI>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(x2::NTHREADS, 1)
+gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
+                  const GArgs args) {
+    constexpr int NS = x2::NS, NP = x2::NP, G = x2::G, GW = x2::GW, NEXP = x2::NEXP, NEPI = x2::NEPI;
+    constexpr int EPI_WARP0 = x2::EPI_WARP0, TMA_WARP = x2::TMA_WARP, MMA_WARP = x2::MMA_WARP;
+    constexpr int PSLOT = x2::PSLOT, BSLOT = x2::BSLOT, ACC_COLS = x2::ACC_COLS, A_COL0 = x2::A_COL0;
+    constexpr int SF_COL = x2::SF_COL, BNP = x2::BNP, BNH = x2::BNH;
+    using x2::cta_rank; using x2::cluster_id; using x2::num_clusters; using x2::cluster_sync;
+    using x2::arrive_remote; using x2::wait_cluster_uniform; using x2::mma_mxf4_ts2; using x2::commit_both;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *ring = smem;                                        // [NP][PSLOT]
+    uint8_t *bexp = smem + (size_t)NP * PSLOT;                   // [NS][BSLOT]
+    uint32_t *trs = reinterpret_cast<uint32_t *>(bexp + (size_t)NS * BSLOT);   // [NEPI][32][32]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(trs + NEPI * 32 * 32);
+    uint64_t *pfull = bars;            // [NP] TMA -> expanders (local)
+    uint64_t *pempty = pfull + NP;     // [NP] expanders -> TMA (local)
+    uint64_t *full = pempty + NP;      // [NS] expanders of both CTAs -> leader MMA
+    uint64_t *empty = full + NS;       // [NS] MMA -> expanders (multicast commit)
+    uint64_t *accf = empty + NS;       // [2]  MMA -> epilogues (multicast commit)
+    uint64_t *acce = accf + 2;         // [2]  epilogues of both CTAs -> leader MMA
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acce + 2);
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const uint32_t rank = cta_rank();
+    const bool leader = rank == 0;
+    const int64_t nbits = args.nbits;
+    const int nst = args.nst;
+    // pair tiles: nlb = lane blocks of 256 rows, ncb = column blocks of 128
+    const uint32_t nlb32 = (uint32_t)args.nlb, ncb32 = (uint32_t)args.ncb;
+    const uint32_t ntiles = nlb32 * ncb32;
+    const uint32_t cid = cluster_id(), ncl = num_clusters();
+    const int64_t my_tiles = ntiles > cid ? (int64_t)((ntiles - 1u - cid) / ncl + 1u) : 0;
+    const int64_t total_it = my_tiles * nst;
+    const int64_t full32 = nbits / 32;
+    constexpr uint32_t RG = 8;   // grouped raster (see gemm_tc4_kernel), lane block fastest
+    auto tile_lb = [&](uint32_t t) -> uint32_t {
+        const uint32_t g = t / (RG * ncb32), w = t - g * RG * ncb32;
+        const uint32_t rows = nlb32 - g * RG < RG ? nlb32 - g * RG : RG;
+        return g * RG + w % rows;
+    };
+    auto tile_cb = [&](uint32_t t) -> uint32_t {
+        const uint32_t g = t / (RG * ncb32), w = t - g * RG * ncb32;
+        const uint32_t rows = nlb32 - g * RG < RG ? nlb32 - g * RG : RG;
+        return w / rows;
+    };
+
+    if (tid == 0) {
+        for (int i = 0; i < NP; ++i) {
+            ptx::mbar_init(&pfull[i], 1);
+            ptx::mbar_init(&pempty[i], GW);
+        }
+        for (int i = 0; i < NS; ++i) {
+            ptx::mbar_init(&full[i], 2 * GW);
+            ptx::mbar_init(&empty[i], 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            ptx::mbar_init(&accf[i], 1);
+            ptx::mbar_init(&acce[i], 2 * NEPI);
+        }
+        ptx::fence_mbar_init();
+    }
+    if (warp == TMA_WARP && lane == 0) {
+        ptx::prefetch_tensormap(&tmL);
+        ptx::prefetch_tensormap(&tmC);
+    }
+    if (warp == MMA_WARP) {   // both CTAs, same warp id: one 2-SM allocation
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(ptx::smem_u32(tmem_slot))
+                     : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    }
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+    if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {
+        const int q = warp & 3;
+        uint32_t v[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = 0x7F7F7F7Fu;   // ue8m0 2^0 in every scale byte
+        tmem_st32(tmem + ((uint32_t)(q * 32) << 16) + SF_COL, v);
+        ptx::tmem_st_wait();
+    }
+    ptx::tc_fence_before();
+    cluster_sync();   // barriers initialised and TMEM allocated in both CTAs
+    ptx::tc_fence_after();
+
+    if (warp == TMA_WARP) {
+        // ------------------------------------------------------------ TMA producer (each CTA)
+        if (lane == 0) {
+            int p = 0;
+            uint32_t round = 0;
+            for (int64_t tl = 0; tl < my_tiles; ++tl) {
+                const uint32_t t32 = cid + (uint32_t)tl * ncl;
+                const int32_t rl = (int32_t)(tile_lb(t32) * (2 * BM) + rank * BM);
+                const int32_t rc = (int32_t)(tile_cb(t32) * BNP + rank * BNH);
+                for (int s = 0; s < nst; ++s) {
+                    if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);
+                    ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
+                    ptx::tma_load_2d(ring + p * PSLOT, &tmL, &pfull[p], s * KW, rl);
+                    ptx::tma_load_2d(ring + p * PSLOT + BM * PROW, &tmC, &pfull[p], s * KW, rc);
+                    if (++p == NP) { p = 0; ++round; }
+                }
+            }
+        }
+    } else if (warp < NEXP) {
+        // ------------------------------------------------------------ expanders (each CTA)
+        // group g = warp / 6: warps 0-3 expand the 128 lane rows (lane quarter q) into TMEM,
+        // warps 4-5 the 64 column rows (32 each) into the stage's shared-memory B operand.
+        // A warps take the TMEM lane quarter warp % 4 (a warp may only access that quarter:
+        // the 4 A warps of a group are 4 consecutive warp ids, so they cover all four)
+        const int g = warp / GW, r6 = warp - g * GW;
+        const bool is_a = r6 < 4;
+        const int row = is_a ? (warp & 3) * 32 + lane : (r6 - 4) * 32 + lane;
+        const int sw = (row >> 1) & 3;                  // TMA 64B swizzle of a 64-byte row
+        const uint32_t tAq = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)A_COL0;
+        int s = g % nst;
+        int slot = g % NS;
+        uint32_t use = (uint32_t)(g / NS);
+        static_assert(NP % G == 0, "each packed slot belongs to one expander group");
+        int pk = g;
+        uint32_t pround = 0;
+        for (int64_t it = g; it < total_it; it += G) {
+            if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
+            ptx::mbar_wait_warp(&pfull[pk], pround & 1);
+            if (args.debug_skip) {   // profiling experiment: tokens only (results invalid)
+                __syncwarp();
+                if (lane == 0) { ptx::mbar_arrive(&pempty[pk]); arrive_remote(&full[slot], 0); }
+                s += G;
+                while (s >= nst) s -= nst;
+                slot += G;
+                if (slot >= NS) { slot -= NS; ++use; }
+                pk += G;
+                if (pk >= NP) { pk -= NP; ++pround; }
+                continue;
+            }
+            const uint8_t *src = ring + pk * PSLOT + (is_a ? 0 : BM * PROW) + row * PROW;
+            uint32_t w[KW];
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const uint4 x = *reinterpret_cast<const uint4 *>(src + ((c ^ sw) << 4));
+                w[4 * c] = x.x; w[4 * c + 1] = x.y; w[4 * c + 2] = x.z; w[4 * c + 3] = x.w;
+            }
+            const int64_t w0 = (int64_t)s * KW;
+            if (w0 + KW > full32) {
+#pragma unroll
+                for (int i = 0; i < KW; ++i) w[i] &= word_mask(w0 + i, nbits);
+            }
+            if (is_a) {
+                const uint32_t tA = tAq + 64 * slot;
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    uint32_t v[32];
+#pragma unroll
+                    for (int i = 0; i < 8; ++i)
+                        expandA(w[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+                    tmem_st32(tA + 32 * h, v);
+                }
+                ptx::tmem_st_wait();
+                ptx::tc_fence_before();
+            } else {
+                uint8_t *dstB = bexp + (size_t)slot * BSLOT + row * 16;
+#pragma unroll
+                for (int i = 0; i < KW; ++i) {          // chunk i of the K-major operand = word i
+                    uint4 o;
+                    expandB(w[i], o.x, o.y, o.z, o.w);
+                    *reinterpret_cast<uint4 *>(dstB + (size_t)i * BNH * 16) = o;
+                }
+                ptx::fence_proxy_async_smem();
+            }
+            __syncwarp();
+            if (lane == 0) {
+                ptx::mbar_arrive(&pempty[pk]);
+                arrive_remote(&full[slot], 0);   // the leader's MMA waits for both CTAs
+            }
+            s += G;
+            while (s >= nst) s -= nst;
+            slot += G;
+            if (slot >= NS) { slot -= NS; ++use; }
+            pk += G;
+            if (pk >= NP) { pk -= NP; ++pround; }
+        }
+    } else if (warp == MMA_WARP) {
+        // ------------------------------------------------------------ MMA issuer (leader only)
+        if (leader) {
+            constexpr uint32_t IDESC = idesc_mxf4(2 * BM, BNP);
+            const uint32_t tmu = __reduce_or_sync(0xffffffffu, tmem);
+            const uint32_t sfa = tmu + SF_COL, sfb = tmu + SF_COL + 16;
+            const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(bexp), BNH * 16, 128);
+            constexpr uint32_t BSTEP = (2 * BNH * 16) >> 4;
+            int b = 0;
+            uint32_t round = 0;
+            for (int64_t tl = 0; tl < my_tiles; ++tl) {
+                const int acc = (int)(tl & 1);
+                if (tl >= 2) wait_cluster_uniform(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+                ptx::tc_fence_after();
+                const uint32_t d = tmu + (uint32_t)(acc * ACC_COLS);
+                for (int s = 0; s < nst; ++s) {
+                    wait_cluster_uniform(&full[b], round & 1);
+                    ptx::tc_fence_after();
+                    const uint32_t a0 = tmu + (uint32_t)(A_COL0 + 64 * b);
+                    const uint64_t b0 = bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4);
+#pragma unroll
+                    for (int k = 0; k < KBITS / 64; ++k)
+                        mma_mxf4_ts2(d, a0 + 8 * k, b0 + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                    commit_both(&empty[b]);
+                    if (++b == NS) { b = 0; ++round; }
+                }
+                commit_both(&accf[acc]);
+            }
+        }
+        __syncwarp();
+    } else {
+        // ------------------------------------------------------------ epilogue (each CTA)
+        // warp e: TMEM lane quarter e % 4 of this CTA's 128 lane rows, columns [64 h, 64 h + 64)
+        const int e = warp - EPI_WARP0;
+        const int q = e & 3, h = e >> 2;
+        const int li = q * 32 + lane;
+        const int c0 = 64 * h;
+        const int64_t n = nbits;
+        const bool small_n = n <= 46340;
+        const bool need_pop = EPI == EPI_LD || args.op != 0;
+        const bool want_dp = EPI == EPI_LD && args.dprime != nullptr;
+        for (int64_t tl = 0; tl < my_tiles; ++tl) {
+            const int acc = (int)(tl & 1);
+            const uint32_t ph = (uint32_t)((tl >> 1) & 1);
+            const uint32_t t32 = cid + (uint32_t)tl * ncl;
+            const int64_t gl = (int64_t)tile_lb(t32) * (2 * BM) + rank * BM + li;
+            const int64_t gc0 = (int64_t)tile_cb(t32) * BNP + c0;
+            const int ncols = gc0 < args.nc ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
+            uint32_t pl = 0, pcol0 = 0, pcol1 = 0;
+            if (need_pop) {
+                if (gl < args.nl) pl = __ldg(args.popL + gl);
+                if (lane < ncols) pcol0 = __ldg(args.popC + gc0 + lane);
+                if (32 + lane < ncols) pcol1 = __ldg(args.popC + gc0 + 32 + lane);
+            }
+            ptx::mbar_wait_warp(&accf[acc], ph);
+            ptx::tc_fence_after();
+            const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * ACC_COLS + c0);
+            const float ia = EPI == EPI_LD ? inv_exact((int64_t)pl * (n - (int64_t)pl)) : 0.f;
+#pragma unroll 1
+            for (int hh = 0; hh < 2; ++hh) {
+                uint32_t v[32];
+                __syncwarp();
+                tmem_ld32(ta + 32 * hh, v);
+                ptx::tmem_ld_wait();
+                if (hh == 1) {
+                    ptx::tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) arrive_remote(&acce[acc], 0);   // drained: the leader may reuse it
+                }
+                epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, gl - lane, gc0 + 32 * hh, pl,
+                                    hh ? pcol1 : pcol0, ia, small_n, want_dp);
+            }
+        }
+    }
+
+    ptx::tc_fence_before();
+    __syncthreads();
+    cluster_sync();   // no CTA leaves (or frees TMEM) while its peer may still signal it
+    if (warp == MMA_WARP) {
+        ptx::tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, 512;" ::"r"(tmem) : "memory");
+    }
+}
+
 typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -674,12 +1056,12 @@ EncodeTiledFn encode_fn() {
     return fn;
 }
 
-bool make_map(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32) {
+bool make_map(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32, uint32_t box_rows = 128) {
     EncodeTiledFn enc = encode_fn();
     if (!enc) return false;
     const cuuint64_t dims[2] = {(cuuint64_t)ld32, (cuuint64_t)rows};
     const cuuint64_t strides[1] = {(cuuint64_t)ld32 * 4};
-    const cuuint32_t box[2] = {KW, 128};
+    const cuuint32_t box[2] = {KW, box_rows};
     const cuuint32_t estr[2] = {1, 1};
     return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(base), dims, strides, box, estr,
                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -716,6 +1098,28 @@ cudaError_t launch_g(const GArgs &g, const uint32_t *L, int64_t ldl32, const uin
     return cudaGetLastError();
 }
 
+template <int EPI>
+cudaError_t launch_g2(GArgs g, const uint32_t *L, int64_t ldl32, const uint32_t *Cn, int64_t ldc32, cudaStream_t s) {
+    CUtensorMap tmL, tmC;
+    if (!make_map(&tmL, L, g.nl, ldl32, 128) || !make_map(&tmC, Cn, g.nc, ldc32, x2::BNH))
+        return cudaErrorInvalidValue;
+    auto kern = gemm_tc4x2_kernel<EPI>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)x2::SMEM);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    g.nlb = (g.nl + 2 * BM - 1) / (2 * BM);
+    g.ncb = (g.nc + x2::BNP - 1) / x2::BNP;
+    const int64_t npairs = g.nlb * g.ncb;
+    const int pairs = num_sms() / 2;
+    const int grid = 2 * (int)(npairs < pairs ? npairs : pairs);
+    kern<<<grid, x2::NTHREADS, x2::SMEM, s>>>(tmL, tmC, g);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
 }  // namespace
 
 bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
@@ -748,6 +1152,14 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.debug_skip = skip ? 1 : 0;
     static const char *ord = std::getenv("SNP_GEMM_ORDER");
     g.order = ord ? (ord[0] - '0') : 2;
+    // CTA-pair kernel: opt-in (SNP_GEMM_X2=1) for the unswapped shapes with more than one
+    // lane block.  Measured slower on B200 (LD-32K counts 9.1 ms vs 7.0 ms; with expansion
+    // skipped 7.8 vs 4.7 ms: the M = 256, N = 128 pair MMAs run at about half the per-SM
+    // rate of the 1-CTA M = N = 128 ones here), so the 1-CTA kernel is the default.
+    static const char *x2e = std::getenv("SNP_GEMM_X2");
+    const bool use_x2 = !swap && g.nl > BM && x2e && x2e[0] == '1';
+    if (use_x2)
+        return epi == EPI_LD ? launch_g2<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g2<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
     return epi == EPI_LD ? launch_g<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
 }
 

@@ -5,6 +5,8 @@ and exactly 0 where the oracle is 0 (BASELINE.json north_star).  Inputs come fro
 snpgen (seeded); the oracle always sees the generator's unpacked bytes, never
 anything the CUDA path produced.
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -463,3 +465,33 @@ def test_cfg2_search_1m(snp, variant):
             del counts
     finally:
         _variant(snp, "auto")
+
+
+def test_ld_cta_pair_kernel_subprocess():
+    """The opt-in CTA-pair LD kernel (SNP_GEMM_X2=1, read once per process) on ragged
+    shapes spanning several pair tiles and K stages, counts + r2 + D' vs the oracle."""
+    import subprocess
+    import sys
+    code = r'''
+import numpy as np, torch, sys
+sys.path.insert(0, ".")
+import oracle, snpgen
+import paper_conf_ipps_binderlp19_b200 as snp
+torch.cuda.set_device(0)
+for (m, n, nbits) in [(512, 256, 1024), (700, 300, 1500), (2048, 2048, 4096)]:
+    ga = snpgen.ld_genotypes(51, np.arange(m), nbits, structure=True)
+    gb = snpgen.ld_genotypes(52, np.arange(n), nbits, structure=True)
+    A = snp.snp_pack(torch.from_numpy(ga).cuda()); B = snp.snp_pack(torch.from_numpy(gb).cuda())
+    r2, dp, cnt = snp.snp_ld_r2(A, B, nbits, dprime=True, counts=True)
+    r2_ref, dp_ref, n_ref = oracle.ld(ga, gb)
+    assert np.array_equal(cnt.cpu().numpy().view(np.uint32), n_ref), (m, n, nbits)
+    for got, ref in ((r2, r2_ref), (dp, dp_ref)):
+        g = got.cpu().numpy().astype(np.float64); z = ref == 0
+        assert (g[z] == 0).all() and (np.abs(g[~z] - ref[~z]) <= 1e-6 * np.abs(ref[~z])).all()
+print("ok")
+'''
+    env = dict(os.environ, SNP_GEMM_X2="1")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
