@@ -265,6 +265,10 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     __syncthreads();
     ptx::tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    // launched with programmatic stream serialization: everything above overlapped the
+    // previous kernel in the stream (the key-init kernel); its results (and the packed
+    // queries from before it) are visible after this wait
+    asm volatile("griddepcontrol.wait;" ::: "memory");
 
     // ---- prologue: expand the whole query batch once (resident MMA B operand).  Warp w
     // takes words w, w + 26, ...; lane = query row (BN / 32 rows per lane), so the 16-byte
@@ -614,6 +618,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 }
 
 __global__ void fastid_search_init(unsigned long long *keys, int64_t n, unsigned int *done) {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");   // let the search kernel start
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         keys[i] = ~0ULL;
     if (blockIdx.x == 0 && threadIdx.x == 0) *done = 0u;
@@ -754,8 +759,22 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }
-    kern<<<grid, nthreads, smem, s>>>(tm, f);
+    // programmatic dependent launch: the kernel's setup (barriers, TMEM allocation, tensor
+    // map prefetch) overlaps the preceding kernel; it waits (griddepcontrol.wait) before
+    // touching any data that kernel produces
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3((unsigned)nthreads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t le = cudaLaunchKernelEx(&cfg, kern, tm, f);
     count_launches(1);
+    if (le != cudaSuccess) return le;
     return cudaGetLastError();
 }
 

@@ -135,8 +135,13 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
                     a.popA = pa;
                 }
                 if (!a.popB) {
-                    if ((e = launch_row_popc(B64, a.n, a.nbits, a.ldb32 / 2, pb, s)) != cudaSuccess) return set_cuda_error(e);
-                    a.popB = pb;
+                    if (a.B == a.A && a.n == a.m && a.ldb32 == a.lda32) {
+                        a.popB = a.popA;   // self-LD (B aliases A): one popcount pass
+                    } else {
+                        if ((e = launch_row_popc(B64, a.n, a.nbits, a.ldb32 / 2, pb, s)) != cudaSuccess)
+                            return set_cuda_error(e);
+                        a.popB = pb;
+                    }
                 }
             }
             e = launch_gemm_tc4(a, epi, s);
