@@ -52,6 +52,9 @@ constexpr int PSTAGE = BM * KBITS / 8;  // 8 KB packed per stage, 64-byte rows, 
 #ifndef FASTID_G
 #define FASTID_G 4
 #endif
+#ifndef FASTID_NEPI2
+#define FASTID_NEPI2 8   // epilogue warps of the GG = 2 kernels
+#endif
 #ifndef FASTID_NEPI
 #define FASTID_NEPI 8
 #endif
@@ -61,9 +64,10 @@ constexpr int PSTAGE = BM * KBITS / 8;  // 8 KB packed per stage, 64-byte rows, 
 // 203 vs 220 us on FastID-1M).
 // The warp scheduler favours higher warp ids, so the latency-critical single-thread
 // roles get the highest ids: MMA issuer last, TMA producer next, epilogue below them.
-constexpr int NEPI = FASTID_NEPI;       // epilogue warps: lane quarter w % 4, column block w / 4
+// epilogue warps: lane quarter w % 4, column block w / 4 (Roles<GG>::NEPI)
 template <int GG>
 struct Roles {
+    static constexpr int NEPI = GG == 2 ? FASTID_NEPI2 : FASTID_NEPI;
     static constexpr int G = GG;
     static constexpr int NEXP = 4 * GG;
     static constexpr int EPI_WARP0 = NEXP;
@@ -210,7 +214,7 @@ __global__ void __launch_bounds__(Roles<GG>::NTHREADS, 1)
 fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     constexpr int G = GG, NEXP = Roles<GG>::NEXP, EPI_WARP0 = Roles<GG>::EPI_WARP0;
     constexpr int TMA_WARP = Roles<GG>::TMA_WARP, MMA_WARP = Roles<GG>::MMA_WARP;
-    constexpr int NTHREADS = Roles<GG>::NTHREADS;
+    constexpr int NTHREADS = Roles<GG>::NTHREADS, NEPI = Roles<GG>::NEPI;
     using C = FCfg<BN>;
     constexpr int NS = C::NS;
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -554,10 +558,10 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                     }
                     if (sv[j] && colok) {
                         const uint32_t x = key >> 5;   // valid rows: laneterm = lane < 32
-                        uint32_t *o = op_[j] + (int64_t)u * ldo;
-                        if (ACC) *o += x;
-                        else __stcs(o, x);   // streaming store: written once, never re-read here
+                        if (ACC) *op_[j] += x;
+                        else __stcs(op_[j], x);   // streaming store: written once, never re-read here
                     }
+                    op_[j] += ldo;   // running pointer: one 64-bit add per store, not a product
                     if (BEST) {
                         const uint32_t m = __reduce_min_sync(0xffffffffu, key);
                         mk[j] = lane == u ? m : mk[j];
