@@ -76,6 +76,7 @@ struct GArgs {
     int trace;
     int debug_skip;   // profiling experiment: expanders only pass tokens (results invalid)
     int order;        // tile raster: 2 grouped (default), 1 lane-block-major, 0 column-block-major
+    int off32;        // every output element offset (row * ldo + col) fits in 32 bits
     const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
 };
 
@@ -228,6 +229,44 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
         return;
     }
     float *rp = args.r2 + o0;
+    if (small_n && !want_dp && rows == 32 && args.off32) {
+        // the benchmarked LD path, full 32-row block: fully unrolled, 32-bit element
+        // offsets (off32: every output offset < 2^32), the 8 swizzled LDS column offsets
+        // precomputed; per element 2 SHFL (row terms), LDS, 2 IMAD, I2F, 3 FMUL, FMNMX,
+        // 1 address IMAD per output array and 1-2 STG
+        const float ib = inv_exact((int64_t)pb * (n - (int64_t)pb));
+        const int32_t npb = -pb;
+        const bool has_c = args.C != nullptr;
+        uint32_t cofs[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) cofs[k] = (uint32_t)(((((lane >> 2) ^ k)) << 2) + (lane & 3));
+        uint32_t off = (uint32_t)o0;
+        const uint32_t ld32 = (uint32_t)ldo;
+        float *const r2b = args.r2;
+        uint32_t *const cb = args.C;
+        const uint32_t okr = colok ? 1u : 0u, okc = (colok && has_c) ? 1u : 0u;
+#pragma unroll
+        for (int r = 0; r < 32; ++r) {
+            const int32_t plr = (int32_t)__shfl_sync(0xffffffffu, pl, r);
+            const float iar = __shfl_sync(0xffffffffu, ia, r);
+            const int32_t c = (int32_t)tw[r * 32 + cofs[r & 7]];
+            const int32_t num = n32 * c + plr * npb;
+            const float fn = (float)num;
+            const float r2v = fminf(__fmul_rn(__fmul_rn(fn, iar), __fmul_rn(fn, ib)), 1.0f);
+            // predicated evict-first stores (outputs are written once; the packed operands
+            // stay in L2): no branch, so the shuffles stay in a converged straight line
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(
+                             r2b + off),
+                         "f"(r2v), "r"(okr)
+                         : "memory");
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(
+                             cb + off),
+                         "r"(c), "r"(okc)
+                         : "memory");
+            off += ld32;
+        }
+        return;
+    }
     if (small_n && !want_dp) {
         // the benchmarked LD path: per element 2 IMAD, I2F, 3 FMUL, FMNMX, 1-2 STG
         const float ib = inv_exact((int64_t)pb * (n - (int64_t)pb));
@@ -1150,6 +1189,7 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.trace = trace ? 1 : 0;
     static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
     g.debug_skip = skip ? 1 : 0;
+    g.off32 = (uint64_t)(swap ? a.n : a.m) * (uint64_t)a.ldc < (1ull << 32) ? 1 : 0;
     static const char *ord = std::getenv("SNP_GEMM_ORDER");
     g.order = ord ? (ord[0] - '0') : 2;
     // CTA-pair kernel: opt-in (SNP_GEMM_X2=1) for the unswapped shapes with more than one
