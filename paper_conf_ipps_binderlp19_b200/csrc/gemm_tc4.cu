@@ -77,6 +77,8 @@ struct GArgs {
     int debug_skip;   // profiling experiment: expanders only pass tokens (results invalid)
     int order;        // tile raster: 2 grouped (default), 1 lane-block-major, 0 column-block-major
     int off32;        // every output element offset (row * ldo + col) fits in 32 bits
+    int op2;          // EPI_COUNTS, swapped layout: second op written to C2 (or C2 = NULL)
+    uint32_t *C2;
     const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
 };
 
@@ -553,7 +555,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         const int64_t ldo = args.ldo;
         const int64_t n = nbits;
         const bool small_n = n <= 46340;                 // n^2 < 2^31: exact int32 LD arithmetic
-        const bool need_pop = EPI == EPI_LD || args.op != 0;
+        const bool need_pop = EPI == EPI_LD || args.op != 0 || (args.C2 && args.op2 != 0);
         const bool want_dp = EPI == EPI_LD && args.dprime != nullptr;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
@@ -611,31 +613,25 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                         pc[k] = __shfl_sync(0xffffffffu, pcol, uu + k);
                     }
                     if (EPI == EPI_COUNTS) {
-                        uint32_t r[4];
-#pragma unroll
-                        for (int k = 0; k < 4; ++k) {
-                            const uint32_t pq = args.swap ? pc[k] : pl, pd = args.swap ? pl : pc[k];
-                            const int op = args.op;
-                            r[k] = op == 0 ? c[k] : op == 1 ? pq + pd - 2u * c[k] : op == 2 ? pq - c[k] : pd - c[k];
-                        }
+                        // swapped layout (lane = output column): per output column k the 32
+                        // lanes store 32 consecutive words.  Up to two ops from the one AND
+                        // count (f1: XOR + ANDNOT in one pass over the database).
                         if (!rows_ok) continue;
-                        if (full_vec) {
-                            uint32_t *o = args.C + gl * ldo + gc0 + u0;
-                            if (((uintptr_t)o & 15u) == 0) {
-                                uint4 rr = make_uint4(r[0], r[1], r[2], r[3]);
-                                if (args.accumulate) {
-                                    const uint4 pv = *reinterpret_cast<const uint4 *>(o);
-                                    rr.x += pv.x; rr.y += pv.y; rr.z += pv.z; rr.w += pv.w;
-                                }
-                                *reinterpret_cast<uint4 *>(o) = rr;
-                                continue;
-                            }
-                        }
 #pragma unroll
-                        for (int k = 0; k < 4; ++k) {
-                            if (u0 + k >= ncols) break;
-                            uint32_t *o = args.swap ? args.C + (gc0 + u0 + k) * ldo + gl : args.C + gl * ldo + gc0 + u0 + k;
-                            *o = args.accumulate ? *o + r[k] : r[k];
+                        for (int jj = 0; jj < 2; ++jj) {
+                            uint32_t *const Cb = jj ? args.C2 : args.C;
+                            if (jj && !Cb) break;
+                            const int op = jj ? args.op2 : args.op;
+#pragma unroll
+                            for (int k = 0; k < 4; ++k) {
+                                if (u0 + k >= ncols) break;
+                                const uint32_t pq = pc[k], pd = pl;
+                                const uint32_t r = op == 0 ? c[k] : op == 1 ? pq + pd - 2u * c[k]
+                                                 : op == 2 ? pq - c[k] : pd - c[k];
+                                uint32_t *o = Cb + (gc0 + u0 + k) * ldo + gl;
+                                if (args.accumulate) *o += r;
+                                else __stcs(o, r);
+                            }
                         }
                     } else {
                         float r2v[4], dpv[4] = {0.f, 0.f, 0.f, 0.f};
@@ -1034,7 +1030,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
         const int c0 = 64 * h;
         const int64_t n = nbits;
         const bool small_n = n <= 46340;
-        const bool need_pop = EPI == EPI_LD || args.op != 0;
+        const bool need_pop = EPI == EPI_LD || args.op != 0 || (args.C2 && args.op2 != 0);
         const bool want_dp = EPI == EPI_LD && args.dprime != nullptr;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
@@ -1177,6 +1173,9 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.nbits = a.nbits;
     g.swap = swap ? 1 : 0;
     g.op = a.op;
+    g.op2 = a.op2;
+    g.C2 = a.C2;
+    if (g.C2 && !swap) return cudaErrorInvalidValue;   // two-op epilogue: swapped layout only
     g.accumulate = a.accumulate;
     g.ldo = a.ldc;
     g.C = a.C;

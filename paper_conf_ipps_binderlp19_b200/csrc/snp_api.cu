@@ -123,7 +123,7 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
         if (kern == SNP_KERNEL_FASTID_MXF4) {
             e = launch_fastid_tc4(a, epi, s);   // derives popcounts from the streamed words
         } else if (kern == SNP_KERNEL_TC_MXF4) {
-            if (epi == EPI_LD || a.op != SNP_OP_AND) {
+            if (epi == EPI_LD || a.op != SNP_OP_AND || (a.C2 && a.op2 != SNP_OP_AND)) {
                 // the general kernel reads row popcounts: cheap pre-pass if not given
                 if (ws_bytes < pops_bytes(a.m, a.n) || !ws) return SNP_E_WORKSPACE;
                 uint32_t *pa = reinterpret_cast<uint32_t *>(ws);
@@ -444,11 +444,35 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
     if (nd > 0) p += align256((size_t)nq * ch * 4);
     void *gws = p;
     const size_t gws_bytes = ws_bytes - (size_t)(p - (char *)ws);
+    const int variant = choose_variant(nq, nd, nbits);
+    // two ops whose counts are both stored come from ONE pass of the general tensor kernel
+    // (swapped layout: database rows on TMEM lanes), which writes both identities of the
+    // same AND count; the CUDA-core variant computes each op directly
+    const bool pairable = variant == SNP_VARIANT_TC && nd > nq &&
+                          tc_kernel_for(nq, nd, nbits, EPI_COUNTS) == SNP_KERNEL_TC_MXF4;
     for (int j = 0; j < nops; ++j) {
         const bool best = a.best_count[j] != nullptr;
         unsigned long long *kj = keys + (int64_t)j * nq;
         if (best && (e = launch_best_init(kj, nq, s)) != cudaSuccess) return set_cuda_error(e);
-        const int variant = choose_variant(nq, nd, nbits);
+        if (pairable && j + 1 < nops && a.counts[j] && a.counts[j + 1] && nd > 0) {
+            GemmArgs g{};
+            g.A = a.Q; g.B = a.D; g.m = nq; g.n = nd; g.lda32 = a.ldq32; g.ldb32 = a.ldd32;
+            g.nbits = nbits; g.op = ops[j]; g.ldc = ldo; g.C = a.counts[j]; g.popB = popD;
+            g.op2 = ops[j + 1]; g.C2 = a.counts[j + 1];
+            if ((st = run_gemm(g, EPI_COUNTS, variant, gws, gws_bytes, s)) != SNP_OK) return st;
+            for (int jj = j; jj <= j + 1; ++jj) {
+                if (!a.best_count[jj]) continue;
+                unsigned long long *kk = keys + (int64_t)jj * nq;
+                if (jj != j && (e = launch_best_init(kk, nq, s)) != cudaSuccess) return set_cuda_error(e);
+                if ((e = launch_best_reduce(a.counts[jj], nq, nd, ldo, 0, kk, s)) != cudaSuccess)
+                    return set_cuda_error(e);
+                if ((e = launch_best_finalize(kk, nq, index_base, a.best_count[jj], a.best_index[jj], s)) !=
+                    cudaSuccess)
+                    return set_cuda_error(e);
+            }
+            ++j;
+            continue;
+        }
         if (a.counts[j] && nd > 0) {
             GemmArgs g{};
             g.A = a.Q; g.B = a.D; g.m = nq; g.n = nd; g.lda32 = a.ldq32; g.ldb32 = a.ldd32;

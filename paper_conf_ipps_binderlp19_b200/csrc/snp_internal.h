@@ -29,6 +29,8 @@ struct GemmArgs {
     float *dprime;       // EPI_LD optional
     const uint32_t *popA;  // EPI_LD (and tensor identities)
     const uint32_t *popB;
+    int op2 = 0;           // gemm_tc4, swapped layout (m < n) only: a second op from the same
+    uint32_t *C2 = nullptr;  // AND count, written to C2 (NULL: one op)
 };
 
 // CUDA-core LOP3 + POPC variant (bitgemm_popc.cu).
