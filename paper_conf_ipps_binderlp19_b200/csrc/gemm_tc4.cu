@@ -320,6 +320,48 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
     }
 }
 
+
+// Counts epilogue of the swapped layout (lane = output column j = database row, the 32
+// accumulator columns u = output rows i = queries): for each u the 32 lanes store 32
+// consecutive words.  Each op is x = cq pQ + cd pD + cc c, two IMADs;
+// running output pointers; up to two ops (C, C2) from the same count.
+__device__ __forceinline__ void op_coef(int op, uint32_t &cq, uint32_t &cd, uint32_t &cc) {
+    cq = (op == 1 || op == 2) ? 1u : 0u;
+    cd = (op == 1 || op == 3) ? 1u : 0u;
+    cc = op == 0 ? 1u : op == 1 ? (uint32_t)-2 : (uint32_t)-1;
+}
+__device__ __forceinline__ void epi_swapped_counts(const GArgs &args, uint32_t (&v)[32], int lane, int64_t gl,
+                                                   int64_t col0, int ncols, uint32_t pl, uint32_t pcol) {
+    const bool small = args.nbits < (1LL << 23);
+    const bool rowok = gl < args.nl;
+    const int64_t ldo = args.ldo;
+    const bool two = args.C2 != nullptr;
+    const bool acc = args.accumulate != 0;
+    uint32_t cq1, cd1, cc1, cq2, cd2, cc2;
+    op_coef(args.op, cq1, cd1, cc1);
+    op_coef(two ? args.op2 : 0, cq2, cd2, cc2);
+    const uint32_t b1 = cd1 * pl, b2 = cd2 * pl;   // database-row terms (this lane)
+    uint32_t *o1 = args.C + col0 * ldo + gl;
+    uint32_t *o2 = two ? args.C2 + col0 * ldo + gl : nullptr;
+#pragma unroll
+    for (int u = 0; u < 32; ++u) {
+        const uint32_t pq = __shfl_sync(0xffffffffu, pcol, u);   // query popcount of column u
+        const uint32_t c = acc_count(v[u], small);
+        const bool ok = rowok && u < ncols;
+        const uint32_t x1 = cc1 * c + (cq1 * pq + b1);
+        if (ok) {
+            if (acc) *o1 += x1;
+            else __stcs(o1, x1);
+        }
+        o1 += ldo;
+        if (two) {
+            const uint32_t x2 = cc2 * c + (cq2 * pq + b2);
+            if (ok) __stcs(o2, x2);
+            o2 += ldo;
+        }
+    }
+}
+
 template <int EPI>
 __global__ void __launch_bounds__(NTHREADS, 1)
 gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
@@ -598,6 +640,10 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 if (!args.swap) {
                     epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, gl - lane, gc0 + 32 * hh, pl, pcol,
                                         ia, small_n, want_dp);
+                    continue;
+                }
+                if (EPI == EPI_COUNTS) {
+                    epi_swapped_counts(args, v, lane, gl, gc0 + 32 * hh, ncols - 32 * hh, pl, pcol);
                     continue;
                 }
                 if (!__any_sync(0xffffffffu, rows_ok)) continue;   // warp-uniform skip only:
