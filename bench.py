@@ -575,8 +575,12 @@ def run_ours(args):
                 "kernel_ms": kern_ms, "kernel": kernel, "peak_src": f"{peaks['src']} MEASURED_PEAKS.json copy"}
     roof["traffic"] = roof_hbm["traffic"] = traffic
     roof["alg_cmp_per_launch"] = wlrun["kernel_cmp"]
-    # north_star: LD against the chosen pipe's peak, FastID against HBM bandwidth
-    if wl["kind"] == "fastid":
+    # the binding roof of this launch: its algorithmic bytes at the HBM peak vs its
+    # comparisons at the pipe's peak (FastID at 64 queries is HBM-bound, LD and FastID
+    # with 1,024 queries are compute-bound; north_star)
+    t_hbm = wlrun["kernel_bytes"] / (peaks["hbm_gbs"] * 1e9)
+    t_pipe = 2 * kcmp / (roof["peak"] * 1e12)
+    if t_hbm >= t_pipe:
         roof_primary, roof_secondary = roof_hbm, roof
     else:
         roof_primary, roof_secondary = roof, roof_hbm

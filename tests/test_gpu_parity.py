@@ -381,10 +381,12 @@ def test_search_kernel_choice(snp):
     assert snp.snp_last_kernel() == "fastid_mxf4"
 
 
-def test_search_ties_lowest_index_across_ctas(snp):
+@pytest.mark.parametrize("nq", [40, 100])
+def test_search_ties_lowest_index_across_ctas(snp, nq):
     """Many exact ties spread over every CTA, warp and lane quarter: the merged best
-    must be the lowest database index (reading R4), for counts and best-only."""
-    nbits, nd, nq = 1000, 200_000, 40
+    must be the lowest database index (reading R4), for counts and best-only.  nq = 40
+    runs the FastID kernel, nq = 100 the general kernel's fused two-op best."""
+    nbits, nd = 1000, 200_000
     base = snpgen.fastid_db(41, np.arange(13), nbits)
     idx = (np.arange(nd) * 7 + 3) % 13                # row j = base[idx[j]]
     db = base[idx]
