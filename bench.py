@@ -548,8 +548,14 @@ def run_ours(args):
 
     # roofline of the dominant kernel (the bit-GEMM launch), live CUDA-event durations
     kcmp = wlrun["kernel_cmp"]
+    kcmp_eff = kcmp
+    if kernel == "tc_mxf4_sym":
+        # f3 symmetric self-LD executes only the upper-triangle 128 x 128 tiles (SURVEY §8d:
+        # roofline on the executed work, M*N*nbits reported as the effective rate)
+        T = -(-wl["m"] // 128)
+        kcmp = T * (T + 1) // 2 * 128 * 128 * wl["nbits"]
     tops = 2 * kcmp / (kern_ms / 1e3) / 1e12
-    if kernel in ("tc_mxf4", "fastid_mxf4"):
+    if kernel in ("tc_mxf4", "tc_mxf4_sym", "fastid_mxf4"):
         roof = {"bound": "tensor", "achieved": tops, "peak": peaks["f4_tops"], "unit": "TOPS",
                 "peak_src": f"fp4 dense = 4 x bf16 burst ({peaks['src']} MEASURED_PEAKS.json)"}
     elif kernel == "tc_i8":
@@ -574,7 +580,10 @@ def run_ours(args):
                 "frac": hbm_gbs / peaks["hbm_gbs"], "alg_bytes_per_launch": wlrun["kernel_bytes"],
                 "kernel_ms": kern_ms, "kernel": kernel, "peak_src": f"{peaks['src']} MEASURED_PEAKS.json copy"}
     roof["traffic"] = roof_hbm["traffic"] = traffic
-    roof["alg_cmp_per_launch"] = wlrun["kernel_cmp"]
+    roof["alg_cmp_per_launch"] = kcmp
+    if kcmp != kcmp_eff:
+        roof["effective_cmp_per_launch"] = kcmp_eff
+        roof["effective_tops"] = 2 * kcmp_eff / (kern_ms / 1e3) / 1e12
     # the binding roof of this launch: its algorithmic bytes at the HBM peak vs its
     # comparisons at the pipe's peak (FastID at 64 queries is HBM-bound, LD and FastID
     # with 1,024 queries are compute-bound; north_star)

@@ -77,6 +77,7 @@ struct GArgs {
     int debug_skip;   // profiling experiment: expanders only pass tokens (results invalid)
     int order;        // tile raster: 2 grouped (default), 1 lane-block-major, 0 column-block-major
     int off32;        // every output element offset (row * ldo + col) fits in 32 bits
+    int sym;          // f3 symmetric self-LD: only tiles lb <= cb, off-diagonal ones mirrored
     int op2;          // EPI_COUNTS, swapped layout: second op written to C2 (or C2 = NULL)
     uint32_t *C2;
     const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
@@ -188,13 +189,92 @@ __device__ __forceinline__ uint32_t acc_count(uint32_t v, bool small) {
 //           r2 = min(1, (num / da) (num / db)) with 1/da, 1/db from 2 roundings each: 9
 //           fp32 roundings in total, relative error <= 9 * 2^-24 = 5.4e-7;
 //           exactly 0 where num = 0.  D' = num / Dmax (correctly rounded division).
+
+// f3 symmetric self-LD: the mirror image of an off-diagonal block.  Block (rows row0 + lane,
+// columns col0 + u) is also block (rows col0 + u, columns row0 + lane) of the output, and
+// every output is symmetric (AND / XOR counts, r2, D'), so before the transpose (lane = row
+// i, c[u] = column col0 + u) each u is one coalesced 128-byte store of row col0 + u.
+template <int EPI>
+__device__ __forceinline__ void epi_mirror(const GArgs &args, const uint32_t (&c)[32], int lane, int64_t row0,
+                                           int64_t col0, uint32_t pl, uint32_t pcol, float ia, bool small_n,
+                                           bool want_dp) {
+    const int64_t gi = row0 + lane;                 // becomes the output column
+    const bool ok_i = gi < args.nl;
+    const int64_t ldo = args.ldo;
+    const int64_t n = args.nbits;
+    const int32_t n32 = (int32_t)n;
+    const int ncol = (int)(args.nc - col0 < 32 ? args.nc - col0 : 32);   // output rows here
+    const float ibl = EPI == EPI_LD ? inv_exact((int64_t)pcol * (n - (int64_t)pcol)) : 0.f;
+    const int64_t o0 = col0 * ldo + gi;
+    if (EPI == EPI_LD && small_n && !want_dp && args.off32) {
+        // the benchmarked path: 32-bit element offsets, predicated evict-first stores
+        float *const r2b = args.r2;
+        uint32_t *const cb = args.C;
+        const bool has_c = cb != nullptr;
+        uint32_t off = (uint32_t)o0;
+        const uint32_t ld32 = (uint32_t)ldo;
+        const int32_t npl = -(int32_t)pl;
+#pragma unroll
+        for (int u = 0; u < 32; ++u) {
+            const int32_t pb = (int32_t)__shfl_sync(0xffffffffu, pcol, u);
+            const float ib = __shfl_sync(0xffffffffu, ibl, u);
+            const int32_t num = n32 * (int32_t)c[u] + npl * pb;
+            const float fn = (float)num;
+            const float r2v = fminf(__fmul_rn(__fmul_rn(fn, ia), __fmul_rn(fn, ib)), 1.0f);
+            const uint32_t okr = (ok_i && u < ncol) ? 1u : 0u, okc = (okr && has_c) ? 1u : 0u;
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(
+                             r2b + off),
+                         "f"(r2v), "r"(okr)
+                         : "memory");
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(
+                             cb + off),
+                         "r"(c[u]), "r"(okc)
+                         : "memory");
+            off += ld32;
+        }
+        return;
+    }
+#pragma unroll
+    for (int u = 0; u < 32; ++u) {   // fully unrolled: c[u] stays in registers
+        const uint32_t pb = __shfl_sync(0xffffffffu, pcol, u);   // popcount of SNP col0 + u
+        const float ib = EPI == EPI_LD ? __shfl_sync(0xffffffffu, ibl, u) : 0.f;
+        if (!ok_i || u >= ncol) continue;
+        const int64_t o = o0 + (int64_t)u * ldo;
+        const uint32_t cu = c[u];
+        if (EPI == EPI_COUNTS) {
+            const uint32_t x = args.op == 0 ? cu : pl + pb - 2u * cu;   // AND or XOR (symmetric)
+            if (args.accumulate) args.C[o] += x;
+            else __stcs(args.C + o, x);
+        } else {
+            float r2v, dpv = 0.f;
+            if (small_n) {
+                const int32_t num = n32 * (int32_t)cu - (int32_t)pl * (int32_t)pb;
+                const float fn = (float)num;
+                r2v = fminf(__fmul_rn(__fmul_rn(fn, ia), __fmul_rn(fn, ib)), 1.0f);
+                if (want_dp && num != 0) {
+                    const int32_t pa_ = (int32_t)pl, pb_ = (int32_t)pb;
+                    const int32_t dmax = num > 0 ? min(pa_ * (n32 - pb_), (n32 - pa_) * pb_)
+                                                 : min(pa_ * pb_, (n32 - pa_) * (n32 - pb_));
+                    dpv = __fdiv_rn(fn, (float)dmax);
+                }
+            } else {
+                ld_stats_f32(n, (int64_t)pl, (int64_t)pb, (int64_t)cu, r2v, dpv);
+            }
+            __stcs(args.r2 + o, r2v);
+            if (want_dp) __stcs(args.dprime + o, dpv);
+            if (args.C) __stcs(args.C + o, cu);
+        }
+    }
+}
+
 template <int EPI>
 __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[32], uint32_t *tw, int lane,
                                                int64_t row0, int64_t col0, uint32_t pl, uint32_t pcol, float ia,
-                                               bool small_n, bool want_dp) {
+                                               bool small_n, bool want_dp, bool mirror) {
     const bool small = args.nbits < (1LL << 23);
 #pragma unroll
     for (int i = 0; i < 32; ++i) c[i] = acc_count(c[i], small);   // in place: c is the TMEM load
+    if (mirror) epi_mirror<EPI>(args, c, lane, row0, col0, pl, pcol, ia, small_n, want_dp);
     __syncwarp();   // the previous block's reads of tw are done
 #pragma unroll
     for (int k = 0; k < 8; ++k) {
@@ -382,7 +462,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t nbits = args.nbits;
     const int nst = args.nst;
-    const int64_t ntiles = args.nlb * args.ncb;
+    const int64_t ntiles = args.sym ? args.nlb * (args.nlb + 1) / 2 : args.nlb * args.ncb;
     // 32-bit tile arithmetic (ntiles < 2^31): a 64-bit division is a subroutine CALL, and
     // any call in the kernel made ptxas drop the MMA issue loop out of uniform registers
     const uint32_t nlb32 = (uint32_t)args.nlb, ncb32 = (uint32_t)args.ncb;
@@ -393,7 +473,33 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     // its whole column sweep (DRAM reads ~ nlb/RG x the column operand instead of ~nlb x).
     // order 1: lane-block-major; order 0: column-block-major.
     constexpr uint32_t RG = 16;
+    // f3: the upper triangle (lb <= cb) of the T x T tile grid in groups of RG lane blocks;
+    // inside a group column block major, lane block fastest (a triangle, then a rectangle)
+    auto decode_sym = [&](uint32_t t, uint32_t &lb, uint32_t &cb) {
+        const uint32_t T = nlb32;
+        uint32_t g0 = 0;
+        for (;;) {
+            const uint32_t R = T - g0 < RG ? T - g0 : RG;
+            const uint32_t nt = R * (R + 1) / 2 + R * (T - g0 - R);
+            if (t < nt || R < RG) break;
+            t -= nt;
+            g0 += R;
+        }
+        const uint32_t R = T - g0 < RG ? T - g0 : RG;
+        const uint32_t tri = R * (R + 1) / 2;
+        if (t < tri) {
+            uint32_t k = 0;
+            while ((k + 1) * (k + 2) / 2 <= t) ++k;
+            cb = g0 + k;
+            lb = g0 + (t - k * (k + 1) / 2);
+        } else {
+            t -= tri;
+            cb = g0 + R + t / R;
+            lb = g0 + t % R;
+        }
+    };
     auto tile_lb = [&](uint32_t t) -> uint32_t {
+        if (args.sym) { uint32_t lb, cb; decode_sym(t, lb, cb); return lb; }
         if (args.order == 2) {
             const uint32_t g = t / (RG * ncb32), w = t - g * RG * ncb32;
             const uint32_t rows = nlb32 - g * RG < RG ? nlb32 - g * RG : RG;
@@ -402,6 +508,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         return args.order ? t / ncb32 : t % nlb32;
     };
     auto tile_cb = [&](uint32_t t) -> uint32_t {
+        if (args.sym) { uint32_t lb, cb; decode_sym(t, lb, cb); return cb; }
         if (args.order == 2) {
             const uint32_t g = t / (RG * ncb32), w = t - g * RG * ncb32;
             const uint32_t rows = nlb32 - g * RG < RG ? nlb32 - g * RG : RG;
@@ -458,7 +565,10 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
                 const int64_t t = blockIdx.x + tl * gridDim.x;
                 const uint32_t t32 = (uint32_t)t;
-                const int32_t rl = (int32_t)(tile_lb(t32) * BM), rc = (int32_t)(tile_cb(t32) * BN);
+                uint32_t lbt, cbt;
+                if (args.sym) decode_sym(t32, lbt, cbt);
+                else { lbt = tile_lb(t32); cbt = tile_cb(t32); }
+                const int32_t rl = (int32_t)(lbt * BM), rc = (int32_t)(cbt * BN);
                 for (int s = 0; s < nst; ++s) {
                     if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
                     ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
@@ -604,8 +714,12 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
             const int64_t t = blockIdx.x + tl * gridDim.x;
             const uint32_t t32 = (uint32_t)t;
-            const int64_t gl = (int64_t)tile_lb(t32) * BM + li;
-            const int64_t gc0 = (int64_t)tile_cb(t32) * BN + c0;
+            uint32_t lbt, cbt;
+            if (args.sym) decode_sym(t32, lbt, cbt);
+            else { lbt = tile_lb(t32); cbt = tile_cb(t32); }
+            const bool mirror = args.sym && lbt != cbt;   // f3: also write the mirror block
+            const int64_t gl = (int64_t)lbt * BM + li;
+            const int64_t gc0 = (int64_t)cbt * BN + c0;
             const bool rows_ok = gl < args.nl && gc0 < args.nc;
             const int ncols = gc0 < args.nc ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
             // popcounts: lane j holds the column popcounts of columns c0 + j and c0 + 32 + j
@@ -639,7 +753,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 const uint32_t pcol = hh ? pcol1 : pcol0;
                 if (!args.swap) {
                     epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, gl - lane, gc0 + 32 * hh, pl, pcol,
-                                        ia, small_n, want_dp);
+                                        ia, small_n, want_dp, mirror);
                     continue;
                 }
                 if (EPI == EPI_COUNTS) {
@@ -1107,7 +1221,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
                     if (lane == 0) arrive_remote(&acce[acc], 0);   // drained: the leader may reuse it
                 }
                 epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, gl - lane, gc0 + 32 * hh, pl,
-                                    hh ? pcol1 : pcol0, ia, small_n, want_dp);
+                                    hh ? pcol1 : pcol0, ia, small_n, want_dp, false);
             }
         }
     }
@@ -1172,7 +1286,7 @@ cudaError_t launch_g(const GArgs &g, const uint32_t *L, int64_t ldl32, const uin
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    const int64_t ntiles = g.nlb * g.ncb;
+    const int64_t ntiles = g.sym ? g.nlb * (g.nlb + 1) / 2 : g.nlb * g.ncb;
     const int grid = (int)(ntiles < num_sms() ? ntiles : num_sms());
     kern<<<grid, NTHREADS, SMEM, s>>>(tmL, tmC, g);
     count_launches(1);
@@ -1202,6 +1316,11 @@ cudaError_t launch_g2(GArgs g, const uint32_t *L, int64_t ldl32, const uint32_t 
 }
 
 }  // namespace
+
+namespace {
+thread_local bool g_last_sym = false;
+}
+bool gemm_tc4_last_sym() { return g_last_sym; }
 
 bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
     return m >= 1 && n >= 1 && nbits >= 1 && nbits < (1LL << 24) && m < (1LL << 31) && n < (1LL << 31);
@@ -1235,6 +1354,15 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
     g.debug_skip = skip ? 1 : 0;
     g.off32 = (uint64_t)(swap ? a.n : a.m) * (uint64_t)a.ldc < (1ull << 32) ? 1 : 0;
+    // f3 symmetric self-LD (B aliases A, symmetric output: LD statistics, AND or XOR
+    // counts): only the upper-triangle tiles are computed, off-diagonal ones mirrored.
+    // SNP_GEMM_SYM=0 computes every tile.
+    static const char *syme = std::getenv("SNP_GEMM_SYM");
+    // Only with at least two waves of full tiles: below that the doubled epilogue of the
+    // mirrored tiles is exposed (LD-2K: 256 tiles, 37 us full vs 46 us triangle).
+    const int64_t full_tiles = ((a.m + BM - 1) / BM) * ((a.n + BN - 1) / BN);
+    g.sym = (!swap && a.A == a.B && a.m == a.n && a.lda32 == a.ldb32 && (epi == EPI_LD || a.op <= 1) &&
+             full_tiles > 2 * num_sms() && !(syme && syme[0] == '0')) ? 1 : 0;
     static const char *ord = std::getenv("SNP_GEMM_ORDER");
     g.order = ord ? (ord[0] - '0') : 2;
     // CTA-pair kernel: opt-in (SNP_GEMM_X2=1) for the unswapped shapes with more than one
@@ -1243,6 +1371,8 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     // rate of the 1-CTA M = N = 128 ones here), so the 1-CTA kernel is the default.
     static const char *x2e = std::getenv("SNP_GEMM_X2");
     const bool use_x2 = !swap && g.nl > BM && x2e && x2e[0] == '1';
+    if (use_x2) g.sym = 0;
+    g_last_sym = g.sym != 0;
     if (use_x2)
         return epi == EPI_LD ? launch_g2<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g2<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
     return epi == EPI_LD ? launch_g<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);

@@ -148,7 +148,7 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
         } else {
             e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
         }
-        g_last_kernel = kern;
+        g_last_kernel = (kern == SNP_KERNEL_TC_MXF4 && gemm_tc4_last_sym()) ? SNP_KERNEL_TC_MXF4_SYM : kern;
     } else {
         e = launch_bitgemm_popc(a, epi, s);
         g_last_kernel = SNP_KERNEL_POPC;

@@ -78,6 +78,8 @@ cudaError_t launch_bitgemm_tc(const GemmArgs &a, int epi, void *ws, size_t ws_by
 // General tcgen05 mxf4 kernel (gemm_tc4.cu): 128x128 tiles, TMA-fed, A in TMEM.
 bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits);
 cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s);
+// Whether the most recent launch_gemm_tc4 on this thread ran the symmetric (f3) schedule.
+bool gemm_tc4_last_sym();
 
 // FastID-shaped tcgen05 mxf4 kernel (fastid_tc4.cu): <= 128 queries resident in shared
 // memory, database streamed by TMA.  The queries are the user's first operand.

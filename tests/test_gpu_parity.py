@@ -313,7 +313,7 @@ def test_cfg3_ld_32k_full_cross_variant(snp, mode):
                 got = snp.snp_ld_counts(A, A, nbits)
             else:
                 _, _, got = snp.snp_ld_r2(A, A, nbits, counts=True)
-            assert snp.snp_last_kernel() == "tc_mxf4"
+            assert snp.snp_last_kernel().startswith("tc_mxf4")
             assert int((got.view(torch.int32) != ref).sum().item()) == 0
             del got
     finally:
@@ -497,3 +497,20 @@ print("ok")
     r = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True, text=True,
                        timeout=600)
     assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
+
+
+@pytest.mark.parametrize("m,nbits", [(2300, 1025), (2200, 64)])
+def test_selfld_symmetric_mirror(snp, m, nbits):
+    """f3: self-LD (B aliases A) computes only the upper-triangle tiles and mirrors the
+    off-diagonal ones (used from > 2 waves of tiles: m >= 2177 here, ragged last tile);
+    every output (counts, r2, D') vs the oracle, and the matrices are exactly symmetric."""
+    g = snpgen.ld_genotypes(61, np.arange(m), nbits, structure=True)
+    A = pack_dev(snp, g, garbage_seed=9)
+    r2, dp, cnt = snp.snp_ld_r2(A, A, nbits, dprime=True, counts=True)
+    r2_ref, dp_ref, n_ref = oracle.ld(g, g)
+    c = u32(cnt)
+    assert np.array_equal(c, n_ref) and np.array_equal(c, c.T)
+    check_r2(r2.cpu().numpy(), r2_ref)
+    check_r2(dp.cpu().numpy(), dp_ref)
+    x = snp.snp_fastid(A, A, nbits, "xor")                 # symmetric op through the same path
+    assert np.array_equal(u32(x), oracle.counts(g, g, "xor"))
