@@ -267,6 +267,92 @@ __device__ __forceinline__ void epi_mirror(const GArgs &args, const uint32_t (&c
     }
 }
 
+
+// f3 fast path for an off-diagonal full 32 x 32 block of the benchmarked LD output (r2 +
+// counts, n <= 46340, no D'): r2 is computed ONCE in the pre-transpose layout (lane = row
+// i), stored mirrored straight away, and staged through the warp's transpose buffer for
+// the normal-orientation stores; the counts follow through the same buffer.
+__device__ __forceinline__ void st_cs_pred_f32(float *p, float v, uint32_t ok) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(p), "f"(v),
+                 "r"(ok)
+                 : "memory");
+}
+__device__ __forceinline__ void st_cs_pred_u32(uint32_t *p, uint32_t v, uint32_t ok) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
+                 "r"(ok)
+                 : "memory");
+}
+__device__ __forceinline__ void epi_ld_sym_fast(const GArgs &args, const uint32_t (&c)[32], uint32_t *tw, int lane,
+                                                int64_t row0, int64_t col0, uint32_t pl, uint32_t pcol, float ia) {
+    const int64_t ldo = args.ldo;
+    const int32_t n32 = (int32_t)args.nbits;
+    const uint32_t ld32 = (uint32_t)ldo;
+    float *const r2b = args.r2;
+    uint32_t *const cb = args.C;
+    const uint32_t has_c = cb != nullptr ? 1u : 0u;
+    const bool ok_i = row0 + lane < args.nl;                         // mirror column / normal row
+    const int ncol = (int)(args.nc - col0 < 32 ? args.nc - col0 : 32);
+    const uint32_t okn = (col0 + lane < args.nc) ? 1u : 0u;           // normal column
+    const uint32_t *twl = tw + (lane & 3);
+    const uint32_t xl = (uint32_t)(lane >> 2);
+    // 1. stage the counts (row i = lane, 16-byte chunks XOR-swizzled by row)
+    __syncwarp();   // the previous block's reads of tw are done
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        const uint32_t a = ptx::smem_u32(tw + lane * 32 + ((k ^ (lane & 7)) << 2));
+        asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(c[4 * k]), "r"(c[4 * k + 1]),
+                     "r"(c[4 * k + 2]), "r"(c[4 * k + 3])
+                     : "memory");
+    }
+    __syncwarp();
+    // 2. counts in the normal orientation (lane = column)
+    if (has_c) {
+        uint32_t off = (uint32_t)(row0 * ldo + col0 + lane);
+#pragma unroll
+        for (int r = 0; r < 32; ++r) {
+            st_cs_pred_u32(cb + off, twl[r * 32 + ((xl ^ (uint32_t)(r & 7)) << 2)], okn);
+            off += ld32;
+        }
+    }
+    __syncwarp();
+    // 3. r2 once per element from this lane's own row chunks: mirrored stores (row col0 + u,
+    //    column row0 + lane; counts too), and r2 written back over the chunk just read
+    const float ibl = inv_exact((int64_t)pcol * ((int64_t)n32 - (int64_t)pcol));
+    const int32_t npl = -(int32_t)pl;
+    uint32_t offm = (uint32_t)(col0 * ldo + row0 + lane);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        const uint32_t a = ptx::smem_u32(tw + lane * 32 + ((k ^ (lane & 7)) << 2));
+        uint32_t cc[4];
+        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(cc[0]), "=r"(cc[1]), "=r"(cc[2]), "=r"(cc[3])
+                     : "r"(a) : "memory");
+        float r[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const int u = 4 * k + t;
+            const int32_t pb = (int32_t)__shfl_sync(0xffffffffu, pcol, u);
+            const float ib = __shfl_sync(0xffffffffu, ibl, u);
+            const int32_t num = n32 * (int32_t)cc[t] + npl * pb;
+            const float fn = (float)num;
+            r[t] = fminf(__fmul_rn(__fmul_rn(fn, ia), __fmul_rn(fn, ib)), 1.0f);
+            const uint32_t ok = (ok_i && u < ncol) ? 1u : 0u;
+            st_cs_pred_f32(r2b + offm, r[t], ok);
+            st_cs_pred_u32(cb + offm, cc[t], ok & has_c);
+            offm += ld32;
+        }
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(r[0]), "f"(r[1]), "f"(r[2]), "f"(r[3])
+                     : "memory");
+    }
+    __syncwarp();
+    // 4. r2 in the normal orientation
+    uint32_t off = (uint32_t)(row0 * ldo + col0 + lane);
+#pragma unroll
+    for (int r = 0; r < 32; ++r) {
+        st_cs_pred_f32(r2b + off, __uint_as_float(twl[r * 32 + ((xl ^ (uint32_t)(r & 7)) << 2)]), okn);
+        off += ld32;
+    }
+}
+
 template <int EPI>
 __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[32], uint32_t *tw, int lane,
                                                int64_t row0, int64_t col0, uint32_t pl, uint32_t pcol, float ia,
@@ -274,6 +360,10 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
     const bool small = args.nbits < (1LL << 23);
 #pragma unroll
     for (int i = 0; i < 32; ++i) c[i] = acc_count(c[i], small);   // in place: c is the TMEM load
+    if (EPI == EPI_LD && mirror && small_n && !want_dp && args.off32 && args.nl - row0 >= 32) {
+        epi_ld_sym_fast(args, c, tw, lane, row0, col0, pl, pcol, ia);
+        return;
+    }
     if (mirror) epi_mirror<EPI>(args, c, lane, row0, col0, pl, pcol, ia, small_n, want_dp);
     __syncwarp();   // the previous block's reads of tw are done
 #pragma unroll
