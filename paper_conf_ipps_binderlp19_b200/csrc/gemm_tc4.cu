@@ -190,6 +190,17 @@ __device__ __forceinline__ uint32_t acc_count(uint32_t v, bool small) {
 //           fp32 roundings in total, relative error <= 9 * 2^-24 = 5.4e-7;
 //           exactly 0 where num = 0.  D' = num / Dmax (correctly rounded division).
 
+// predicated evict-first stores (no branch around them: shuffles stay converged)
+__device__ __forceinline__ void st_cs_pred_f32(float *p, float v, uint32_t ok) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(p), "f"(v),
+                 "r"(ok)
+                 : "memory");
+}
+__device__ __forceinline__ void st_cs_pred_u32(uint32_t *p, uint32_t v, uint32_t ok) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
+                 "r"(ok)
+                 : "memory");
+}
 // f3 symmetric self-LD: the mirror image of an off-diagonal block.  Block (rows row0 + lane,
 // columns col0 + u) is also block (rows col0 + u, columns row0 + lane) of the output, and
 // every output is symmetric (AND / XOR counts, r2, D'), so before the transpose (lane = row
@@ -206,6 +217,19 @@ __device__ __forceinline__ void epi_mirror(const GArgs &args, const uint32_t (&c
     const int ncol = (int)(args.nc - col0 < 32 ? args.nc - col0 : 32);   // output rows here
     const float ibl = EPI == EPI_LD ? inv_exact((int64_t)pcol * (n - (int64_t)pcol)) : 0.f;
     const int64_t o0 = col0 * ldo + gi;
+    if (EPI == EPI_COUNTS && !args.accumulate && args.off32) {
+        uint32_t off = (uint32_t)o0;
+        const uint32_t ld32 = (uint32_t)ldo;
+        const bool xo = args.op == 1;   // XOR (else AND): the symmetric ops
+#pragma unroll
+        for (int u = 0; u < 32; ++u) {
+            const uint32_t pb = __shfl_sync(0xffffffffu, pcol, u);
+            const uint32_t x = xo ? pl + pb - 2u * c[u] : c[u];
+            st_cs_pred_u32(args.C + off, x, (ok_i && u < ncol) ? 1u : 0u);
+            off += ld32;
+        }
+        return;
+    }
     if (EPI == EPI_LD && small_n && !want_dp && args.off32) {
         // the benchmarked path: 32-bit element offsets, predicated evict-first stores
         float *const r2b = args.r2;
@@ -272,16 +296,6 @@ __device__ __forceinline__ void epi_mirror(const GArgs &args, const uint32_t (&c
 // counts, n <= 46340, no D'): r2 is computed ONCE in the pre-transpose layout (lane = row
 // i), stored mirrored straight away, and staged through the warp's transpose buffer for
 // the normal-orientation stores; the counts follow through the same buffer.
-__device__ __forceinline__ void st_cs_pred_f32(float *p, float v, uint32_t ok) {
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(p), "f"(v),
-                 "r"(ok)
-                 : "memory");
-}
-__device__ __forceinline__ void st_cs_pred_u32(uint32_t *p, uint32_t v, uint32_t ok) {
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
-                 "r"(ok)
-                 : "memory");
-}
 __device__ __forceinline__ void epi_ld_sym_fast(const GArgs &args, const uint32_t (&c)[32], uint32_t *tw, int lane,
                                                 int64_t row0, int64_t col0, uint32_t pl, uint32_t pcol, float ia) {
     const int64_t ldo = args.ldo;
@@ -382,6 +396,26 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
     const int32_t pb = (int32_t)pcol;
     const int rows = (int)(args.nl - row0 < 32 ? args.nl - row0 : 32);   // warp-uniform
     const int64_t o0 = row0 * ldo + gc;
+    if (EPI == EPI_COUNTS && rows == 32 && !args.accumulate && args.off32) {
+        // full block, fully unrolled: x = cq pQ + cd pD + cc c, predicated
+        // evict-first stores at 32-bit element offsets
+        const int op = args.op;
+        const uint32_t cq = (op == 1 || op == 2) ? 1u : 0u, cdp = (op == 1 || op == 3) ? pcol : 0u;
+        const uint32_t cc = op == 0 ? 1u : op == 1 ? (uint32_t)-2 : (uint32_t)-1;
+        const uint32_t *twl = tw + (lane & 3);
+        const uint32_t xl = (uint32_t)(lane >> 2);
+        const uint32_t okn = colok ? 1u : 0u;
+        uint32_t off = (uint32_t)o0;
+        const uint32_t ld32 = (uint32_t)ldo;
+#pragma unroll
+        for (int r = 0; r < 32; ++r) {
+            const uint32_t plr = __shfl_sync(0xffffffffu, pl, r);
+            const uint32_t c = twl[r * 32 + ((xl ^ (uint32_t)(r & 7)) << 2)];
+            st_cs_pred_u32(args.C + off, cc * c + (cq * plr + cdp), okn);
+            off += ld32;
+        }
+        return;
+    }
     if (EPI == EPI_COUNTS) {
         uint32_t *cp = args.C + o0;
         const int op = args.op;
