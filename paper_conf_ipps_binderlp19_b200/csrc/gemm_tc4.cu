@@ -680,6 +680,10 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     ptx::tc_fence_before();
     __syncthreads();
     ptx::tc_fence_after();
+    // programmatic dependent launch: the setup above overlapped the previous kernel (the
+    // row-popcount pre-pass); its results are visible after this wait, and nothing global
+    // was read or written before it
+    asm volatile("griddepcontrol.wait;" ::: "memory");
 
     if (warp == TMA_WARP) {
         // ------------------------------------------------------------ TMA producer
@@ -1412,8 +1416,19 @@ cudaError_t launch_g(const GArgs &g, const uint32_t *L, int64_t ldl32, const uin
     }
     const int64_t ntiles = g.sym ? g.nlb * (g.nlb + 1) / 2 : g.nlb * g.ncb;
     const int grid = (int)(ntiles < num_sms() ? ntiles : num_sms());
-    kern<<<grid, NTHREADS, SMEM, s>>>(tmL, tmC, g);
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3((unsigned)NTHREADS);
+    cfg.dynamicSmemBytes = SMEM;
+    cfg.stream = s;
+    cudaLaunchAttribute pdl[1];
+    pdl[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    pdl[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = pdl;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, tmL, tmC, g);
     count_launches(1);
+    if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
 

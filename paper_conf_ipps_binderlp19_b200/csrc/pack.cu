@@ -67,6 +67,10 @@ __global__ void pack_byte_kernel(const uint8_t *__restrict__ g, int64_t rows, in
 // One warp per row; lanes stride over the row's words; last word masked.
 __global__ void row_popc_kernel(const uint64_t *__restrict__ x, int64_t rows, int64_t nbits,
                                 int64_t ldw, uint32_t *__restrict__ popc) {
+    // programmatic dependent launch: wait for the producer of x (e.g. snp_pack), then let
+    // the consumer (the bit-GEMM) start its setup while the popcounts are being computed
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -110,8 +114,18 @@ cudaError_t launch_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int6
                             uint32_t *popc, cudaStream_t s) {
     const int threads = 256;
     const int blocks = grid_for(rows * 32, threads);
-    row_popc_kernel<<<blocks, threads, 0, s>>>(x, rows, nbits, ldw, popc);
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3((unsigned)threads);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, row_popc_kernel, x, rows, nbits, ldw, popc);
     count_launches(1);
+    if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
 
