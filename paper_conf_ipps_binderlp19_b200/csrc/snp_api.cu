@@ -349,6 +349,18 @@ bool search_fused(int64_t nq, int64_t nd, int64_t nbits) {
            tc_kernel_for(nq, nd, nbits, EPI_COUNTS) == SNP_KERNEL_FASTID_MXF4;
 }
 
+// a7 measured dispatch (configs[4] sweep, profiles/round1/sweep.txt): for more than 64
+// queries at nbits <= 4096 the fused FastID kernel run on 64-query slices (one database
+// pass each) beats the general kernel + best pass (e.g. M = 128 x 1M x 2048: 0.28 vs
+// 0.63 ms, M = 8192 x 1M x 4096: 26 vs 31 ms); above 4096 bits the general kernel wins.
+constexpr int64_t SLICE_Q = 64;
+bool search_sliced(int64_t nq, int64_t nd, int64_t nbits) {
+    const char *e = std::getenv("SNP_SEARCH_SLICES");   // "0": never (A/B measurement hook)
+    if (e && e[0] == '0') return false;
+    return nq > SLICE_Q && nd > 0 && nbits <= 4096 && choose_variant(nq, nd, nbits) == SNP_VARIANT_TC &&
+           fastid_tc4_supported(SLICE_Q, nd, nbits) && nd >= 4 * SLICE_Q;
+}
+
 }  // namespace
 
 extern "C" {
@@ -357,6 +369,7 @@ size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, 
     if (nq <= 0 || nbits <= 0 || nops < 1 || nops > 4) return 0;
     if (nd < 0) return 0;
     if (search_fused(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(nq, nops);
+    if (search_sliced(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(SLICE_Q, nops);
     size_t b = align256((size_t)nops * nq * 8);
     if (nd == 0) return b;
     b += align256((size_t)nq * search_chunk_rows(nq, nd) * 4);
@@ -429,6 +442,27 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
         a.keys = reinterpret_cast<unsigned long long *>(ws);
         a.done = reinterpret_cast<unsigned int *>((char *)ws + align256((size_t)nops * nq * 8));
         if ((e = launch_fastid_search_tc4(a, s)) != cudaSuccess) return set_cuda_error(e);
+        g_last_variant = SNP_VARIANT_TC;
+        g_last_kernel = SNP_KERNEL_FASTID_MXF4;
+        return SNP_OK;
+    }
+
+    if (search_sliced(nq, nd, nbits)) {
+        // 64-query slices through the fused kernel, one database pass each; the key
+        // workspace is reused slice after slice (stream order; each launch re-initialises it)
+        for (int64_t q0 = 0; q0 < nq; q0 += SLICE_Q) {
+            SearchArgs b = a;
+            b.Q = a.Q + q0 * a.ldq32;
+            b.nq = nq - q0 < SLICE_Q ? nq - q0 : SLICE_Q;
+            for (int j = 0; j < nops; ++j) {
+                b.counts[j] = a.counts[j] ? a.counts[j] + q0 * ldo : nullptr;
+                b.best_count[j] = a.best_count[j] ? a.best_count[j] + q0 : nullptr;
+                b.best_index[j] = a.best_index[j] ? a.best_index[j] + q0 : nullptr;
+            }
+            b.keys = reinterpret_cast<unsigned long long *>(ws);
+            b.done = reinterpret_cast<unsigned int *>((char *)ws + align256((size_t)nops * SLICE_Q * 8));
+            if ((e = launch_fastid_search_tc4(b, s)) != cudaSuccess) return set_cuda_error(e);
+        }
         g_last_variant = SNP_VARIANT_TC;
         g_last_kernel = SNP_KERNEL_FASTID_MXF4;
         return SNP_OK;

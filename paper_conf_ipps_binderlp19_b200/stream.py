@@ -1,0 +1,86 @@
+"""f2 — end-to-end streaming FastID search.
+
+The paper measures FastID end to end, with the database moved to the device in chunks and
+the transfers overlapped with the comparisons by double buffering.  Here the
+packed database stays in pinned host memory and is streamed through two device buffers:
+the H2D copy of chunk k+1 runs on a copy stream (copy engine) while chunk k is searched on
+the compute stream (``snp_fastid_search``, per-query best match, no count matrix), events
+order buffer reuse.  Each chunk's best (count, global index) lands in its own row of a
+``[chunks, nq]`` table; chunks are contiguous and increasing, so the final merge is the
+multi-GPU merge with the lowest-global-index tie-break (reading R4).
+
+Host logic only (chunk planning, stream/event ordering, argument marshalling): every
+comparison runs in the library's kernels.
+"""
+from __future__ import annotations
+
+import torch
+
+
+def chunk_plan(nd: int, chunk_rows: int, align: int = 128) -> list[tuple[int, int]]:
+    """Contiguous [r0, r1) database chunks of at most chunk_rows rows (a multiple of
+    align, at least align); the last one is ragged.  nd = 0 gives no chunks."""
+    if nd < 0 or chunk_rows < 1 or align < 1:
+        raise ValueError("nd >= 0, chunk_rows >= 1, align >= 1")
+    step = max(align, chunk_rows // align * align)
+    return [(r0, min(nd, r0 + step)) for r0 in range(0, nd, step)]
+
+
+def stream_search(Q: torch.Tensor, D_host: torch.Tensor, nbits: int, ops=("xor", "andnot"),
+                  popD_host: torch.Tensor | None = None, chunk_rows: int = 1 << 20,
+                  index_base: int = 0):
+    """Per-query best match of every op over a database in pinned host memory.
+
+    Q: packed queries on the device; D_host: packed database rows (uint64, pinned CPU);
+    popD_host: optional pinned uint32 row popcounts (else counted on the device per
+    chunk).  Returns a list (one per op) of (best_count uint32-in-int64, best_index int64)
+    device tensors of length nq; an empty database gives (0xFFFFFFFF, -1)."""
+    from . import snp_fastid_search, snp_fastid_search_workspace_bytes, snp_row_popc
+    from .multigpu import merge_best
+    if isinstance(ops, str):
+        ops = (ops,)
+    if D_host.is_cuda or not D_host.is_pinned():
+        raise ValueError("D_host must be a pinned CPU tensor")
+    if popD_host is not None and (popD_host.is_cuda or not popD_host.is_pinned()):
+        raise ValueError("popD_host must be a pinned CPU tensor")
+    dev = Q.device
+    nq, nd = Q.shape[0], D_host.shape[0]
+    plan = chunk_plan(nd, chunk_rows)
+    nops = len(ops)
+    bc = torch.full((nops, max(1, len(plan)), nq), 0xFFFFFFFF, dtype=torch.int64, device=dev)
+    bi = torch.full((nops, max(1, len(plan)), nq), -1, dtype=torch.int64, device=dev)
+    if not plan:
+        return [(bc[j, 0], bi[j, 0]) for j in range(nops)]
+    rows_max = max(r1 - r0 for r0, r1 in plan)
+    nbuf = min(2, len(plan))
+    Dbuf = [torch.empty((rows_max, D_host.shape[1]), dtype=D_host.dtype, device=dev) for _ in range(nbuf)]
+    Pbuf = [torch.empty(rows_max, dtype=torch.uint32, device=dev) for _ in range(nbuf)] if popD_host is not None else None
+    # per-chunk results are written as uint32 counts / int64 indices, then widened
+    cnt32 = torch.empty((nops, len(plan), nq), dtype=torch.uint32, device=dev)
+    ws = torch.empty(max(1, snp_fastid_search_workspace_bytes(nq, rows_max, nbits, nops)), dtype=torch.uint8,
+                     device=dev)
+    comp = torch.cuda.current_stream(dev)
+    copy = torch.cuda.Stream(dev)
+    copy.wait_stream(comp)   # the buffers (and Q) were just allocated / produced on comp
+    copied = [torch.cuda.Event() for _ in range(nbuf)]
+    freed = [torch.cuda.Event() for _ in range(nbuf)]
+    for k, (r0, r1) in enumerate(plan):
+        b, rows = k % nbuf, r1 - r0
+        with torch.cuda.stream(copy):
+            if k >= nbuf:
+                copy.wait_event(freed[b])          # chunk k - nbuf is done with buffer b
+            Dbuf[b][:rows].copy_(D_host[r0:r1], non_blocking=True)
+            if Pbuf is not None:
+                Pbuf[b][:rows].copy_(popD_host[r0:r1], non_blocking=True)
+            copied[b].record(copy)
+        comp.wait_event(copied[b])
+        D = Dbuf[b][:rows]
+        pd = Pbuf[b][:rows] if Pbuf is not None else snp_row_popc(D, nbits)
+        snp_fastid_search(Q, D, nbits, ops, counts=False,
+                          best=[(cnt32[j, k], bi[j, k]) for j in range(nops)],
+                          index_base=index_base + r0, ws=ws, popD=pd)
+        freed[b].record(comp)
+    for buf in Dbuf + (Pbuf or []):
+        buf.record_stream(copy)
+    bc[:, :len(plan)] = cnt32.view(torch.int32).to(torch.int64) & 0xFFFFFFFF
+    return [merge_best(bc[j], bi[j]) for j in range(nops)]

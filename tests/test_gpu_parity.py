@@ -341,8 +341,10 @@ def test_cfg2_fastid_full_cross_variant(snp):
 # ------------------------------------------------------------------ f1 fused search
 
 ALL_OPS = ("and", "xor", "andnot", "notand")
+# > 64 queries: 64-query slices of the fused kernel up to 4096 bits (a7), above that the
+# general kernel (two ops per pass) + best pass
 SEARCH_SHAPES = [(1, 4, 1), (3, 700, 129), (33, 1000, 4096), (64, 2000, 777), (64, 300, 100),
-                 (70, 513, 1000), (130, 300, 2049)]
+                 (70, 513, 1000), (130, 300, 2049), (100, 3000, 5000)]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -514,3 +516,39 @@ def test_selfld_symmetric_mirror(snp, m, nbits):
     check_r2(dp.cpu().numpy(), dp_ref)
     x = snp.snp_fastid(A, A, nbits, "xor")                 # symmetric op through the same path
     assert np.array_equal(u32(x), oracle.counts(g, g, "xor"))
+
+
+@pytest.mark.parametrize("with_pop", [False, True])
+def test_stream_search_chunks(snp, with_pop):
+    """f2: database in pinned host memory streamed in ragged chunks through two device
+    buffers; per-query best of XOR and ANDNOT vs the oracle (lowest index on ties)."""
+    from paper_conf_ipps_binderlp19_b200.stream import stream_search
+    nq, nd, nbits = 40, 5000, 777
+    db = snpgen.fastid_db(71, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(71, nq, nd, nbits)
+    q[3] = db[4500]                                    # exact copy in the last chunk
+    D_host = pack_dev(snp, db).cpu().pin_memory()
+    pop = snp.snp_row_popc(D_host.to(DEV), nbits).cpu().pin_memory() if with_pop else None
+    Q = pack_dev(snp, q)
+    res = stream_search(Q, D_host, nbits, ("xor", "andnot"), popD_host=pop, chunk_rows=1500, index_base=11)
+    torch.cuda.synchronize()
+    for j, op in enumerate(("xor", "andnot")):
+        rb, ri = oracle.best(oracle.counts(q, db, op), 11)
+        assert np.array_equal(res[j][0].cpu().numpy().astype(np.uint32), rb), op
+        assert np.array_equal(res[j][1].cpu().numpy(), ri), op
+
+
+def test_search_general_kernel_forced(snp, monkeypatch):
+    """More than 64 queries at few bits with the 64-query slicing disabled: the general
+    kernel's paired-op pass (counts of two ops from one AND count) + best pass."""
+    monkeypatch.setenv("SNP_SEARCH_SLICES", "0")
+    nq, nd, nbits = 70, 513, 1000
+    db = snpgen.fastid_db(81, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(81, nq, nd, nbits)
+    counts, best = snp.snp_fastid_search(pack_dev(snp, q), pack_dev(snp, db), nbits, ALL_OPS, index_base=3)
+    assert snp.snp_last_kernel() == "tc_mxf4"
+    for j, op in enumerate(ALL_OPS):
+        ref = oracle.counts(q, db, op)
+        assert np.array_equal(u32(counts[j]), ref), op
+        rb, ri = oracle.best(ref, 3)
+        assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), op

@@ -113,3 +113,17 @@ def test_merge_best_edge_cases():
     assert i.tolist() == [200, 11, 202]
     c, i = merge_best(torch.tensor([[0xFFFFFFFF]]), torch.tensor([[-1]]))
     assert c.tolist() == [0xFFFFFFFF] and i.tolist() == [-1]
+
+
+def test_stream_chunk_plan():
+    """f2 host logic: contiguous, ordered, 128-aligned chunks covering [0, nd)."""
+    from paper_conf_ipps_binderlp19_b200.stream import chunk_plan
+    assert chunk_plan(0, 1000) == []
+    assert chunk_plan(100, 1000) == [(0, 100)]
+    assert chunk_plan(1000, 300) == [(0, 256), (256, 512), (512, 768), (768, 1000)]
+    assert chunk_plan(1000, 5) == [(r, min(1000, r + 128)) for r in range(0, 1000, 128)]
+    for nd, ch in [(1, 1), (12345, 4096), (4096, 4096)]:
+        p = chunk_plan(nd, ch)
+        assert p[0][0] == 0 and p[-1][1] == nd
+        assert all(a[1] == b[0] for a, b in zip(p, p[1:]))
+        assert all(r0 % 128 == 0 for r0, _ in p)
