@@ -281,13 +281,11 @@ def setup_fastid(wl, rank, world, dev):
     else:
         ws = {op: (torch.empty(snp.snp_fastid_workspace_bytes(nq, nd, nbits, op), dtype=torch.uint8, device=dev))
               for op in OPS}
-    gathered = {op: (torch.empty(world * nq, dtype=torch.int32, device=dev),
-                     torch.empty(world * nq, dtype=torch.int64, device=dev)) for op in OPS}
     merged = {}
     res_host = {op: (torch.empty(nq, dtype=torch.uint32).pin_memory(), torch.empty(nq, dtype=torch.int64).pin_memory())
                 for op in OPS}
     st = dict(D=D, Q=Q, qbytes=qbytes, qhost=qhost, outs=outs, best=best, ws=ws, lo=lo, nd=nd,
-              gathered=gathered, res_host=res_host)
+              res_host=res_host)
     cmp_rank = 2 * nq * nd * nbits
     cmp_all = 2 * nq * (nd_total if wl["scaling"] == "strong" else wl["nd"] * world) * nbits
 
@@ -326,16 +324,14 @@ def setup_fastid(wl, rank, world, dev):
                 if kev is not None:
                     kev[2 * i + 1].record(s)
                 _best(op)()                                                # a6
+        if world > 1:
+            # global best per query and op, lowest global index on ties: both
+            # ops' (count, index) packed into int64 keys, ONE all-gather, ONE min
+            from paper_conf_ipps_binderlp19_b200 import multigpu
+            keys = torch.stack([multigpu.pack_best(*best[op]) for op in OPS])
+            merged["keys"] = multigpu.gather_best(keys)
         for op in OPS:
             bc, bi = best[op]
-            if world > 1:
-                import torch.distributed as dist
-                from paper_conf_ipps_binderlp19_b200 import multigpu
-                gc, gi = gathered[op]
-                dist.all_gather_into_tensor(gc, bc.view(torch.int32))
-                dist.all_gather_into_tensor(gi, bi)
-                # global best per query, lowest global index on ties
-                merged[op] = multigpu.merge_best(gc.view(world, nq).to(torch.int64), gi.view(world, nq))
             if host:   # e2e: D2H of the step's result (per-query best count and index)
                 res_host[op][0].copy_(bc, non_blocking=True)
                 res_host[op][1].copy_(bi, non_blocking=True)

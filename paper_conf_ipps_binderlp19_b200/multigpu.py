@@ -42,6 +42,38 @@ def merge_best(gc: torch.Tensor, gi: torch.Tensor):
     return best_cnt, best_idx
 
 
+KEY_IDX_BITS = 40                     # global database index < 2^40; count < 2^23 above it
+KEY_NONE = (1 << 63) - 1              # an empty shard: larger than every real key
+
+
+def pack_best(bc: torch.Tensor, bi: torch.Tensor) -> torch.Tensor:
+    """(best count, global best index) -> one int64 key ``count << 40 | index`` whose
+    minimum over shards is the global best with the lowest-index tie-break (reading R4):
+    ONE all-gather and ONE min replace two gathers and an argmin merge."""
+    c = (bc.view(torch.int32) if bc.dtype == torch.uint32 else bc).to(torch.int64) & 0xFFFFFFFF
+    key = (c << KEY_IDX_BITS) | bi.to(torch.int64)
+    return torch.where(bi < 0, torch.full_like(key, KEY_NONE), key)
+
+
+def unpack_best(key: torch.Tensor):
+    """Inverse of pack_best; KEY_NONE -> (0xFFFFFFFF, -1)."""
+    none = key == KEY_NONE
+    c = torch.where(none, torch.full_like(key, 0xFFFFFFFF), key >> KEY_IDX_BITS)
+    i = torch.where(none, torch.full_like(key, -1), key & ((1 << KEY_IDX_BITS) - 1))
+    return c, i
+
+
+def gather_best(keys: torch.Tensor, group=None) -> torch.Tensor:
+    """keys: [..., nq] local packed keys (any number of ops stacked) -> global minimum over
+    the ranks with one all_gather_into_tensor."""
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    if world == 1:
+        return keys
+    g = torch.empty((world,) + tuple(keys.shape), dtype=keys.dtype, device=keys.device)
+    dist.all_gather_into_tensor(g.view(-1), keys.contiguous().view(-1), group=group)
+    return g.min(dim=0).values
+
+
 def fastid_step(Q: torch.Tensor, D_shard: torch.Tensor, nbits: int, op: str, index_base: int,
                 out: torch.Tensor | None = None, compute=None, best=None, group=None):
     """One sharded FastID step.  Q must be allocated on every rank (its content on
@@ -57,12 +89,7 @@ def fastid_step(Q: torch.Tensor, D_shard: torch.Tensor, nbits: int, op: str, ind
     if world == 1:
         return counts, bc.to(torch.int64), bi
     nq = bc.numel()
-    bc = bc.view(torch.int32) if bc.dtype == torch.uint32 else bc
-    gc = torch.empty(world * nq, dtype=bc.dtype, device=bc.device)
-    gi = torch.empty(world * nq, dtype=bi.dtype, device=bi.device)
-    dist.all_gather_into_tensor(gc, bc.contiguous(), group=group)
-    dist.all_gather_into_tensor(gi, bi.contiguous(), group=group)
-    c, i = merge_best(gc.view(world, nq).to(torch.int64), gi.view(world, nq))
+    c, i = unpack_best(gather_best(pack_best(bc, bi), group=group))
     return counts, c, i
 
 

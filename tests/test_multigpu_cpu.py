@@ -127,3 +127,19 @@ def test_stream_chunk_plan():
         assert p[0][0] == 0 and p[-1][1] == nd
         assert all(a[1] == b[0] for a, b in zip(p, p[1:]))
         assert all(r0 % 128 == 0 for r0, _ in p)
+
+
+def test_pack_best_keys():
+    """Packed (count << 40 | index) keys: min == lowest count, then lowest index; empty
+    shards never win; round trip."""
+    from paper_conf_ipps_binderlp19_b200.multigpu import pack_best, unpack_best
+    bc = torch.tensor([[5, 3, 0xFFFFFFFF, 4], [3, 3, 7, 4]], dtype=torch.int64)
+    bi = torch.tensor([[10, 11, -1, (1 << 39) + 5], [200, 201, 202, 6]], dtype=torch.int64)
+    k = pack_best(bc, bi)
+    c, i = unpack_best(k.min(dim=0).values)
+    assert c.tolist() == [3, 3, 7, 4] and i.tolist() == [200, 11, 202, 6]
+    c, i = unpack_best(pack_best(torch.tensor([0xFFFFFFFF]), torch.tensor([-1])))
+    assert c.tolist() == [0xFFFFFFFF] and i.tolist() == [-1]
+    u = torch.tensor([0x7FFFFF, 0], dtype=torch.int32).view(torch.uint32)   # uint32 counts
+    c, i = unpack_best(pack_best(u, torch.tensor([3, 4])))
+    assert c.tolist() == [0x7FFFFF, 0] and i.tolist() == [3, 4]
