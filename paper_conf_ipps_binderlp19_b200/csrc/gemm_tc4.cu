@@ -78,6 +78,7 @@ struct GArgs {
     int order;        // tile raster: 2 grouped (default), 1 lane-block-major, 0 column-block-major
     int off32;        // every output element offset (row * ldo + col) fits in 32 bits
     int sym;          // f3 symmetric self-LD: only tiles lb <= cb, off-diagonal ones mirrored
+    int v4;           // outputs 16-byte aligned with ldo % 4 == 0: vector copy-out
     int op2;          // EPI_COUNTS, swapped layout: second op written to C2 (or C2 = NULL)
     uint32_t *C2;
     const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
@@ -367,6 +368,75 @@ __device__ __forceinline__ void epi_ld_sym_fast(const GArgs &args, const uint32_
     }
 }
 
+
+// Full 32 x 32 LD block with a 16-byte-aligned output (32 valid columns, ldo % 4 == 0):
+// r2 is computed in the pre-transpose layout (lane = row i, u = column: the column terms are
+// shuffled), optionally stored mirrored (f3), and both r2 and the counts leave through the
+// transpose buffer with 16-byte copies: per warp instruction 4 rows x 128 bytes (one
+// LDS.128 + one STG.128 per 4 elements instead of one LDS + one STG per element).
+__device__ __forceinline__ void copy_out_v4(const uint32_t *tw, int lane, uint32_t *dst, uint32_t off0, uint32_t ld32) {
+    const int cchunk = lane & 7, rsub = lane >> 3;
+#pragma unroll
+    for (int it = 0; it < 8; ++it) {
+        const int r = 4 * it + rsub;
+        uint4 x = *reinterpret_cast<const uint4 *>(tw + r * 32 + ((cchunk ^ (r & 7)) << 2));
+        uint4 *d = reinterpret_cast<uint4 *>(dst + off0 + (uint32_t)r * ld32 + 4u * (uint32_t)cchunk);
+        __stcs(d, x);
+    }
+}
+__device__ __forceinline__ void epi_ld_fast_v4(const GArgs &args, const uint32_t (&c)[32], uint32_t *tw, int lane,
+                                               int64_t row0, int64_t col0, uint32_t pl, uint32_t pcol, float ia,
+                                               bool mirror) {
+    const int64_t ldo = args.ldo;
+    const int32_t n32 = (int32_t)args.nbits;
+    const uint32_t ld32 = (uint32_t)ldo;
+    float *const r2b = args.r2;
+    uint32_t *const cb = args.C;
+    const uint32_t has_c = cb != nullptr ? 1u : 0u;
+    const uint32_t off_n = (uint32_t)(row0 * ldo + col0);           // normal block origin
+    __syncwarp();   // the previous block's reads of tw are done
+    if (has_c) {    // counts: stage (row i = lane, chunks XOR-swizzled by row), copy out
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t a = ptx::smem_u32(tw + lane * 32 + ((k ^ (lane & 7)) << 2));
+            asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(c[4 * k]), "r"(c[4 * k + 1]),
+                         "r"(c[4 * k + 2]), "r"(c[4 * k + 3])
+                         : "memory");
+        }
+        __syncwarp();
+        copy_out_v4(tw, lane, cb, off_n, ld32);
+        __syncwarp();
+    }
+    const bool ok_i = row0 + lane < args.nl;
+    const float ibl = inv_exact((int64_t)pcol * ((int64_t)n32 - (int64_t)pcol));
+    const int32_t npl = -(int32_t)pl;
+    uint32_t offm = (uint32_t)(col0 * ldo + row0 + lane);           // mirror: row col0 + u
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        float r[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const int u = 4 * k + t;
+            const int32_t pb = (int32_t)__shfl_sync(0xffffffffu, pcol, u);
+            const float ib = __shfl_sync(0xffffffffu, ibl, u);
+            const int32_t num = n32 * (int32_t)c[u] + npl * pb;
+            const float fn = (float)num;
+            r[t] = fminf(__fmul_rn(__fmul_rn(fn, ia), __fmul_rn(fn, ib)), 1.0f);
+            if (mirror) {
+                const uint32_t ok = ok_i ? 1u : 0u;
+                st_cs_pred_f32(r2b + offm, r[t], ok);
+                st_cs_pred_u32(cb + offm, c[u], ok & has_c);
+                offm += ld32;
+            }
+        }
+        const uint32_t a = ptx::smem_u32(tw + lane * 32 + ((k ^ (lane & 7)) << 2));
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(r[0]), "f"(r[1]), "f"(r[2]), "f"(r[3])
+                     : "memory");
+    }
+    __syncwarp();
+    copy_out_v4(tw, lane, reinterpret_cast<uint32_t *>(r2b), off_n, ld32);
+}
+
 template <int EPI>
 __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[32], uint32_t *tw, int lane,
                                                int64_t row0, int64_t col0, uint32_t pl, uint32_t pcol, float ia,
@@ -374,6 +444,11 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
     const bool small = args.nbits < (1LL << 23);
 #pragma unroll
     for (int i = 0; i < 32; ++i) c[i] = acc_count(c[i], small);   // in place: c is the TMEM load
+    if (EPI == EPI_LD && small_n && !want_dp && args.off32 && args.v4 && args.nl - row0 >= 32 &&
+        args.nc - col0 >= 32) {
+        epi_ld_fast_v4(args, c, tw, lane, row0, col0, pl, pcol, ia, mirror);
+        return;
+    }
     if (EPI == EPI_LD && mirror && small_n && !want_dp && args.off32 && args.nl - row0 >= 32) {
         epi_ld_sym_fast(args, c, tw, lane, row0, col0, pl, pcol, ia);
         return;
@@ -1493,6 +1568,7 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
     g.debug_skip = skip ? 1 : 0;
     g.off32 = (uint64_t)(swap ? a.n : a.m) * (uint64_t)a.ldc < (1ull << 32) ? 1 : 0;
+    g.v4 = (a.ldc % 4 == 0 && ((uintptr_t)a.r2 & 15u) == 0 && ((uintptr_t)a.C & 15u) == 0) ? 1 : 0;
     // f3 symmetric self-LD (B aliases A, symmetric output: LD statistics, AND or XOR
     // counts): only the upper-triangle tiles are computed, off-diagonal ones mirrored.
     // SNP_GEMM_SYM=0 computes every tile.
