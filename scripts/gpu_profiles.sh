@@ -9,3 +9,5 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:fast
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:gemm_tc4 -s 2 -c 1 -o gpurun_out/prof/full_ld32k python bench.py --workload ld32k --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --no-graph > /dev/null 2>&1; echo ncu4=$?
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:bitgemm_popc -s 2 -c 1 -o gpurun_out/prof/full_fastid1m_popc python bench.py --variant popc --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --no-graph > /dev/null 2>&1; echo ncu5=$?
 ls -la gpurun_out/prof
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k "regex:pack_|popc|tc4|best_|bitgemm|fastid" -c 60 --csv --log-file gpurun_out/prof/launches_ld2k.csv python bench.py --workload ld2k --steps 3 --warmup 3 --no-cpu-baseline --no-e2e --no-graph > /dev/null 2>&1; echo ncu6=$?
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:gemm_tc4 -s 3 -c 1 -o gpurun_out/prof/full_ld2k python bench.py --workload ld2k --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --no-graph > /dev/null 2>&1; echo ncu7=$?

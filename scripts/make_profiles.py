@@ -52,14 +52,15 @@ tpath = os.path.join(ROOT, "profiles", "traffic.json")
 if os.path.exists(tpath):
     traffic = json.load(open(tpath))
 summary = []
-for wl, per_step in (("fastid1m", 9), ("ld32k", 4)):
+for wl, per_step in (("fastid1m", 9), ("ld32k", 4), ("ld2k", 3), ("fastid20m", 5)):
     p = os.path.join(SRC, f"launches_{wl}.csv")
     if os.path.exists(p):
         ks, tot, agg = launches(p, per_step, 2)
         summary.append(f"## launch list {wl} (ncu gpu__time_duration.sum, cold-cache serialised; last 2 steps, {len(ks)} launches)")
         for k, (n, v) in sorted(agg.items(), key=lambda x: -x[1][1]):
             summary.append(f"  {k:24s} launches {n:3d}  total {v / 1e3:10.1f} us  share {100 * v / tot:5.1f} %")
-for name, wl, kern in (("full_fastid1m", "fastid1m", "fastid_mxf4"), ("full_ld32k", "ld32k", "tc_mxf4"),
+for name, wl, kern in (("full_fastid1m", "fastid1m", "fastid_mxf4"), ("full_ld32k", "ld32k", "tc_mxf4_sym"),
+                       ("full_ld2k", "ld2k", "tc_mxf4"), ("full_fastid20m", "fastid20m", "tc_mxf4"),
                        ("full_fastid1m_popc", "fastid1m", "popc")):
     rep = os.path.join(SRC, name + ".ncu-rep")
     if not os.path.exists(rep):
