@@ -229,7 +229,36 @@ def cpu_baseline(wl, seconds, cores=None):
         cmp = rows * m * nbits
         sample = f"{rows} SNP rows x {m} SNPs x {nbits} samples, counts + r2 + D' (full workload: {m} rows)"
     return {"value": cmp / dt, "unit": "comparisons/s", "cores": cores, "kind": "oracle",
-            "sample": sample, "seconds": round(dt, 3)}
+            "sample": sample, "seconds": round(dt, 3), "host": host_popcount_peak(cores)}
+
+
+def host_popcount_peak(cores):
+    """The host's theoretical popcount throughput as the paper states it for CPUs
+    (cores x clock x bits per cycle): 64 bits/cycle/core with POPCNT, 512 with
+    AVX-512 VPOPCNTDQ.  Context for the oracle number, not a target."""
+    model, mhz, flags = "?", None, ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                k, _, v = line.partition(":")
+                k = k.strip()
+                if k == "model name" and model == "?":
+                    model = v.strip()
+                elif k == "cpu MHz" and mhz is None:
+                    mhz = float(v)
+                elif k == "flags" and not flags:
+                    flags = v
+    except OSError:
+        pass
+    try:
+        with open("/sys/devices/system/cpu/cpu0/cpufreq/cpuinfo_max_freq") as f:
+            mhz = int(f.read()) / 1e3
+    except (OSError, ValueError):
+        pass
+    bits = 512 if "avx512_vpopcntdq" in flags.split() else 64
+    peak = cores * (mhz or 0) * 1e6 * bits
+    return {"model": model, "mhz": mhz, "popcount_bits_per_cycle": bits,
+            "theoretical_cmp_per_s": peak, "oracle_note": "the oracle is plain bit-by-bit C (not tuned)"}
 
 
 # ----------------------------------------------------------------------------- workloads

@@ -552,3 +552,32 @@ def test_search_general_kernel_forced(snp, monkeypatch):
         assert np.array_equal(u32(counts[j]), ref), op
         rb, ri = oracle.best(ref, 3)
         assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), op
+
+
+def test_cfg4_fastid_20m_full_size():
+    """configs[3] at full size on one GPU (1,024 queries x 20,000,000 profiles x 8,192
+    SNPs, the launch configuration bench.py times for the best matches): planted identity
+    copies are found (best count <= flips at the planted row, which at these sizes no other
+    row approaches), every best index is in range, and a 1M-row database slice of the XOR /
+    ANDNOT counts matches the oracle on sampled rows."""
+    import paper_conf_ipps_binderlp19_b200 as snpm
+    nq, nd, nbits, seed = 1024, 20_000_000, 8192, 1004
+    D = _gen_dev_fastid(seed, nd, nbits, chunk=262144)
+    q, plan = snpgen.fastid_queries(seed, nq, nd, nbits)
+    Q = snpm.snp_pack(to_dev(q))
+    _, best = snpm.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=False)
+    bx, ix = u32(best[0][0]), best[0][1].cpu().numpy()
+    assert ((ix >= 0) & (ix < nd)).all()
+    for qi, (kind, js, flips) in enumerate(plan):
+        if kind == "copy":
+            assert bx[qi] <= len(flips) and ix[qi] == js[0], (qi, bx[qi], ix[qi], js)
+    # counts on a slice of the database: all queries x rows [r0, r0 + 1M), sampled rows
+    r0 = 7_000_000
+    Dsl = D[r0:r0 + 1_000_000]
+    cols = _sample_cols(1_000_000, 128, 200, 11)
+    dbs = snpgen.fastid_db(seed, cols + r0, nbits)
+    for op in ("xor", "andnot"):
+        out = snpm.snp_fastid(Q, Dsl, nbits, op)
+        got = u32(out.view(torch.int32)[:, torch.from_numpy(cols).to(DEV)])
+        assert np.array_equal(got, oracle.counts(q, dbs, op)), op
+        del out
