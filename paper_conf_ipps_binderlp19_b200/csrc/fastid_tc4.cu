@@ -363,14 +363,20 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         uint32_t pround = 0, bround = 0;
         for (int64_t it = g; it < total_it; it += G) {
             publish_until(tl);
+#if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             const bool tr = args.trace && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
+#endif
+#if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 0] = clock64();
+#endif
             ptx::mbar_wait_warp(&pfull[p], pround & 1);
 #ifdef FASTID_TRACE2
             if (tr) g_fastid_trace[8 * it + 4] = clock64();
 #endif
             if (bround > 0) ptx::mbar_wait_warp(&empty[b], (bround - 1) & 1);
+#if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 1] = clock64();
+#endif
             // 64-byte row of the stage; TMA 64B swizzle: 16-byte chunk c of row r sits at
             // chunk c ^ ((r >> 1) & 3)  (conflict-free LDS.128 across the warp)
             const uint8_t *src = ring + p * PSTAGE + arow * 64;
@@ -404,7 +410,9 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             ptx::tmem_st_wait();
             ptx::tc_fence_before();
             __syncwarp();
+#if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 2] = clock64();
+#endif
             if (lane == 0) ptx::mbar_arrive(&full[b]);
             s += G;
             while (s >= nst) { s -= nst; ++tl; }

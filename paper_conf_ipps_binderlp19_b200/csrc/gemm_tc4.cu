@@ -74,7 +74,8 @@ struct GArgs {
     int64_t nlb, ncb;
     int nst;
     int trace;
-    int debug_skip;   // profiling experiment: expanders only pass tokens (results invalid)
+    int debug_skip;   // profiling experiment (build with -DGEMM_DEBUG_SKIP): expanders only pass
+                      // tokens, results invalid
     int order;        // tile raster: 2 grouped (default), 1 lane-block-major, 0 column-block-major
     int off32;        // every output element offset (row * ldo + col) fits in 32 bits
     int sym;          // f3 symmetric self-LD: only tiles lb <= cb, off-diagonal ones mirrored
@@ -800,14 +801,21 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         int pk = g;                                     // packed slot (group g: g, g + G, ...)
         uint32_t pround = 0;
         for (int64_t it = g; it < total_it; it += G) {
+#ifdef GEMM_TRACE
             const bool tr = args.trace && blockIdx.x == 0 && r8 == 0 && lane == 0 && it < 2048;
+#endif
+#ifdef GEMM_TRACE
             if (tr) g_gemm_trace[8 * it + 0] = clock64();
+#endif
             // empty BEFORE pfull: both groups share the slots, so a warp may reach use u+2 of
             // a slot while its pfull barrier is only at phase u+1; waiting for the MMA to
             // release use u+1 first rules out parity aliasing on pfull (same parity as u)
             if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
             ptx::mbar_wait_warp(&pfull[pk], pround & 1);
+#ifdef GEMM_TRACE
             if (tr) g_gemm_trace[8 * it + 1] = clock64();
+#endif
+#ifdef GEMM_DEBUG_SKIP
             if (args.debug_skip) {
                 __syncwarp();
                 if (lane == 0) { ptx::mbar_arrive(&pempty[pk]); ptx::mbar_arrive(&full[slot]); }
@@ -819,6 +827,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 if (pk >= NP) { pk -= NP; ++pround; }
                 continue;
             }
+#endif
             const uint8_t *src = ring + pk * PSLOT + (is_a ? 0 : BM * PROW) + row * PROW;
             uint32_t w[KW];
 #pragma unroll
@@ -826,7 +835,9 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 const uint4 x = *reinterpret_cast<const uint4 *>(src + ((c ^ sw) << 4));
                 w[4 * c] = x.x; w[4 * c + 1] = x.y; w[4 * c + 2] = x.z; w[4 * c + 3] = x.w;
             }
+#ifdef GEMM_TRACE
             if (tr) g_gemm_trace[8 * it + 2] = clock64();
+#endif
             const int64_t w0 = (int64_t)s * KW;
             if (w0 + KW > full32) {
 #pragma unroll
@@ -862,7 +873,9 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 ptx::mbar_arrive(&pempty[pk]);
                 ptx::mbar_arrive(&full[slot]);
             }
+#ifdef GEMM_TRACE
             if (tr) g_gemm_trace[8 * it + 3] = clock64();
+#endif
             s += G;
             while (s >= nst) { s -= nst; ++tl; }
             slot += G;
@@ -1297,6 +1310,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
         for (int64_t it = g; it < total_it; it += G) {
             if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
             ptx::mbar_wait_warp(&pfull[pk], pround & 1);
+#ifdef GEMM_DEBUG_SKIP
             if (args.debug_skip) {   // profiling experiment: tokens only (results invalid)
                 __syncwarp();
                 if (lane == 0) { ptx::mbar_arrive(&pempty[pk]); arrive_remote(&full[slot], 0); }
@@ -1308,6 +1322,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
                 if (pk >= NP) { pk -= NP; ++pround; }
                 continue;
             }
+#endif
             const uint8_t *src = ring + pk * PSLOT + (is_a ? 0 : BM * PROW) + row * PROW;
             uint32_t w[KW];
 #pragma unroll
