@@ -581,3 +581,35 @@ def test_cfg4_fastid_20m_full_size():
         got = u32(out.view(torch.int32)[:, torch.from_numpy(cols).to(DEV)])
         assert np.array_equal(got, oracle.counts(q, dbs, op)), op
         del out
+
+
+def test_fuzz_shapes(snp):
+    """Seeded random shapes through every dispatch path (fused / sliced / general search,
+    f3 symmetric and full-tile LD, swapped and unswapped layouts) vs the oracle."""
+    rng = np.random.default_rng(2024)
+    cases = [(int(rng.integers(1, 200)), int(rng.integers(256, 4000)), int(rng.integers(1, 5000)))
+             for _ in range(8)]
+    for nq, nd, nbits in cases:
+        db = snpgen.fastid_db(91, np.arange(nd), nbits)
+        q, _ = snpgen.fastid_queries(91, nq, nd, nbits)
+        counts, best = snp.snp_fastid_search(pack_dev(snp, q, garbage_seed=1), pack_dev(snp, db, garbage_seed=2),
+                                             nbits, ("xor", "andnot"), index_base=5)
+        for j, op in enumerate(("xor", "andnot")):
+            ref = oracle.counts(q, db, op)
+            assert np.array_equal(u32(counts[j]), ref), (nq, nd, nbits, op)
+            rb, ri = oracle.best(ref, 5)
+            assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), \
+                (nq, nd, nbits, op)
+    for m, n, nbits, self_ld in [(2200, 2200, 97, True), (2400, 2400, 33, True), (700, 300, 1300, False),
+                                 (300, 700, 64, False), (1, 1, 1, True), (130, 130, 5000, True)]:
+        ga = snpgen.ld_genotypes(92, np.arange(m), nbits, structure=True)
+        gb = ga if self_ld else snpgen.ld_genotypes(93, np.arange(n), nbits, structure=True)
+        A = pack_dev(snp, ga, garbage_seed=3)
+        B = A if self_ld else pack_dev(snp, gb, garbage_seed=4)
+        r2, dp, cnt = snp.snp_ld_r2(A, B, nbits, dprime=True, counts=True)
+        r2_ref, dp_ref, n_ref = oracle.ld(ga, gb)
+        assert np.array_equal(u32(cnt), n_ref), (m, n, nbits)
+        check_r2(r2.cpu().numpy(), r2_ref)
+        check_r2(dp.cpu().numpy(), dp_ref)
+        r2b, _, _ = snp.snp_ld_r2(A, B, nbits)                 # r2 only (no counts / D')
+        check_r2(r2b.cpu().numpy(), r2_ref)
