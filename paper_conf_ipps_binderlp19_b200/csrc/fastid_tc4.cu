@@ -39,8 +39,13 @@ __device__ unsigned int g_fastid_launch_ctr;   // per CTA: start, main loop star
 namespace {
 
 constexpr int BM = 128;
-constexpr int KBITS = 512;
-static_assert(KBITS == 512, "a stage is exactly the 8 K=64 MMAs of mma8_mxf4_ts_commit");
+#ifndef FASTID_KBITS
+#define FASTID_KBITS 512
+#endif
+constexpr int KBITS = FASTID_KBITS;     // bits per stage: 512 (64-byte rows) or 256 (32-byte rows)
+static_assert(KBITS == 512 || KBITS == 256, "stage size");
+constexpr int KW = KBITS / 32;          // packed words per row per stage
+constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 #ifndef FASTID_NP
 #define FASTID_NP 8
 #endif
@@ -48,7 +53,8 @@ static_assert(KBITS == 512, "a stage is exactly the 8 K=64 MMAs of mma8_mxf4_ts_
 #define FASTID_NS 4
 #endif
 constexpr int NP = FASTID_NP;           // packed TMA ring depth (64 KB in flight per SM)
-constexpr int PSTAGE = BM * KBITS / 8;  // 8 KB packed per stage, 64-byte rows, 64B-swizzled
+constexpr int PSTAGE = BM * KBITS / 8;  // packed per stage (8 KB: 64-byte rows, 64B swizzle;
+                                        // 4 KB: 32-byte rows, 32B swizzle)
 #ifndef FASTID_G
 #define FASTID_G 4
 #endif
@@ -83,7 +89,7 @@ struct FCfg {
     static_assert(NS % 4 == 0 && NP % 4 == 0, "rings must be multiples of the group count");
     static constexpr int ACC_COLS = BN;
     static constexpr int A_COL0 = 2 * ACC_COLS;
-    static constexpr int SF_COL = A_COL0 + NS * 64;
+    static constexpr int SF_COL = A_COL0 + NS * ACOLS;
     static_assert(SF_COL + 32 <= 512, "TMEM budget");
 };
 
@@ -379,28 +385,29 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #endif
             // 64-byte row of the stage; TMA 64B swizzle: 16-byte chunk c of row r sits at
             // chunk c ^ ((r >> 1) & 3)  (conflict-free LDS.128 across the warp)
-            const uint8_t *src = ring + p * PSTAGE + arow * 64;
-            const int sw = (arow >> 1) & 3;
-            uint32_t wv[16];
+            // (32-byte rows, 32B swizzle: chunk c of row r sits at c ^ ((r >> 2) & 1))
+            const uint8_t *src = ring + p * PSTAGE + arow * (KBITS / 8);
+            const int sw = KBITS == 512 ? (arow >> 1) & 3 : (arow >> 2) & 1;
+            uint32_t wv[KW];
 #pragma unroll
-            for (int c = 0; c < 4; ++c) {
+            for (int c = 0; c < KW / 4; ++c) {
                 const uint4 x = *reinterpret_cast<const uint4 *>(src + ((c ^ sw) << 4));
                 wv[4 * c] = x.x; wv[4 * c + 1] = x.y; wv[4 * c + 2] = x.z; wv[4 * c + 3] = x.w;
             }
-            const int64_t w0 = (int64_t)s * (KBITS / 32);
-            if (w0 + 16 > full32) {
+            const int64_t w0 = (int64_t)s * KW;
+            if (w0 + KW > full32) {
 #pragma unroll
-                for (int i = 0; i < 16; ++i) wv[i] &= word_mask(w0 + i, nbits);
+                for (int i = 0; i < KW; ++i) wv[i] &= word_mask(w0 + i, nbits);
             }
             if (!pre) {
 #pragma unroll
-                for (int i = 0; i < 16; ++i) popa += __popc(wv[i]);
+                for (int i = 0; i < KW; ++i) popa += __popc(wv[i]);
             }
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&pempty[p]);
-            const uint32_t tbase = tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + 64 * b);
+            const uint32_t tbase = tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + ACOLS * b);
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
+            for (int h = 0; h < KW / 8; ++h) {
                 uint32_t v[32];
 #pragma unroll
                 for (int i = 0; i < 8; ++i)
@@ -460,7 +467,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #ifdef FASTID_TRACE2
                 if (args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 5] = clock64();
 #endif
-                const uint32_t a0 = tmu + (uint32_t)(C::A_COL0 + 64 * b);
+                const uint32_t a0 = tmu + (uint32_t)(C::A_COL0 + ACOLS * b);
 #pragma unroll
                 for (int k = 0; k < KBITS / 64; ++k)
                     ptx::mma_mxf4_ts(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa,
@@ -720,7 +727,8 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     const cuuint32_t box[2] = {KBITS / 32, BM};
     const cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(a.D), dims, strides, box, estr,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, KBITS == 512 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
 
