@@ -1586,13 +1586,12 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.v4 = (a.ldc % 4 == 0 && ((uintptr_t)a.r2 & 15u) == 0 && ((uintptr_t)a.C & 15u) == 0) ? 1 : 0;
     // f3 symmetric self-LD (B aliases A, symmetric output: LD statistics, AND or XOR
     // counts): only the upper-triangle tiles are computed, off-diagonal ones mirrored.
-    // SNP_GEMM_SYM=0 computes every tile.
+    // With the vectorised mirror epilogue this wins from two tile rows up (LD-2K 41.6 ->
+    // 35.5 us, LD-32K 7.1 -> 4.0 ms).  SNP_GEMM_SYM=0 computes every tile.
     static const char *syme = std::getenv("SNP_GEMM_SYM");
-    // Only with at least two waves of full tiles: below that the doubled epilogue of the
-    // mirrored tiles is exposed (LD-2K: 256 tiles, 37 us full vs 46 us triangle).
     const int64_t full_tiles = ((a.m + BM - 1) / BM) * ((a.n + BN - 1) / BN);
     g.sym = (!swap && a.A == a.B && a.m == a.n && a.lda32 == a.ldb32 && (epi == EPI_LD || a.op <= 1) &&
-             full_tiles > 2 * num_sms() && !(syme && syme[0] == '0')) ? 1 : 0;
+             full_tiles > 1 && !(syme && syme[0] == '0')) ? 1 : 0;
     static const char *ord = std::getenv("SNP_GEMM_ORDER");
     g.order = ord ? (ord[0] - '0') : 2;
     // CTA-pair kernel: opt-in (SNP_GEMM_X2=1) for the unswapped shapes with more than one

@@ -501,11 +501,11 @@ print("ok")
     assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
 
 
-@pytest.mark.parametrize("m,nbits", [(2300, 1025), (2200, 64)])
+@pytest.mark.parametrize("m,nbits", [(2300, 1025), (2200, 64), (300, 1025), (129, 64), (1000, 700)])
 def test_selfld_symmetric_mirror(snp, m, nbits):
     """f3: self-LD (B aliases A) computes only the upper-triangle tiles and mirrors the
-    off-diagonal ones (used from > 2 waves of tiles: m >= 2177 here, ragged last tile);
-    every output (counts, r2, D') vs the oracle, and the matrices are exactly symmetric."""
+    off-diagonal ones (from two tile rows up, ragged last tile here); every output
+    (counts, r2, D') vs the oracle, and the matrices are exactly symmetric."""
     g = snpgen.ld_genotypes(61, np.arange(m), nbits, structure=True)
     A = pack_dev(snp, g, garbage_seed=9)
     r2, dp, cnt = snp.snp_ld_r2(A, A, nbits, dprime=True, counts=True)
