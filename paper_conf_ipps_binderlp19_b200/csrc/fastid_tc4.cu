@@ -350,9 +350,9 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         const int g = warp >> 2, qa = warp & 3;
         const int arow = qa * 32 + lane;
         uint32_t popa = 0;
-        int64_t cur_tl = 0;   // tile whose popcount partial is being accumulated
+        int cur_tl = 0;       // tile whose popcount partial is being accumulated
         const bool pre = args.popDg != nullptr;
-        auto publish_until = [&](int64_t upto) {
+        auto publish_until = [&](int upto) {
             if (pre) return;
             for (; cur_tl < upto; ++cur_tl) {
                 const int acc = (int)(cur_tl & 1);
@@ -363,11 +363,14 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 if (lane == 0) ptx::mbar_arrive(&popf[acc]);
             }
         };
-        int64_t tl = g / nst;
+        // 32-bit loop state (total_it < 2^31: fastid_tc4_supported bounds nd): the loop
+        // bookkeeping is a visible share of the expander instruction stream
+        int tl = g / nst;
         int s = g % nst;
         int p = g, b = g;
         uint32_t pround = 0, bround = 0;
-        for (int64_t it = g; it < total_it; it += G) {
+        const int total_it32 = (int)total_it;
+        for (int it = g; it < total_it32; it += G) {
             publish_until(tl);
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             const bool tr = args.trace && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
@@ -428,7 +431,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             b += G;
             if (b >= NS) { b -= NS; ++bround; }
         }
-        publish_until(my_tiles);
+        publish_until((int)my_tiles);
     } else if (warp == MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
         // The whole warp runs the loop (converged, uniform values); the elected lane issues.
