@@ -613,3 +613,26 @@ def test_fuzz_shapes(snp):
         check_r2(dp.cpu().numpy(), dp_ref)
         r2b, _, _ = snp.snp_ld_r2(A, B, nbits)                 # r2 only (no counts / D')
         check_r2(r2b.cpu().numpy(), r2_ref)
+
+
+@pytest.mark.parametrize("self_ld", [True, False])
+def test_ld_unaligned_output_rows(snp, self_ld):
+    """Output row strides that are not a multiple of 4 words (no 16-byte row copies): the
+    scalar full-block and mirror epilogues, counts + r2 + D' and counts + r2, vs the oracle."""
+    m, nbits = 300, 1025
+    ga = snpgen.ld_genotypes(95, np.arange(m), nbits, structure=True)
+    gb = ga if self_ld else snpgen.ld_genotypes(96, np.arange(m), nbits, structure=True)
+    A = pack_dev(snp, ga)
+    B = A if self_ld else pack_dev(snp, gb)
+    r2_ref, dp_ref, n_ref = oracle.ld(ga, gb)
+    for ld in (m + 2, m + 3):
+        for want_dp in (True, False):
+            r2b = torch.full((m, ld), -1.0, dtype=torch.float32, device=DEV)
+            cb = torch.zeros((m, ld), dtype=torch.int32, device=DEV).view(torch.uint32)
+            dpb = torch.full((m, ld), -2.0, dtype=torch.float32, device=DEV) if want_dp else None
+            snp.snp_ld_r2(A, B, nbits, r2=r2b[:, :m], counts=cb[:, :m], dprime=None if dpb is None else dpb[:, :m])
+            assert np.array_equal(u32(cb)[:, :m], n_ref), (ld, want_dp)
+            check_r2(r2b[:, :m].cpu().numpy(), r2_ref)
+            assert (r2b[:, m:].cpu().numpy() == -1.0).all()
+            if dpb is not None:
+                check_r2(dpb[:, :m].cpu().numpy(), dp_ref)
