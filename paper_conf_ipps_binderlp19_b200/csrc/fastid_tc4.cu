@@ -52,6 +52,10 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 #ifndef FASTID_NS
 #define FASTID_NS 4
 #endif
+#ifndef FASTID_NACC
+#define FASTID_NACC 2   // TMEM accumulators (the MMA may run NACC - 1 tiles ahead of the epilogue)
+#endif
+constexpr int NACC = FASTID_NACC;
 constexpr int NP = FASTID_NP;           // packed TMA ring depth (64 KB in flight per SM)
 constexpr int PSTAGE = BM * KBITS / 8;  // packed per stage (8 KB: 64-byte rows, 64B swizzle;
                                         // 4 KB: 32-byte rows, 32B swizzle)
@@ -88,7 +92,7 @@ struct FCfg {
     static constexpr int NS = FASTID_NS;            // TMEM A stages of 64 columns (multiple of G)
     static_assert(NS % 4 == 0 && NP % 4 == 0, "rings must be multiples of the group count");
     static constexpr int ACC_COLS = BN;
-    static constexpr int A_COL0 = 2 * ACC_COLS;
+    static constexpr int A_COL0 = NACC * ACC_COLS;
     static constexpr int SF_COL = A_COL0 + NS * ACOLS;
     static_assert(SF_COL + 32 <= 512, "TMEM budget");
 };
@@ -231,13 +235,13 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     uint64_t *pempty = pfull + NP;           // [NP] expanders -> TMA
     uint64_t *full = pempty + NP;            // [NS] expanders -> MMA
     uint64_t *empty = full + NS;             // [NS] MMA -> expanders
-    uint64_t *accf = empty + NS;             // [2]
-    uint64_t *acce = accf + 2;               // [2]
-    uint64_t *popf = acce + 2;               // [2]
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popf + 2);
+    uint64_t *accf = empty + NS;             // [NACC]
+    uint64_t *acce = accf + NACC;            // [NACC]
+    uint64_t *popf = acce + NACC;            // [NACC]
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popf + NACC);
     uint32_t *popQ = tmem_slot + 4;          // [BN]
     uint32_t *popD = popQ + BN;              // [2 acc][G][BM]
-    uint32_t *popQ32 = popD + 2 * G * BM;    // [BN] 32 * popQ (epilogue key term)
+    uint32_t *popQ32 = popD + NACC * G * BM; // [BN] 32 * popQ (epilogue key term)
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     __shared__ unsigned int launch_k;
@@ -261,7 +265,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             ptx::mbar_init(&full[i], 4);
             ptx::mbar_init(&empty[i], 1);
         }
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < NACC; ++i) {
             ptx::mbar_init(&accf[i], 1);
             ptx::mbar_init(&acce[i], NEPI);
             ptx::mbar_init(&popf[i], NEXP);
@@ -355,8 +359,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         auto publish_until = [&](int upto) {
             if (pre) return;
             for (; cur_tl < upto; ++cur_tl) {
-                const int acc = (int)(cur_tl & 1);
-                if (cur_tl >= 2) ptx::mbar_wait_warp(&acce[acc], (uint32_t)(((cur_tl >> 1) - 1) & 1));
+                const int acc = cur_tl % NACC;
+                if (cur_tl >= NACC) ptx::mbar_wait_warp(&acce[acc], (uint32_t)((cur_tl / NACC - 1) & 1));
                 popD[(acc * G + g) * BM + arow] = popa;
                 popa = 0;
                 __syncwarp();
@@ -450,11 +454,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         uint32_t bround = 0;
         int64_t itm = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
-            const int acc = (int)(tl & 1);
+            const uint32_t tl32 = (uint32_t)tl;
+            const int acc = (int)(tl32 % NACC);
 #ifdef FASTID_TRACE2
             if (args.trace && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 0] = clock64();
 #endif
-            if (tl >= 2) ptx::mbar_wait_uniform(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+            if (tl32 >= NACC) ptx::mbar_wait_uniform(&acce[acc], (tl32 / NACC - 1) & 1u);
 #ifdef FASTID_TRACE2
             if (args.trace && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 1] = clock64();
 #endif
@@ -498,8 +503,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #pragma unroll
         for (int j = 0; j < NOPS; ++j) { bc[j] = 0xffffffffu; bi[j] = 0xffffffffu; }
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
-            const int acc = (int)(tl & 1);
-            const uint32_t ph = (uint32_t)((tl >> 1) & 1);
+            const int acc = (int)((uint32_t)tl % NACC);
+            const uint32_t ph = ((uint32_t)tl / NACC) & 1u;
             const int64_t t = blockIdx.x + tl * gridDim.x;
             const bool pre = args.popDg != nullptr;
             const int64_t gd_l = t * BM + li;   // this lane's local database row
