@@ -52,7 +52,7 @@ tpath = os.path.join(ROOT, "profiles", "traffic.json")
 if os.path.exists(tpath):
     traffic = json.load(open(tpath))
 summary = []
-for wl, per_step in (("fastid1m", 9), ("ld32k", 4), ("ld2k", 3), ("fastid20m", 5)):
+for wl, per_step in (("fastid1m", 3), ("ld32k", 3), ("ld2k", 3), ("fastid20m", 6)):
     p = os.path.join(SRC, f"launches_{wl}.csv")
     if os.path.exists(p):
         ks, tot, agg = launches(p, per_step, 2)
