@@ -52,6 +52,12 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 #ifndef FASTID_NS
 #define FASTID_NS 4
 #endif
+// Per-half-stage full barriers (the MMA starts on the first 256 bits while the expanders
+// write the second half): measured on FastID-1M, 207 -> 195 us with 4 expander groups
+// (popcounts counted in-kernel) but 185 -> 191 us with 2 groups, so only for GG = 4.
+#ifndef FASTID_HALF
+#define FASTID_HALF 4   // the GG that uses half-stage barriers (0: none)
+#endif
 #ifndef FASTID_NACC
 #define FASTID_NACC 2   // TMEM accumulators (the MMA may run NACC - 1 tiles ahead of the epilogue)
 #endif
@@ -225,6 +231,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     constexpr int G = GG, NEXP = Roles<GG>::NEXP, EPI_WARP0 = Roles<GG>::EPI_WARP0;
     constexpr int TMA_WARP = Roles<GG>::TMA_WARP, MMA_WARP = Roles<GG>::MMA_WARP;
     constexpr int NTHREADS = Roles<GG>::NTHREADS, NEPI = Roles<GG>::NEPI;
+    constexpr int NHALF = (GG == FASTID_HALF && KBITS == 512) ? 2 : 1;
     using C = FCfg<BN>;
     constexpr int NS = C::NS;
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -233,8 +240,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     uint64_t *bars = reinterpret_cast<uint64_t *>(ring + NP * PSTAGE);
     uint64_t *pfull = bars;                  // [NP] TMA -> expanders
     uint64_t *pempty = pfull + NP;           // [NP] expanders -> TMA
-    uint64_t *full = pempty + NP;            // [NS] expanders -> MMA
-    uint64_t *empty = full + NS;             // [NS] MMA -> expanders
+    uint64_t *full = pempty + NP;            // [NS][NHALF] expanders -> MMA
+    uint64_t *empty = full + NS * NHALF;     // [NS] MMA -> expanders
     uint64_t *accf = empty + NS;             // [NACC]
     uint64_t *acce = accf + NACC;            // [NACC]
     uint64_t *popf = acce + NACC;            // [NACC]
@@ -262,7 +269,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             ptx::mbar_init(&pempty[i], 4);
         }
         for (int i = 0; i < NS; ++i) {
-            ptx::mbar_init(&full[i], 4);
+            for (int h = 0; h < NHALF; ++h) ptx::mbar_init(&full[i * NHALF + h], 4);
             ptx::mbar_init(&empty[i], 1);
         }
         for (int i = 0; i < NACC; ++i) {
@@ -420,6 +427,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 for (int i = 0; i < 8; ++i)
                     expandA(wv[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
                 tmem_st32(tbase + 32 * h, v);
+                if (NHALF == 2 && h == 0) {   // publish the first half: the MMA may start on it
+                    ptx::tmem_st_wait();
+                    ptx::tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) ptx::mbar_arrive(&full[b * NHALF]);
+                }
             }
             ptx::tmem_st_wait();
             ptx::tc_fence_before();
@@ -427,7 +440,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 2] = clock64();
 #endif
-            if (lane == 0) ptx::mbar_arrive(&full[b]);
+            if (lane == 0) ptx::mbar_arrive(&full[b * NHALF + NHALF - 1]);
             s += G;
             while (s >= nst) { s -= nst; ++tl; }
             p += G;
@@ -470,16 +483,21 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #ifdef FASTID_TRACE2
                 if (args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 3] = clock64();
 #endif
-                ptx::mbar_wait_uniform(&full[b], bround & 1);
+                ptx::mbar_wait_uniform(&full[b * NHALF], bround & 1);
                 ptx::tc_fence_after();
 #ifdef FASTID_TRACE2
                 if (args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 5] = clock64();
 #endif
                 const uint32_t a0 = tmu + (uint32_t)(C::A_COL0 + ACOLS * b);
 #pragma unroll
-                for (int k = 0; k < KBITS / 64; ++k)
+                for (int k = 0; k < KBITS / 64; ++k) {
+                    if (NHALF == 2 && k == KBITS / 128) {   // second half of the stage
+                        ptx::mbar_wait_uniform(&full[b * NHALF + 1], bround & 1);
+                        ptx::tc_fence_after();
+                    }
                     ptx::mma_mxf4_ts(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa,
                                      sfb);
+                }
                 ptx::mma_commit_uniform(&empty[b]);
                 bd += SSTEP;
                 if (++b == NS) { b = 0; ++bround; }
