@@ -43,6 +43,10 @@ constexpr int NS = 3;                          // expanded slots (TMEM A stage +
 #define GEMM_NP 6
 #endif
 constexpr int NP = GEMM_NP;                    // packed TMA ring: NP x 16 KB in flight per SM
+#ifndef GEMM_HALF
+#define GEMM_HALF 0
+#endif
+constexpr int GH = GEMM_HALF ? 2 : 1;          // full barriers per stage (half-stage publishing)
                                                // (3 slots left the expanders waiting on L2)
 #ifndef GEMM_G
 #define GEMM_G 2
@@ -653,8 +657,8 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     uint64_t *bars = reinterpret_cast<uint64_t *>(trs + NEPI * 32 * 32);
     uint64_t *pfull = bars;            // [NP] TMA -> expanders
     uint64_t *pempty = pfull + NP;     // [NP] expanders -> TMA
-    uint64_t *full = pempty + NP;      // [NS] expanders -> MMA
-    uint64_t *empty = full + NS;       // [NS] MMA -> expanders
+    uint64_t *full = pempty + NP;      // [NS][GH] expanders -> MMA
+    uint64_t *empty = full + NS * GH;  // [NS] MMA -> expanders
     uint64_t *accf = empty + NS;       // [2]
     uint64_t *acce = accf + 2;         // [2]
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acce + 2);
@@ -727,7 +731,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             ptx::mbar_init(&pempty[i], 8);
         }
         for (int i = 0; i < NS; ++i) {
-            ptx::mbar_init(&full[i], 8);
+            for (int h = 0; h < GH; ++h) ptx::mbar_init(&full[i * GH + h], 8);
             ptx::mbar_init(&empty[i], 1);
         }
         for (int i = 0; i < 2; ++i) {
@@ -818,7 +822,10 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
 #ifdef GEMM_DEBUG_SKIP
             if (args.debug_skip) {
                 __syncwarp();
-                if (lane == 0) { ptx::mbar_arrive(&pempty[pk]); ptx::mbar_arrive(&full[slot]); }
+                if (lane == 0) {
+                    ptx::mbar_arrive(&pempty[pk]);
+                    for (int h = 0; h < GH; ++h) ptx::mbar_arrive(&full[slot * GH + h]);
+                }
                 s += G;
                 while (s >= nst) { s -= nst; ++tl; }
                 slot += G;
@@ -852,6 +859,12 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                     for (int i = 0; i < 8; ++i)
                         expandA(w[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
                     tmem_st32(tA + 32 * h, v);
+                    if (GH == 2 && h == 0) {   // publish the first 256 bits
+                        ptx::tmem_st_wait();
+                        ptx::tc_fence_before();
+                        __syncwarp();
+                        if (lane == 0) ptx::mbar_arrive(&full[slot * GH]);
+                    }
                 }
                 ptx::tmem_st_wait();
                 ptx::tc_fence_before();
@@ -862,6 +875,11 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                     uint4 o;
                     expandB(w[i], o.x, o.y, o.z, o.w);
                     *reinterpret_cast<uint4 *>(dstB + (size_t)i * BN * 16) = o;
+                    if (GH == 2 && i == KW / 2 - 1) {   // publish the first 256 bits
+                        ptx::fence_proxy_async_smem();
+                        __syncwarp();
+                        if (lane == 0) ptx::mbar_arrive(&full[slot * GH]);
+                    }
                 }
                 ptx::fence_proxy_async_smem();
             }
@@ -871,7 +889,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 // (an arrive right after the loads could let the next TMA overwrite data
                 // that is still in flight to registers)
                 ptx::mbar_arrive(&pempty[pk]);
-                ptx::mbar_arrive(&full[slot]);
+                ptx::mbar_arrive(&full[slot * GH + GH - 1]);
             }
 #ifdef GEMM_TRACE
             if (tr) g_gemm_trace[8 * it + 3] = clock64();
@@ -900,13 +918,18 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             ptx::tc_fence_after();
             const uint32_t d = tmu + (uint32_t)(acc * ACC_COLS);
             for (int s = 0; s < nst; ++s) {
-                ptx::mbar_wait_uniform(&full[b], round & 1);
+                ptx::mbar_wait_uniform(&full[b * GH], round & 1);
                 ptx::tc_fence_after();
                 const uint32_t a0 = tmu + (uint32_t)(A_COL0 + 64 * b);
                 const uint64_t b0 = bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4);
 #pragma unroll
-                for (int k = 0; k < KBITS / 64; ++k)
+                for (int k = 0; k < KBITS / 64; ++k) {
+                    if (GH == 2 && k == KBITS / 128) {
+                        ptx::mbar_wait_uniform(&full[b * GH + 1], round & 1);
+                        ptx::tc_fence_after();
+                    }
                     ptx::mma_mxf4_ts(d, a0 + 8 * k, b0 + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                }
                 ptx::mma_commit_uniform(&empty[b]);
                 if (++b == NS) { b = 0; ++round; }
             }
