@@ -828,12 +828,22 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
 
 // Shape filter: queries on the column side (<= 128 rows, the user's first operand),
 // their whole expanded K range resident in shared memory, exact fp32 range.
+// Resident query width: 64 columns while the expanded batch fits in shared memory (up to
+// ~6500 SNPs), else 32 (N = 32 MMAs, up to ~9700 SNPs) for batches of <= 32 queries
+// (configs[4] sweep: 1..32 queries x 20M x 8192 SNPs took the general kernel + best pass
+// at 9-12 ms against a 3.1 ms database read).
+int fastid_bn(int64_t m, int64_t nbits) {
+    if (m <= 64 && smem_bytes(64, nbits) <= MAX_SMEM - 1024) return 64;
+    if (m <= 32 && smem_bytes(32, nbits) <= MAX_SMEM - 1024) return 32;
+    return 0;
+}
+
 bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
     // nbits < 2^23: counts leave the fp32 accumulator by the 2^23 magic add
     if (m < 1 || m > 64 || n < 1 || nbits < 1 || nbits >= (1LL << 23)) return false;
     if (n < 4 * m) return false;
     if (n > (int64_t)0x7fffffff - BM) return false;
-    return smem_bytes(64, nbits) <= MAX_SMEM - 1024;
+    return fastid_bn(m, nbits) != 0;
 }
 
 cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
@@ -846,6 +856,7 @@ cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     sa.nops = 1; sa.ops[0] = a.op; sa.counts[0] = a.C;
     sa.ldo = a.ldc; sa.accumulate = a.accumulate;
     // queries <= 64 (fastid_tc4_supported)
+    if (fastid_bn(sa.nq, sa.nbits) == 32) return sa.popD ? launch_f<32, 2>(sa, s) : launch_f<32, 4>(sa, s);
     return sa.popD ? launch_f<64, 2>(sa, s) : launch_f<64, 4>(sa, s);
 }
 
@@ -854,6 +865,7 @@ size_t fastid_search_tc4_ws_bytes(int64_t nq, int nops) {
 }
 
 cudaError_t launch_fastid_search_tc4(const SearchArgs &a, cudaStream_t s) {
+    if (fastid_bn(a.nq, a.nbits) == 32) return a.popD ? launch_f<32, 2>(a, s) : launch_f<32, 4>(a, s);
     return a.popD ? launch_f<64, 2>(a, s) : launch_f<64, 4>(a, s);
 }
 

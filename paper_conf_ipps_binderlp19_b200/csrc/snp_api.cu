@@ -349,17 +349,22 @@ bool search_fused(int64_t nq, int64_t nd, int64_t nbits) {
            tc_kernel_for(nq, nd, nbits, EPI_COUNTS) == SNP_KERNEL_FASTID_MXF4;
 }
 
-// a7 measured dispatch (configs[4] sweep, profiles/round1/sweep.txt): for more than 64
+// a7 measured dispatch (configs[4] sweeps, profiles/round1/sweep_configs4*.txt): for more than 64
 // queries at nbits <= 4096 the fused FastID kernel run on 64-query slices (one database
 // pass each) beats the general kernel + best pass (e.g. M = 128 x 1M x 2048: 0.28 vs
 // 0.63 ms, M = 8192 x 1M x 4096: 26 vs 31 ms); above 4096 bits the general kernel wins.
-constexpr int64_t SLICE_Q = 64;
-bool search_sliced(int64_t nq, int64_t nd, int64_t nbits) {
+// Returns the slice width (64, or 32 where only the 32-wide kernel fits: 33..64 queries at
+// 6500..9700 bits, 2 x 4.9 ms vs 14.3 ms at 20M x 8192) or 0 for no slicing.
+int64_t search_slice_width(int64_t nq, int64_t nd, int64_t nbits) {
     const char *e = std::getenv("SNP_SEARCH_SLICES");   // "0": never (A/B measurement hook)
-    if (e && e[0] == '0') return false;
-    return nq > SLICE_Q && nd > 0 && nbits <= 4096 && choose_variant(nq, nd, nbits) == SNP_VARIANT_TC &&
-           fastid_tc4_supported(SLICE_Q, nd, nbits) && nd >= 4 * SLICE_Q;
+    if (e && e[0] == '0') return 0;
+    if (nd <= 0 || nq <= 32 || choose_variant(nq, nd, nbits) != SNP_VARIANT_TC) return 0;
+    if (nq > 64 && nbits <= 4096 && fastid_bn(64, nbits) == 64 && fastid_tc4_supported(64, nd, nbits)) return 64;
+    if (nq <= 64 && fastid_bn(64, nbits) == 0 && fastid_bn(32, nbits) == 32 && fastid_tc4_supported(32, nd, nbits))
+        return 32;
+    return 0;
 }
+bool search_sliced(int64_t nq, int64_t nd, int64_t nbits) { return search_slice_width(nq, nd, nbits) != 0; }
 
 }  // namespace
 
@@ -369,7 +374,7 @@ size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, 
     if (nq <= 0 || nbits <= 0 || nops < 1 || nops > 4) return 0;
     if (nd < 0) return 0;
     if (search_fused(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(nq, nops);
-    if (search_sliced(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(SLICE_Q, nops);
+    if (search_sliced(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(search_slice_width(nq, nd, nbits), nops);
     size_t b = align256((size_t)nops * nq * 8);
     if (nd == 0) return b;
     b += align256((size_t)nq * search_chunk_rows(nq, nd) * 4);
@@ -447,7 +452,7 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
         return SNP_OK;
     }
 
-    if (search_sliced(nq, nd, nbits)) {
+    if (const int64_t SLICE_Q = search_slice_width(nq, nd, nbits)) {
         // 64-query slices through the fused kernel, one database pass each; the key
         // workspace is reused slice after slice (stream order; each launch re-initialises it)
         for (int64_t q0 = 0; q0 < nq; q0 += SLICE_Q) {

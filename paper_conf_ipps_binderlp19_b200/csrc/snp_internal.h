@@ -84,6 +84,7 @@ bool gemm_tc4_last_sym();
 // FastID-shaped tcgen05 mxf4 kernel (fastid_tc4.cu): <= 128 queries resident in shared
 // memory, database streamed by TMA.  The queries are the user's first operand.
 bool fastid_tc4_supported(int64_t m, int64_t n, int64_t nbits);
+int fastid_bn(int64_t m, int64_t nbits);   // resident query width (64, 32) or 0
 cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s);
 size_t fastid_search_tc4_ws_bytes(int64_t nq, int nops);
 cudaError_t launch_fastid_search_tc4(const SearchArgs &a, cudaStream_t s);

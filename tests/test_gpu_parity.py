@@ -344,7 +344,9 @@ ALL_OPS = ("and", "xor", "andnot", "notand")
 # > 64 queries: 64-query slices of the fused kernel up to 4096 bits (a7), above that the
 # general kernel (two ops per pass) + best pass
 SEARCH_SHAPES = [(1, 4, 1), (3, 700, 129), (33, 1000, 4096), (64, 2000, 777), (64, 300, 100),
-                 (70, 513, 1000), (130, 300, 2049), (100, 3000, 5000)]
+                 (70, 513, 1000), (130, 300, 2049), (100, 3000, 5000),
+                 (20, 3000, 8000), (32, 700, 9000),   # <= 32 queries at > 6500 bits: 32-wide kernel
+                 (50, 1200, 7000)]                    # 33..64 queries there: two 32-query slices
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -376,6 +378,11 @@ def test_search_all_ops_counts_and_best(snp, variant, nq, nd, nbits, pre):
 
 
 def test_search_kernel_choice(snp):
+    for nq, nbits in ((32, 8192), (20, 9000)):   # the 32-wide resident-query kernel
+        db = snpgen.fastid_db(4, np.arange(2048), nbits)
+        q, _ = snpgen.fastid_queries(4, nq, 2048, nbits)
+        snp.snp_fastid_search(pack_dev(snp, q), pack_dev(snp, db), nbits)
+        assert snp.snp_last_kernel() == "fastid_mxf4", (nq, nbits)
     nbits, nd = 4096, 4096
     db = snpgen.fastid_db(3, np.arange(nd), nbits)
     q, _ = snpgen.fastid_queries(3, 64, nd, nbits)
