@@ -267,8 +267,12 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
         popA = pa;
     }
     if (!popB) {
-        if ((e = launch_row_popc(B, n, nbits, ldb, pb, s)) != cudaSuccess) return set_cuda_error(e);
-        popB = pb;
+        if (B == A && n == m && ldb == lda) {
+            popB = popA;   // self-LD (B aliases A): one popcount pass
+        } else {
+            if ((e = launch_row_popc(B, n, nbits, ldb, pb, s)) != cudaSuccess) return set_cuda_error(e);
+            popB = pb;
+        }
     }
     GemmArgs a{};
     a.A = reinterpret_cast<const uint32_t *>(A);
