@@ -405,6 +405,7 @@ def setup_ld(wl, rank, world, dev):
                                            structure=True, xp="torch", device=dev)
     Ghost = G.cpu().pin_memory() if (rank == 0) else None
     B = torch.empty((m, words), dtype=torch.uint64, device=dev)
+    pop = torch.empty(m, dtype=torch.uint32, device=dev)
     r2 = torch.empty((rows, m), dtype=torch.float32, device=dev)
     cnt = torch.empty((rows, m), dtype=torch.uint32, device=dev)
     ws = torch.empty(max(1, snp.snp_ld_workspace_bytes(rows, m, nbits)), dtype=torch.uint8, device=dev)
@@ -416,13 +417,14 @@ def setup_ld(wl, rank, world, dev):
         if rank == 0:
             if host:
                 G.copy_(Ghost, non_blocking=True)                           # e2e H2D
-            snp.snp_pack(G, nbits=nbits, out=B)                            # a1
+            snp.snp_pack_popc(G, nbits=nbits, out=B, popc=pop)             # a1 + a2
         if world > 1:
             import torch.distributed as dist
             dist.broadcast(B.view(torch.int64), src=0)
+            dist.broadcast(pop.view(torch.int32), src=0)
         if kev is not None:
             kev[0].record(s)
-        snp.snp_ld_r2(B[lo:hi], B, nbits, r2=r2, counts=cnt, ws=ws)       # a2 + a3 + a5
+        snp.snp_ld_r2(B[lo:hi], B, nbits, popA=pop[lo:hi], popB=pop, r2=r2, counts=cnt, ws=ws)   # a3 + a5
         if kev is not None:
             kev[1].record(s)
         if host:   # e2e: D2H of the step's result statistic (r2 of the first pair)
@@ -431,8 +433,9 @@ def setup_ld(wl, rank, world, dev):
     def l2flush():
         flush.add_(1)
 
-    parts = [(lambda: snp.snp_pack(G, nbits=nbits, out=B), False),
-             (lambda: snp.snp_ld_r2(B[lo:hi], B, nbits, r2=r2, counts=cnt, ws=ws), True)] if rank == 0 else None
+    parts = [(lambda: snp.snp_pack_popc(G, nbits=nbits, out=B, popc=pop), False),
+             (lambda: snp.snp_ld_r2(B[lo:hi], B, nbits, popA=pop[lo:hi], popB=pop, r2=r2, counts=cnt, ws=ws), True)] \
+        if rank == 0 else None
 
     alg_bytes = (rows + m) * words * 8 + rows * m * 8
     return dict(step=step, parts=parts, cmp_rank=rows * m * nbits, cmp_all=m * m * nbits, kernel_launches_per_step=1,

@@ -96,6 +96,12 @@ size_t snp_fastid_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op)
 snp_status snp_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg_bytes,
                     uint64_t *packed, int64_t ldw, void *stream);
 
+/* a1 + a2 fused — snp_pack followed by snp_row_popc in one pass over g (same
+ * arguments, layout and errors as snp_pack; popc: uint32 [rows], popc[r] = set bits
+ * of packed row r, the p_A / p_B of P:L44 as counts; NULL -> SNP_E_NULL). */
+snp_status snp_pack_popc(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg_bytes,
+                         uint64_t *packed, int64_t ldw, uint32_t *popc, void *stream);
+
 /* a2 — popc[r] = number of set bits among the first nbits of packed row r
  * (p_A / p_B of P:L44 as counts). */
 snp_status snp_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int64_t ldw,

@@ -19,7 +19,7 @@ from ._lib import SnpError, check, lib, status_string  # noqa: F401
 
 __all__ = [
     "SnpError", "OPS", "VARIANTS", "snp_words", "snp_ld_workspace_bytes",
-    "snp_fastid_workspace_bytes", "snp_pack", "snp_row_popc", "snp_ld_counts",
+    "snp_fastid_workspace_bytes", "snp_pack", "snp_pack_popc", "snp_row_popc", "snp_ld_counts",
     "snp_ld_r2", "snp_fastid", "snp_fastid_best", "snp_fastid_search",
     "snp_fastid_search_workspace_bytes", "snp_shard_plan", "snp_set_variant",
     "snp_last_variant", "snp_last_kernel", "snp_launch_count", "status_string",
@@ -97,6 +97,25 @@ def snp_pack(g: torch.Tensor, nbits: int | None = None, ldw: int | None = None,
     _dev_tensor(out, "out", _WORD_DTYPES)
     check(lib().snp_pack(_ptr(g), rows, nbits, _ld(g), _ptr(out), _ld(out), _stream(stream)), "snp_pack")
     return out
+
+
+def snp_pack_popc(g: torch.Tensor, nbits: int | None = None, ldw: int | None = None,
+                  out: torch.Tensor | None = None, popc: torch.Tensor | None = None,
+                  stream=None) -> tuple[torch.Tensor, torch.Tensor]:
+    """a1 + a2 fused: packed uint64 rows and their uint32 popcounts from one pass over g."""
+    _dev_tensor(g, "g", (torch.uint8, torch.bool))
+    rows = g.shape[0]
+    nbits = g.shape[1] if nbits is None else int(nbits)
+    if out is None:
+        ldw = snp_words(nbits) if ldw is None else int(ldw)
+        out = torch.empty((rows, ldw), dtype=torch.uint64, device=g.device)
+    if popc is None:
+        popc = torch.empty(rows, dtype=torch.uint32, device=g.device)
+    _dev_tensor(out, "out", _WORD_DTYPES)
+    _dev_tensor(popc, "popc", _U32)
+    check(lib().snp_pack_popc(_ptr(g), rows, nbits, _ld(g), _ptr(out), _ld(out), _ptr(popc), _stream(stream)),
+          "snp_pack_popc")
+    return out, popc
 
 
 def snp_row_popc(x: torch.Tensor, nbits: int, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:

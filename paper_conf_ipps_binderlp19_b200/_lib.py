@@ -20,6 +20,7 @@ SIGNATURES = {
     "snp_fastid_workspace_bytes": (_sz, [_i64, _i64, _i64, _int]),
     "snp_pack": (_int, [_p, _i64, _i64, _i64, _p, _i64, _p]),
     "snp_row_popc": (_int, [_p, _i64, _i64, _i64, _p, _p]),
+    "snp_pack_popc": (_int, [_p, _i64, _i64, _i64, _p, _i64, _p, _p]),
     "snp_ld_counts": (_int, [_p, _i64, _i64, _p, _i64, _i64, _i64, _p, _i64, _int, _p, _sz, _p]),
     "snp_ld_r2": (_int, [_p, _i64, _i64, _p, _p, _i64, _i64, _p, _i64, _p, _p, _p, _i64, _p, _sz, _p]),
     "snp_fastid": (_int, [_p, _i64, _i64, _p, _p, _i64, _i64, _p, _i64, _int, _p, _i64, _int, _p, _sz, _p]),

@@ -64,6 +64,48 @@ __global__ void pack_byte_kernel(const uint8_t *__restrict__ g, int64_t rows, in
     }
 }
 
+// a1 + a2 fused: one warp per row packs the row's words (as pack_*_kernel) and sums their
+// popcounts, so the LD step reads the genotype bytes once and skips the row_popc pass.
+// Bits past nbits are packed as zero, so the word popcounts need no mask.
+template <bool VEC>
+__global__ void pack_popc_kernel(const uint8_t *__restrict__ g, int64_t rows, int64_t nbits,
+                                 int64_t ldg, uint64_t *__restrict__ packed, int64_t ldw,
+                                 uint32_t *__restrict__ popc) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t r = warp; r < rows; r += nwarps) {
+        uint32_t c = 0;
+        for (int64_t w = lane; w < ldw; w += 32) {
+            const int64_t k0 = w * 64;
+            uint64_t word = 0;
+            if (k0 < nbits) {
+                const uint8_t *src = g + r * ldg + k0;
+                const int64_t valid = nbits - k0;
+                if (VEC && valid >= 64) {
+                    const uint4 *p = reinterpret_cast<const uint4 *>(src);
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        uint4 v = __ldg(p + q);
+                        uint64_t lo = ((uint64_t)v.y << 32) | v.x;
+                        uint64_t hi = ((uint64_t)v.w << 32) | v.z;
+                        word |= (uint64_t)nonzero_bits8(lo) << (16 * q);
+                        word |= (uint64_t)nonzero_bits8(hi) << (16 * q + 8);
+                    }
+                } else {
+                    const int64_t nb = valid < 64 ? valid : 64;
+                    for (int64_t k = 0; k < nb; ++k) word |= (uint64_t)(src[k] != 0) << k;
+                }
+            }
+            packed[r * ldw + w] = word;
+            c += __popcll(word);
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+        if (lane == 0) popc[r] = c;
+    }
+}
+
 // One warp per row; lanes stride over the row's words; last word masked.
 __global__ void row_popc_kernel(const uint64_t *__restrict__ x, int64_t rows, int64_t nbits,
                                 int64_t ldw, uint32_t *__restrict__ popc) {
@@ -106,6 +148,19 @@ cudaError_t launch_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t l
         pack_vec_kernel<<<blocks, threads, 0, s>>>(g, rows, nbits, ldg, packed, ldw);
     else
         pack_byte_kernel<<<blocks, threads, 0, s>>>(g, rows, nbits, ldg, packed, ldw);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pack_popc(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg,
+                             uint64_t *packed, int64_t ldw, uint32_t *popc, cudaStream_t s) {
+    const int threads = 256;
+    const int blocks = grid_for(rows * 32, threads);
+    const bool vec = ((uintptr_t)g % 16 == 0) && (ldg % 16 == 0);
+    if (vec)
+        pack_popc_kernel<true><<<blocks, threads, 0, s>>>(g, rows, nbits, ldg, packed, ldw, popc);
+    else
+        pack_popc_kernel<false><<<blocks, threads, 0, s>>>(g, rows, nbits, ldg, packed, ldw, popc);
     count_launches(1);
     return cudaGetLastError();
 }

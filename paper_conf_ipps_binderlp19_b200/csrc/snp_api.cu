@@ -199,6 +199,19 @@ snp_status snp_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg_b
     return e == cudaSuccess ? SNP_OK : set_cuda_error(e);
 }
 
+snp_status snp_pack_popc(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg_bytes,
+                         uint64_t *packed, int64_t ldw, uint32_t *popc, void *stream) {
+    if (rows < 0 || nbits < 0 || ldg_bytes < 0 || ldw < 0) return SNP_E_SHAPE;
+    if (rows == 0) return SNP_OK;
+    if (!g || !packed || !popc) return SNP_E_NULL;
+    if (nbits < 1 || ldg_bytes < nbits || ldw < words_needed(nbits)) return SNP_E_SHAPE;
+    if (!aligned16(packed) || (ldw & 1)) return SNP_E_ALIGN;
+    snp_status st = check_arch();
+    if (st != SNP_OK) return st;
+    cudaError_t e = launch_pack_popc(g, rows, nbits, ldg_bytes, packed, ldw, popc, (cudaStream_t)stream);
+    return e == cudaSuccess ? SNP_OK : set_cuda_error(e);
+}
+
 snp_status snp_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int64_t ldw,
                         uint32_t *popc, void *stream) {
     snp_status st = check_nbits(nbits);

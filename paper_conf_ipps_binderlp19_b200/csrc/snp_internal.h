@@ -39,6 +39,8 @@ cudaError_t launch_bitgemm_popc(const GemmArgs &a, int epi, cudaStream_t s);
 // pack.cu
 cudaError_t launch_pack(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg,
                         uint64_t *packed, int64_t ldw, cudaStream_t s);
+cudaError_t launch_pack_popc(const uint8_t *g, int64_t rows, int64_t nbits, int64_t ldg,
+                             uint64_t *packed, int64_t ldw, uint32_t *popc, cudaStream_t s);
 cudaError_t launch_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int64_t ldw,
                             uint32_t *popc, cudaStream_t s);
 

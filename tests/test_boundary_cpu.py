@@ -21,7 +21,7 @@ def declared_symbols():
 
 def test_header_declares_expected_calls():
     syms = declared_symbols()
-    for name in ("snp_pack", "snp_row_popc", "snp_ld_counts", "snp_ld_r2", "snp_fastid",
+    for name in ("snp_pack", "snp_pack_popc", "snp_row_popc", "snp_ld_counts", "snp_ld_r2", "snp_fastid",
                  "snp_fastid_best", "snp_shard_plan", "snp_words", "snp_status_string"):
         assert name in syms
 

@@ -77,6 +77,33 @@ def test_pack_unaligned_rows(snp):
     assert np.array_equal(P.cpu().numpy(), oracle.pack(big[:, 3:3 + nbits], snp.snp_words(nbits)))
 
 
+@pytest.mark.parametrize("nbits", [1, 63, 64, 65, 1000, 4095, 4097, 16384])
+@pytest.mark.parametrize("offset", [0, 3])
+def test_pack_popc_fused(snp, nbits, offset):
+    """a1 + a2 in one pass: packed words and row popcounts both equal the oracle's
+    (offset 3 exercises the unaligned byte path; extra ldw words must come back zero)."""
+    rows = 4100 if nbits <= 1000 else 70          # more rows than one grid-stride pass at small nbits
+    rng = np.random.default_rng(nbits + offset)
+    big = (rng.random((rows, nbits + offset)) < 0.3).astype(np.uint8) * \
+        snpgen.random_bytes_nonzero((rows, nbits + offset), 2)
+    g = big[:, offset:offset + nbits]
+    ldw = snp.snp_words(nbits) + 2
+    P, pc = snp.snp_pack_popc(to_dev(big)[:, offset:offset + nbits], nbits=nbits, ldw=ldw)
+    torch.cuda.synchronize()
+    assert np.array_equal(P.cpu().numpy(), oracle.pack(g, ldw))
+    assert np.array_equal(u32(pc), oracle.row_popc(g))
+
+
+def test_pack_popc_empty_and_errors(snp):
+    g = torch.zeros((0, 64), dtype=torch.uint8, device=DEV)
+    P, pc = snp.snp_pack_popc(g, nbits=64)
+    assert P.shape[0] == 0 and pc.shape[0] == 0
+    lib = snp.lib()
+    g1 = torch.ones((2, 64), dtype=torch.uint8, device=DEV)
+    out = torch.empty((2, 8), dtype=torch.uint64, device=DEV)
+    assert lib.snp_pack_popc(g1.data_ptr(), 2, 64, 64, out.data_ptr(), 8, None, None) != 0   # popc NULL
+
+
 @pytest.mark.parametrize("nbits", [1, 64, 65, 1000, 4097])
 def test_row_popc_ignores_padding(snp, nbits):
     g = snpgen.fastid_db(7, np.arange(300), nbits)
