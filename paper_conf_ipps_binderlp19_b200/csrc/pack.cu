@@ -71,6 +71,9 @@ template <bool VEC>
 __global__ void pack_popc_kernel(const uint8_t *__restrict__ g, int64_t rows, int64_t nbits,
                                  int64_t ldg, uint64_t *__restrict__ packed, int64_t ldw,
                                  uint32_t *__restrict__ popc) {
+    // programmatic dependent launch: the bit-GEMM (launched with PDL) may start its setup
+    // now; its griddepcontrol.wait still waits for this grid to finish and flush
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
