@@ -21,7 +21,7 @@ __device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a, uint64_t b, 
                  :: "r"(d), "r"(a), "l"(b), "r"(idesc), "r"(acc), "r"(sfa), "r"(sfb));
 }
 
-template <int MODE, int N, int CONTEND = 0>   // MODE 0: mxf4 SS, 1: mxf4 TS, 2: i8 SS, 3: i8 TS
+template <int MODE, int N, int CONTEND = 0, int M = 128>   // MODE 0: mxf4 SS, 1: mxf4 TS, 2: i8 SS, 3: i8 TS
 // CONTEND 1: warps 1-4 hammer tcgen05.st into other TMEM columns; 2: tcgen05.ld
 __global__ void probe(int iters, long long *out) {
     extern __shared__ __align__(1024) uint8_t sm[];
@@ -37,10 +37,10 @@ __global__ void probe(int iters, long long *out) {
         const uint64_t bd = ptx::smem_desc_kmajor_noswizzle(sb, N * 16, 128);
         long long t0 = clock64();
         for (int i = 0; i < iters; ++i) {
-            if (MODE == 0) mma_mxf4_ss(tmem, ad, bd, idesc_mxf4(128, N), 1, tmem + 480, tmem + 496);
-            else if (MODE == 1) mma_mxf4_ts(tmem, tmem + 256 + (i & 7) * 8, bd, idesc_mxf4(128, N), 1, tmem + 480, tmem + 496);
-            else if (MODE == 2) ptx::mma_i8_ss(tmem, ad, bd, ptx::idesc_u8_s32(128, N), 1);
-            else ptx::mma_i8_ts(tmem, tmem + 256 + (i & 7) * 8, bd, ptx::idesc_u8_s32(128, N), 1);
+            if (MODE == 0) mma_mxf4_ss(tmem, ad, bd, idesc_mxf4(M, N), 1, tmem + 480, tmem + 496);
+            else if (MODE == 1) mma_mxf4_ts(tmem, tmem + 256 + (i & 7) * 8, bd, idesc_mxf4(M, N), 1, tmem + 480, tmem + 496);
+            else if (MODE == 2) ptx::mma_i8_ss(tmem, ad, bd, ptx::idesc_u8_s32(M, N), 1);
+            else ptx::mma_i8_ts(tmem, tmem + 256 + (i & 7) * 8, bd, ptx::idesc_u8_s32(M, N), 1);
         }
         ptx::mma_commit(&bar);
         ptx::mbar_wait(&bar, 0);
@@ -59,11 +59,11 @@ __global__ void probe(int iters, long long *out) {
     if (threadIdx.x < 32) { ptx::tc_fence_after(); ptx::tmem_dealloc<512>(tmem); }
 }
 
-template <int MODE, int N, int CONTEND = 0>
+template <int MODE, int N, int CONTEND = 0, int M = 128>
 void run(const char *name) {
     long long *d; cudaMalloc(&d, 148 * sizeof(long long));
     const int iters = 4096;
-    auto k = probe<MODE, N, CONTEND>;
+    auto k = probe<MODE, N, CONTEND, M>;
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
     k<<<148, 192, 64 * 1024>>>(iters, d);
     cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
@@ -75,9 +75,9 @@ void run(const char *name) {
     cudaError_t err = cudaGetLastError();
     double cyc = (double)h[0] / iters;
     const int K = (MODE <= 1) ? 64 : 32;
-    double macs = 128.0 * N * K * iters * 148;
-    printf("%-14s N=%3d  %7.1f cycles/MMA  %8.1f MAC/clk/SM  %7.0f TMAC/s (event %.3f ms) %s\n", name, N, cyc,
-           128.0 * N * K / cyc, macs / (ms * 1e-3) / 1e12, ms, err == cudaSuccess ? "" : cudaGetErrorString(err));
+    double macs = (double)M * N * K * iters * 148;
+    printf("%-14s M=%3d N=%3d  %7.1f cycles/MMA  %8.1f MAC/clk/SM  %7.0f TMAC/s (event %.3f ms) %s\n", name, M, N, cyc,
+           (double)M * N * K / cyc, macs / (ms * 1e-3) / 1e12, ms, err == cudaSuccess ? "" : cudaGetErrorString(err));
     cudaFree(d);
 }
 
@@ -88,5 +88,11 @@ int main() {
     run<3, 64>("i8 TS"); run<3, 128>("i8 TS"); run<3, 256>("i8 TS");
     run<1, 64, 1>("mxf4 TS +st"); run<1, 128, 1>("mxf4 TS +st"); run<0, 64, 1>("mxf4 SS +st");
     run<1, 64, 2>("mxf4 TS +ld"); run<0, 64, 2>("mxf4 SS +ld");
+    // skinny shapes (few queries): is the per-MMA cost proportional to N below 64?
+    run<1, 16>("mxf4 TS"); run<1, 32>("mxf4 TS"); run<1, 48>("mxf4 TS");
+    run<0, 16>("mxf4 SS"); run<0, 32>("mxf4 SS");
+    run<0, 8, 0, 64>("mxf4 SS"); run<0, 16, 0, 64>("mxf4 SS"); run<0, 32, 0, 64>("mxf4 SS"); run<0, 64, 0, 64>("mxf4 SS");
+    run<0, 128, 0, 64>("mxf4 SS"); run<0, 256, 0, 64>("mxf4 SS");
+    run<1, 8, 0, 64>("mxf4 TS"); run<1, 16, 0, 64>("mxf4 TS"); run<1, 64, 0, 64>("mxf4 TS"); run<1, 256, 0, 64>("mxf4 TS");
     return 0;
 }
