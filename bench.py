@@ -62,6 +62,9 @@ def parse():
                    help="fused: one snp_fastid_search pass for XOR+ANDNOT counts and best matches; "
                         "separate: snp_fastid + snp_fastid_best per op")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target oracle CPU time")
+    p.add_argument("--ld-layout", default="tri", choices=["tri", "rows"],
+                   help="tri: f3 packed upper-triangle tiles, triangle-balanced over ranks (snp_ld_sym); "
+                        "rows: full m x m matrix, output row blocks per rank (snp_ld_r2)")
     a = p.parse_args()
     if a.warmup < 3:
         a.warmup = 3
@@ -81,12 +84,22 @@ def load_peaks():
               "sm_max_mhz": 1965.0}
         src = "fallback (B200_PROFILING.md)"
     sm_mhz = float(pk.get("sm_max_mhz", 1965.0))
+    # POPC issue rate per SM, measured with the paper's §V.D throughput microbenchmark
+    # (tools/alu_probe.cu; profiles/round2/alu_probe.txt): 15.98 / clk / SM
+    popc_clk, popc_src = 16.0, "assumed 16 POPC/clk/SM"
+    try:
+        with open(os.path.join(ROOT, "profiles", "alu_peaks.json")) as f:
+            popc_clk = float(json.load(f)["popc_per_clk_sm"])
+            popc_src = "measured POPC/clk/SM (tools/alu_probe.cu, profiles/alu_peaks.json)"
+    except Exception:
+        pass
     return {
         "src": src,
         "hbm_gbs": float(pk["hbm_gbs"]),
         # POPC pipe: 148 SMs x 16 POPC/clk/SM x 32 bits x max SM clock (P:L281 convention),
         # in TOPS-equivalent (2 ops per bit comparison) — DESIGN.md §6.
-        "popc_tops": 2 * 148 * 16 * 32 * sm_mhz * 1e6 / 1e12,
+        "popc_tops": 2 * 148 * popc_clk * 32 * sm_mhz * 1e6 / 1e12,
+        "popc_src": popc_src, "popc_per_clk_sm": popc_clk,
         # int8 tensor: measured bf16 dense x nominal i8:bf16 ratio 2 (4.5 vs 2.25 PF spec).
         "i8_tops": 2.0 * float(pk["bf16_tflops"]),
         # fp4 (kind::mxf4) tensor: measured bf16 dense x nominal fp4:bf16 ratio 4 (9 vs 2.25 PF).
@@ -313,6 +326,10 @@ def setup_fastid(wl, rank, world, dev):
     merged = {}
     res_host = {op: (torch.empty(nq, dtype=torch.uint32).pin_memory(), torch.empty(nq, dtype=torch.int64).pin_memory())
                 for op in OPS}
+    keys_host = torch.empty((len(OPS), nq), dtype=torch.int64).pin_memory() if world > 1 else None
+    # full e2e (N=1): the count matrices themselves copied back to pinned host memory
+    full_host = ({op: torch.empty((nq, nd), dtype=torch.uint32).pin_memory() for op in OPS}
+                 if world == 1 and nq * nd * 4 * len(OPS) <= (1 << 30) else None)
     st = dict(D=D, Q=Q, qbytes=qbytes, qhost=qhost, outs=outs, best=best, ws=ws, lo=lo, nd=nd,
               res_host=res_host)
     cmp_rank = 2 * nq * nd * nbits
@@ -359,11 +376,16 @@ def setup_fastid(wl, rank, world, dev):
             from paper_conf_ipps_binderlp19_b200 import multigpu
             keys = torch.stack([multigpu.pack_best(*best[op]) for op in OPS])
             merged["keys"] = multigpu.gather_best(keys)
+            if host:   # e2e: D2H of the step's result, the GLOBAL best (count << 40 | index keys)
+                keys_host.copy_(merged["keys"], non_blocking=True)
+            return
         for op in OPS:
             bc, bi = best[op]
             if host:   # e2e: D2H of the step's result (per-query best count and index)
                 res_host[op][0].copy_(bc, non_blocking=True)
                 res_host[op][1].copy_(bi, non_blocking=True)
+            if host == "full":   # full e2e: the count matrices too
+                full_host[op].copy_(outs[op], non_blocking=True)
 
     # the same device-resident step as separately capturable parts (N=1 graph mode)
     pack_part = (lambda: snp.snp_pack(qbytes, nbits=nbits, out=Q), False)
@@ -380,12 +402,22 @@ def setup_fastid(wl, rank, world, dev):
     return dict(step=step, parts=parts, cmp_rank=cmp_rank, cmp_all=cmp_all,
                 kernel_launches_per_step=1 if fused else 2, step_mode=FASTID_STEP,
                 kernel_cmp=nq * nd * nbits, kernel_bytes=alg_bytes,
-                h2d=nq * nbits, d2h=2 * nq * 12, l2_flush=False,
+                h2d=nq * nbits, d2h=(2 * nq * 8 if world > 1 else 2 * nq * 12), l2_flush=False,
+                d2h_full=(len(OPS) * nq * nd * 4 if full_host is not None else None),
+                e2e_result=("global best (count, index) per query for XOR and ANDNOT (merged over ranks); "
+                            "the count matrices stay sharded in HBM" if world > 1 else
+                            "per-query best (count, index) for XOR and ANDNOT; the two nq x nd count matrices "
+                            "stay in HBM (e2e_full copies them back too)"),
                 l2_note=f"inputs larger than L2 ({nd * snp.snp_words(nbits) * 8 / 1e6:.0f} MB database per rank)",
                 state=st, snp=snp)
 
 
+LD_LAYOUT = "tri"
+
+
 def setup_ld(wl, rank, world, dev):
+    if LD_LAYOUT == "tri":
+        return setup_ld_tri(wl, rank, world, dev)
     import torch
 
     import paper_conf_ipps_binderlp19_b200 as snp
@@ -410,6 +442,8 @@ def setup_ld(wl, rank, world, dev):
     cnt = torch.empty((rows, m), dtype=torch.uint32, device=dev)
     ws = torch.empty(max(1, snp.snp_ld_workspace_bytes(rows, m, nbits)), dtype=torch.uint8, device=dev)
     res_host = torch.empty(1, dtype=torch.float32).pin_memory()
+    full_host = ((torch.empty((rows, m), dtype=torch.float32).pin_memory(),
+                  torch.empty((rows, m), dtype=torch.uint32).pin_memory()) if rows * m * 8 <= (1 << 30) else None)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
     def step(kev=None, host=False):
@@ -429,6 +463,9 @@ def setup_ld(wl, rank, world, dev):
             kev[1].record(s)
         if host:   # e2e: D2H of the step's result statistic (r2 of the first pair)
             res_host.copy_(r2.view(-1)[:1], non_blocking=True)
+        if host == "full":   # full e2e: the r2 and count matrices of this rank
+            full_host[0].copy_(r2, non_blocking=True)
+            full_host[1].copy_(cnt, non_blocking=True)
 
     def l2flush():
         flush.add_(1)
@@ -440,7 +477,79 @@ def setup_ld(wl, rank, world, dev):
     alg_bytes = (rows + m) * words * 8 + rows * m * 8
     return dict(step=step, parts=parts, cmp_rank=rows * m * nbits, cmp_all=m * m * nbits, kernel_launches_per_step=1,
                 kernel_cmp=rows * m * nbits, kernel_bytes=alg_bytes, h2d=(m * nbits if rank == 0 else 0),
-                d2h=4, l2_flush=True, flush=l2flush,
+                d2h=4, l2_flush=True, flush=l2flush, d2h_full=(rows * m * 8 if full_host is not None else None),
+                e2e_result="r2 of the first pair (the r2 and count matrices stay in HBM; e2e_full copies them back)",
+                l2_note="L2 flushed (256 MB write) between timed steps, outside the per-step events",
+                state=dict(B=B, r2=r2, cnt=cnt), snp=snp)
+
+
+def setup_ld_tri(wl, rank, world, dev):
+    """LD as symmetric self-LD in the packed upper-triangle tile layout (f3): rank r computes
+    the contiguous tile range of snp_shard_plan_sym (balanced within one tile, no tile twice,
+    no mirrored-block exchange); counts + r2 per tile."""
+    import torch
+
+    import paper_conf_ipps_binderlp19_b200 as snp
+    import snpgen
+    m, nbits = wl["m"], wl["nbits"]
+    b = snp.snp_shard_plan_sym(m, world)
+    lo, hi = b[rank], b[rank + 1]
+    nt = hi - lo
+    words = snp.snp_words(nbits)
+    G = None
+    if rank == 0:
+        G = torch.empty((m, nbits), dtype=torch.uint8, device=dev)
+        for r0 in range(0, m, 2048):
+            r1 = min(m, r0 + 2048)
+            G[r0:r1] = snpgen.ld_genotypes(wl["seed"], torch.arange(r0, r1, device=dev), nbits,
+                                           structure=True, xp="torch", device=dev)
+    Ghost = G.cpu().pin_memory() if (rank == 0) else None
+    B = torch.empty((m, words), dtype=torch.uint64, device=dev)
+    pop = torch.empty(m, dtype=torch.uint32, device=dev)
+    r2 = torch.empty((max(nt, 1), 128, 128), dtype=torch.float32, device=dev)
+    cnt = torch.empty((max(nt, 1), 128, 128), dtype=torch.uint32, device=dev)
+    res_host = torch.empty(1, dtype=torch.float32).pin_memory()
+    out_bytes = nt * 128 * 128 * 8
+    full_host = ((torch.empty_like(r2, device="cpu").pin_memory(), torch.empty_like(cnt, device="cpu").pin_memory())
+                 if out_bytes <= (1 << 30) else None)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def compute():
+        snp.snp_ld_sym(B, nbits, lo, hi, popA=pop, r2=r2, counts=cnt)          # a3 + a5 (f3 tiles)
+
+    def step(kev=None, host=False):
+        s = torch.cuda.current_stream()
+        if rank == 0:
+            if host:
+                G.copy_(Ghost, non_blocking=True)                           # e2e H2D
+            snp.snp_pack_popc(G, nbits=nbits, out=B, popc=pop)             # a1 + a2
+        if world > 1:
+            import torch.distributed as dist
+            dist.broadcast(B.view(torch.int64), src=0)
+            dist.broadcast(pop.view(torch.int32), src=0)
+        if kev is not None:
+            kev[0].record(s)
+        compute()
+        if kev is not None:
+            kev[1].record(s)
+        if host:   # e2e: D2H of the step's result statistic (r2 of the first pair)
+            res_host.copy_(r2.view(-1)[:1], non_blocking=True)
+        if host == "full":   # full e2e: this rank's r2 and count tiles
+            full_host[0].copy_(r2, non_blocking=True)
+            full_host[1].copy_(cnt, non_blocking=True)
+
+    def l2flush():
+        flush.add_(1)
+
+    parts = [(lambda: snp.snp_pack_popc(G, nbits=nbits, out=B, popc=pop), False), (compute, True)] \
+        if rank == 0 else None
+    alg_bytes = m * words * 8 + out_bytes
+    return dict(step=step, parts=parts, cmp_rank=nt * 128 * 128 * nbits, cmp_all=m * m * nbits,
+                kernel_launches_per_step=1, kernel_cmp=nt * 128 * 128 * nbits, kernel_bytes=alg_bytes,
+                h2d=(m * nbits if rank == 0 else 0), d2h=4, l2_flush=True, flush=l2flush,
+                d2h_full=(out_bytes if full_host is not None else None),
+                e2e_result="r2 of the first pair (this rank's r2 and count tiles stay in HBM; e2e_full copies them)",
+                layout=f"packed upper triangle: tiles [{lo}, {hi}) of {b[-1]} (128 x 128, row-major triangle order)",
                 l2_note="L2 flushed (256 MB write) between timed steps, outside the per-step events",
                 state=dict(B=B, r2=r2, cnt=cnt), snp=snp)
 
@@ -535,8 +644,9 @@ def run_ours(args):
     import paper_conf_ipps_binderlp19_b200 as snp
     snp.snp_set_variant(args.variant)
     steps = args.steps or (200 if wl["kind"] == "fastid" else 20)
-    global FASTID_STEP
+    global FASTID_STEP, LD_LAYOUT
     FASTID_STEP = args.fastid_step
+    LD_LAYOUT = args.ld_layout
     wlrun = (setup_fastid if wl["kind"] == "fastid" else setup_ld)(wl, rank, world, dev)
     torch.cuda.synchronize()
 
@@ -572,12 +682,26 @@ def run_ours(args):
         e2e_ms, _ = timed(wlrun, steps, True, world, kernel_events=False)
         e2e = {"value": wlrun["cmp_all"] / (e2e_ms / steps / 1e3), "unit": "comparisons/s",
                "h2d_bytes_per_step": wlrun["h2d"], "d2h_bytes_per_step": wlrun["d2h"],
-               "ms_per_step": e2e_ms / steps}
+               "ms_per_step": e2e_ms / steps, "result": wlrun["e2e_result"],
+               "launch": "eager public-API calls per step (no graph)"}
+        if world == 1 and wlrun.get("d2h_full"):
+            # the same step with every output matrix copied back to the host (PCIe-bound)
+            fsteps = max(3, min(steps, 10))
+            wlrun["step"](None, "full")
+            torch.cuda.synchronize()
+            f_ms, _ = timed(wlrun, fsteps, "full", world, kernel_events=False)
+            e2e["full"] = {"value": wlrun["cmp_all"] / (f_ms / fsteps / 1e3), "unit": "comparisons/s",
+                           "h2d_bytes_per_step": wlrun["h2d"], "d2h_bytes_per_step": wlrun["d2h_full"],
+                           "ms_per_step": f_ms / fsteps, "steps": fsteps}
 
     # roofline of the dominant kernel (the bit-GEMM launch), live CUDA-event durations
     kcmp = wlrun["kernel_cmp"]
     kcmp_eff = kcmp
-    if kernel == "tc_mxf4_sym":
+    if wl["kind"] == "ld" and LD_LAYOUT == "tri":
+        # executed work is the rank's tiles (kernel_cmp); the effective rate counts the
+        # m * m * nbits comparisons of the full symmetric matrix those tiles represent
+        kcmp_eff = wlrun["cmp_all"] // world
+    elif kernel == "tc_mxf4_sym":
         # f3 symmetric self-LD executes only the upper-triangle 128 x 128 tiles (SURVEY §8d:
         # roofline on the executed work, M*N*nbits reported as the effective rate)
         T = -(-wl["m"] // 128)
@@ -591,7 +715,8 @@ def run_ours(args):
                 "peak_src": f"int8 dense = 2 x bf16 burst ({peaks['src']} MEASURED_PEAKS.json)"}
     else:
         roof = {"bound": "alu", "achieved": tops, "peak": peaks["popc_tops"], "unit": "TOPS",
-                "peak_src": "POPC pipe: 148 SM x 16/clk x 32 bit x 1965 MHz (DESIGN.md §6)"}
+                "peak_src": f"POPC pipe: 148 SM x {peaks['popc_per_clk_sm']:.2f}/clk x 32 bit x "
+                            f"{peaks['sm_max_mhz']:.0f} MHz ({peaks['popc_src']})"}
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["kernel_ms"] = kern_ms
     roof["kernel"] = kernel
@@ -637,7 +762,10 @@ def run_ours(args):
                        "variant": variant, "kernel": kernel, "l2": wlrun["l2_note"],
                        **({"step": wlrun["step_mode"]} if "step_mode" in wlrun else {}),
                        "launch": "cuda-graph replay per step" if use_graph else "eager",
-                       "parallelism": f"{'db' if wl['kind'] == 'fastid' else 'row'}-shard x{world}"},
+                       **({"output": wlrun["layout"]} if "layout" in wlrun else {}),
+                       "parallelism": (f"db-shard x{world}" if wl["kind"] == "fastid" else
+                                       f"triangle-tile-shard x{world}" if LD_LAYOUT == "tri" else
+                                       f"row-shard x{world}")},
             "word_ops_per_s": value / 64, "tops_eq": 2 * value / 1e12,
             "roofline": roof_primary, "roofline_secondary": roof_secondary,
             "gpu_launches": launches,

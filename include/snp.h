@@ -35,8 +35,11 @@
  *  - Outputs must not alias inputs.  B == A (self-LD) is allowed.
  *  - The library runs only on compute capability 10.0 (B200, sm_100a); any
  *    other device returns SNP_E_ARCH.  There is no fallback.
- *  - Calls are re-entrant.  Process-wide state: a per-device property cache and
- *    the variant override of snp_set_variant.
+ *  - Calls are re-entrant and thread-safe.  Process-wide state: per-device caches
+ *    (SM count, the dynamic shared-memory opt-in of each kernel, the driver's
+ *    tensor-map encoder; keyed by device, guarded by atomics / a mutex) and the
+ *    variant override of snp_set_variant.  Profiling hooks (pipeline traces, the
+ *    snp_debug_* readers) exist only in -DSNP_PROFILING builds, not in libsnp.so.
  */
 #ifndef SNP_H_
 #define SNP_H_
@@ -74,7 +77,9 @@ typedef enum {
 typedef enum {
     SNP_VARIANT_AUTO = 0, /* pick per shape from the measured dispatch table    */
     SNP_VARIANT_POPC = 1, /* CUDA-core LOP3 + POPC register-blocked bit-GEMM     */
-    SNP_VARIANT_TC = 2    /* tcgen05 kind::i8 tensor-core GEMM on bit-expanded operands */
+    SNP_VARIANT_TC = 2    /* tcgen05 tensor-core GEMM on bit-expanded operands: kind::mxf4
+                             (bits as e2m1 nibbles, fp32 TMEM sums, exact for nbits < 2^24)
+                             and kind::i8 (u8 bits, s32 sums) from nbits = 2^24 up          */
 } snp_variant;
 
 /* Recommended packed leading dimension (uint64 words) for nbits bits:
@@ -120,7 +125,12 @@ snp_status snp_ld_counts(const uint64_t *A, int64_t m, int64_t lda,
  *   num = n*nAB - nA*nB (= n^2 D_AB, exact), den = nA(n-nA) nB(n-nB),
  *   r2 = num^2/den (0 when den == 0, i.e. a monomorphic SNP),
  *   D' = num/Dmax, Dmax = min(nA(n-nB),(n-nA)nB) if num>0 else min(nA nB,(n-nA)(n-nB))
- *   (0 when num == 0).  Computed from exact integers in fp64, stored fp32.
+ *   (0 when num == 0).  num, den and Dmax are exact integers (int32 for n <= 46340, int64
+ *   above); the tensor-core epilogue forms r2 and D' from them in fp32: r2 with at most 9
+ *   roundings (relative error <= 9 * 2^-24 = 5.4e-7), D' with one correctly rounded
+ *   division of two once-rounded integers (<= 3 * 2^-24), stored fp32; exactly 0 where
+ *   the exact value is 0.  The CUDA-core variant computes them in fp64.  Both are within
+ *   the 1e-6 relative bar of the fp64 oracle (north_star).
  * popA/popB: optional precomputed row popcounts (NULL = computed internally).
  * r2: float [m][ldc] (required); dprime: float [m][ldc] or NULL;
  * counts: uint32 nAB [m][ldc] or NULL. */
@@ -128,6 +138,37 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
                      const uint64_t *B, int64_t n, int64_t ldb, const uint32_t *popB,
                      int64_t nbits, float *r2, float *dprime, uint32_t *counts,
                      int64_t ldc, void *ws, size_t ws_bytes, void *stream);
+
+/* f3 — symmetric self-LD in the packed upper-triangle tile layout (LD is
+ * a GEMM of one SNP matrix with itself, §II.A and Fig. 1, so C = C^T and half the
+ * products are redundant).  The m x m output is cut into 128 x 128 tiles, T = ceil(m/128)
+ * per side; tile t <-> (I, J), I <= J < T, in row-major upper-triangle order
+ *     t = start(I) + (J - I),   start(I) = I*T - I*(I-1)/2,   snp_sym_tiles(m) = T(T+1)/2.
+ * A call computes tiles tile_lo .. tile_hi-1 only (one rank's share of
+ * snp_shard_plan_sym) and stores tile t as a dense row-major 128 x 128 block at element
+ * offset (t - tile_lo) * 16384 of each output: element (i, j) of the block is the pair
+ * (SNP 128 I + i, SNP 128 J + j).  Entries of a ragged last tile row/column (index >= m)
+ * are not written.  Diagonal tiles hold both triangles of their block; the full matrix is
+ * the tiles plus their mirror images (snp_sym_unpack).  Statistics as snp_ld_r2 (same
+ * integers, same fp32 epilogue and bound).
+ *   A: [m][lda] packed SNP rows over n = nbits samples.  popA: optional row popcounts.
+ *   r2, dprime (nullable; dprime needs r2), counts (nullable): [tile_hi - tile_lo][128][128]
+ *   float / float / uint32; at least one of r2, counts.  r2 == NULL gives nAB counts only.
+ *   ws: snp_ld_sym_workspace_bytes(m, nbits) bytes when r2 != NULL and popA == NULL.
+ * SNP_E_RANGE for tile_lo < 0, tile_hi < tile_lo or tile_hi > snp_sym_tiles(m).
+ * Kernels: tcgen05 kind::mxf4 (nbits < 2^24) or the CUDA-core variant (forced, or above). */
+int64_t snp_sym_tiles(int64_t m);
+size_t snp_ld_sym_workspace_bytes(int64_t m, int64_t nbits);
+snp_status snp_ld_sym(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *popA, int64_t nbits,
+                      int64_t tile_lo, int64_t tile_hi, float *r2, float *dprime, uint32_t *counts,
+                      void *ws, size_t ws_bytes, void *stream);
+
+/* f3 — scatter packed-triangle tiles tile_lo .. tile_hi-1 (4-byte elements: counts, r2 or
+ * D' viewed as uint32) into the full row-major m x m matrix out[m][ldo] (ldo >= m): block
+ * (I, J) and, for I != J, its transpose at (J, I).  Elements of tiles outside the range are
+ * not written.  HBM-bound copy kernel. */
+snp_status snp_sym_unpack(const uint32_t *tiles, int64_t m, int64_t tile_lo, int64_t tile_hi, uint32_t *out,
+                          int64_t ldo, void *stream);
 
 /* a3 + a4 — FastID comparison counts (Eqs. 2-3):
  *   out[i*ldo + j] (=|+=) sum_k op(Q_ik, D_jk)   for queries i < nq, DB rows j < nd.
@@ -188,6 +229,14 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
  * bounds clamped to rows), block counts balanced to within one.  Deterministic.
  * SNP_E_RANGE for world < 1, align < 1 or rows < 0. */
 snp_status snp_shard_plan(int64_t rows, int world, int64_t align, int64_t *bounds);
+
+/* e + f3 — triangle-area-balanced partition of the symmetric self-LD work (host only):
+ * the snp_sym_tiles(m) equal-cost tiles of snp_ld_sym split into `world` contiguous ranges
+ * tile_bounds[r] .. tile_bounds[r+1] (HOST array of world+1), tile_bounds[r] =
+ * floor(r * total / world): every rank gets floor or ceil of total/world tiles (balanced
+ * within one tile), no tile is computed twice and no exchange of mirrored blocks is needed.
+ * SNP_E_RANGE for world < 1 or m < 0. */
+snp_status snp_shard_plan_sym(int64_t m, int world, int64_t *tile_bounds);
 
 /* Variant override (SNP_VARIANT_AUTO restores the dispatch table).  The
  * environment variable SNP_FORCE_VARIANT=popc|tc sets the initial value. */

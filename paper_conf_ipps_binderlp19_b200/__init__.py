@@ -21,7 +21,8 @@ __all__ = [
     "SnpError", "OPS", "VARIANTS", "snp_words", "snp_ld_workspace_bytes",
     "snp_fastid_workspace_bytes", "snp_pack", "snp_pack_popc", "snp_row_popc", "snp_ld_counts",
     "snp_ld_r2", "snp_fastid", "snp_fastid_best", "snp_fastid_search",
-    "snp_fastid_search_workspace_bytes", "snp_shard_plan", "snp_set_variant",
+    "snp_fastid_search_workspace_bytes", "snp_shard_plan", "snp_shard_plan_sym", "snp_sym_tiles",
+    "snp_ld_sym_workspace_bytes", "snp_ld_sym", "snp_sym_unpack", "snp_set_variant",
     "snp_last_variant", "snp_last_kernel", "snp_launch_count", "status_string",
 ]
 
@@ -287,6 +288,71 @@ def snp_shard_plan(rows: int, world: int, align: int = 128) -> list[int]:
     check(lib().snp_shard_plan(int(rows), int(world), int(align), ctypes.cast(arr, ctypes.c_void_p)),
           "snp_shard_plan")
     return [int(v) for v in arr]
+
+
+SYM_TILE = 128
+
+
+def snp_sym_tiles(m: int) -> int:
+    """f3: number of 128 x 128 tiles in the upper triangle of an m x m self-LD output."""
+    return int(lib().snp_sym_tiles(int(m)))
+
+
+def snp_shard_plan_sym(m: int, world: int) -> list[int]:
+    """e + f3: triangle-balanced contiguous tile ranges per rank (host only)."""
+    arr = (ctypes.c_int64 * (max(1, int(world)) + 1))()
+    check(lib().snp_shard_plan_sym(int(m), int(world), ctypes.cast(arr, ctypes.c_void_p)), "snp_shard_plan_sym")
+    return [int(v) for v in arr][:int(world) + 1]
+
+
+def snp_ld_sym_workspace_bytes(m: int, nbits: int) -> int:
+    return int(lib().snp_ld_sym_workspace_bytes(int(m), int(nbits)))
+
+
+def snp_ld_sym(A: torch.Tensor, nbits: int, tile_lo: int = 0, tile_hi: int | None = None, popA=None,
+               r2: torch.Tensor | bool | None = True, dprime: torch.Tensor | bool | None = None,
+               counts: torch.Tensor | bool | None = None, ws: torch.Tensor | None = None, stream=None):
+    """f3: self-LD tiles [tile_lo, tile_hi) of the row-major upper triangle, each a dense
+    128 x 128 block ([tiles][128][128] outputs).  Returns (r2, dprime, counts), None where
+    not requested (True allocates)."""
+    _dev_tensor(A, "A", _WORD_DTYPES)
+    m = A.shape[0]
+    tile_hi = snp_sym_tiles(m) if tile_hi is None else int(tile_hi)
+    nt = max(0, tile_hi - int(tile_lo))
+    dev = A.device
+
+    def _out(x, dt):
+        if x is True:
+            return torch.empty((nt, SYM_TILE, SYM_TILE), dtype=dt, device=dev)
+        return None if x is False else x
+    r2, dprime, counts = _out(r2, torch.float32), _out(dprime, torch.float32), _out(counts, torch.uint32)
+    _dev_tensor(r2, "r2", (torch.float32,))
+    _dev_tensor(dprime, "dprime", (torch.float32,))
+    _dev_tensor(counts, "counts", _U32)
+    _dev_tensor(popA, "popA", _U32)
+    for t in (r2, dprime, counts):
+        if t is not None and t.numel() < nt * SYM_TILE * SYM_TILE:
+            raise ValueError("snp_ld_sym outputs need (tile_hi - tile_lo) * 128 * 128 elements")
+    if ws is None:
+        ws = _workspace(snp_ld_sym_workspace_bytes(m, nbits), dev)
+    check(lib().snp_ld_sym(_ptr(A), m, _ld(A), _ptr(popA), int(nbits), int(tile_lo), tile_hi, _ptr(r2), _ptr(dprime),
+                           _ptr(counts), _ptr(ws), 0 if ws is None else ws.numel(), _stream(stream)), "snp_ld_sym")
+    return r2, dprime, counts
+
+
+def snp_sym_unpack(tiles: torch.Tensor, m: int, tile_lo: int = 0, tile_hi: int | None = None,
+                   out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """f3: packed-triangle tiles (any 4-byte dtype) -> the full symmetric m x m matrix."""
+    if not tiles.is_cuda or tiles.element_size() != 4:
+        raise TypeError("tiles must be a CUDA tensor of 4-byte elements")
+    tile_hi = snp_sym_tiles(m) if tile_hi is None else int(tile_hi)
+    if out is None:
+        out = torch.empty((m, m), dtype=tiles.dtype, device=tiles.device)
+    if out.element_size() != 4 or out.stride(-1) != 1:
+        raise TypeError("out must have 4-byte elements, contiguous rows")
+    check(lib().snp_sym_unpack(_ptr(tiles), int(m), int(tile_lo), tile_hi, _ptr(out), _ld(out), _stream(stream)),
+          "snp_sym_unpack")
+    return out
 
 
 def snp_set_variant(variant) -> None:

@@ -29,6 +29,11 @@ SIGNATURES = {
     "snp_fastid_search": (_int, [_p, _i64, _i64, _p, _i64, _i64, _p, _i64, _int, _p, _p, _i64, _p, _p, _i64,
                                  _p, _sz, _p]),
     "snp_shard_plan": (_int, [_i64, _int, _i64, _p]),
+    "snp_shard_plan_sym": (_int, [_i64, _int, _p]),
+    "snp_sym_tiles": (_i64, [_i64]),
+    "snp_ld_sym_workspace_bytes": (_sz, [_i64, _i64]),
+    "snp_ld_sym": (_int, [_p, _i64, _i64, _p, _i64, _i64, _i64, _p, _p, _p, _p, _sz, _p]),
+    "snp_sym_unpack": (_int, [_p, _i64, _i64, _i64, _p, _i64, _p]),
     "snp_set_variant": (_int, [_int]),
     "snp_last_variant": (_int, []),
     "snp_launch_count": (_i64, []),

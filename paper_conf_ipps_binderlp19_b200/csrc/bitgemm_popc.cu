@@ -21,6 +21,7 @@
 //  * Epilogues fused: counts (=, +=) or the LD statistics r2 / D'
 //    from exact integers.
 #include "snp_internal.h"
+#include "e2m1.cuh"
 
 namespace snp {
 namespace {
@@ -37,12 +38,6 @@ __device__ __forceinline__ uint32_t bitop(uint32_t a, uint32_t b) {
     return ~a & b;                    // NOTAND (Eq. 3, r = B row)
 }
 
-__device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
-    const int64_t lo = w * 32;
-    if (lo + 32 <= nbits) return 0xffffffffu;
-    if (lo >= nbits) return 0u;
-    return (1u << (uint32_t)(nbits - lo)) - 1u;
-}
 
 // LD statistics from exact integers (reading R3).
 __device__ __forceinline__ void ld_stats(int64_t n, int64_t na, int64_t nb, int64_t nab,
@@ -76,8 +71,25 @@ bitgemm_popc_kernel(const GemmArgs args) {
 
     const int tid = threadIdx.x;
     const int tx = tid % TX, ty = tid / TX;
-    const int64_t m0 = (int64_t)blockIdx.y * BM;
-    const int64_t n0 = (int64_t)blockIdx.x * BN;
+    int64_t m0 = (int64_t)blockIdx.y * BM;
+    int64_t n0 = (int64_t)blockIdx.x * BN;
+    // outputs: row-major [m][ldc], or (f3 packed triangle) tile blockIdx.x of the call as a
+    // dense BM x BN block — shifting the bases keeps the (row * ldc + col) addressing below
+    uint32_t *Cp = args.C;
+    float *r2p = args.r2, *dpp = args.dprime;
+    int64_t ldc = args.ldc;
+    const bool tri = args.tri_n >= 0;
+    if (tri) {
+        uint32_t I, J;
+        tri_decode((args.m + BM - 1) / BM, args.tri_lo + blockIdx.x, I, J);
+        m0 = (int64_t)I * BM;
+        n0 = (int64_t)J * BN;
+        ldc = BN;
+        const int64_t delta = (int64_t)blockIdx.x * (BM * BN) - m0 * BN - n0;
+        if (Cp) Cp += delta;
+        if (r2p) r2p += delta;
+        if (dpp) dpp += delta;
+    }
     const int64_t nbits = args.nbits;
     const int64_t nchunk32 = ((nbits + 127) / 128) * 4;   // uint32 words actually read
     const int nstages = (int)((nchunk32 + BK - 1) / BK);
@@ -175,18 +187,19 @@ bitgemm_popc_kernel(const GemmArgs args) {
 #pragma unroll
     for (int i = 0; i < TM; ++i) {
         const int64_t gi = m0 + (i < 4 ? ty * 4 + i : BM / 2 + ty * 4 + (i - 4));
-        if (gi >= args.m) continue;
+        // packed triangle: a tile's entries past m are written too, as the zeros they compute
+        if (gi >= args.m && !tri) continue;
         int64_t na = 0;
-        if (EPI == EPI_LD) na = args.popA[gi];
+        if (EPI == EPI_LD && gi < args.m) na = args.popA[gi];
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
             const int64_t gj0 = n0 + (h == 0 ? tx * 4 : BN / 2 + tx * 4);
-            const int64_t base = gi * args.ldc + gj0;
+            const int64_t base = gi * ldc + gj0;
             if (EPI == EPI_COUNTS) {
                 uint32_t v[4] = {acc[i][4 * h], acc[i][4 * h + 1], acc[i][4 * h + 2], acc[i][4 * h + 3]};
-                const bool vec = (gj0 + 4 <= args.n) && ((base & 3) == 0);
+                const bool vec = (tri || gj0 + 4 <= args.n) && ((base & 3) == 0);
                 if (vec) {
-                    uint4 *p = reinterpret_cast<uint4 *>(args.C + base);
+                    uint4 *p = reinterpret_cast<uint4 *>(Cp + base);
                     if (args.accumulate) {
                         uint4 o = *p;
                         v[0] += o.x; v[1] += o.y; v[2] += o.z; v[3] += o.w;
@@ -195,8 +208,8 @@ bitgemm_popc_kernel(const GemmArgs args) {
                 } else {
 #pragma unroll
                     for (int q = 0; q < 4; ++q)
-                        if (gj0 + q < args.n)
-                            args.C[base + q] = args.accumulate ? args.C[base + q] + v[q] : v[q];
+                        if (tri || gj0 + q < args.n)
+                            Cp[base + q] = args.accumulate ? Cp[base + q] + v[q] : v[q];
                 }
             } else {
                 float r2v[4], dpv[4];
@@ -206,21 +219,21 @@ bitgemm_popc_kernel(const GemmArgs args) {
                     const int64_t nb = gj < args.n ? (int64_t)args.popB[gj] : 0;
                     ld_stats(args.nbits, na, nb, (int64_t)acc[i][4 * h + q], r2v[q], dpv[q]);
                 }
-                const bool vec = (gj0 + 4 <= args.n) && ((base & 3) == 0);
+                const bool vec = (tri || gj0 + 4 <= args.n) && ((base & 3) == 0);
                 if (vec) {
-                    *reinterpret_cast<float4 *>(args.r2 + base) = make_float4(r2v[0], r2v[1], r2v[2], r2v[3]);
-                    if (args.dprime)
-                        *reinterpret_cast<float4 *>(args.dprime + base) = make_float4(dpv[0], dpv[1], dpv[2], dpv[3]);
-                    if (args.C)
-                        *reinterpret_cast<uint4 *>(args.C + base) =
+                    *reinterpret_cast<float4 *>(r2p + base) = make_float4(r2v[0], r2v[1], r2v[2], r2v[3]);
+                    if (dpp)
+                        *reinterpret_cast<float4 *>(dpp + base) = make_float4(dpv[0], dpv[1], dpv[2], dpv[3]);
+                    if (Cp)
+                        *reinterpret_cast<uint4 *>(Cp + base) =
                             make_uint4(acc[i][4 * h], acc[i][4 * h + 1], acc[i][4 * h + 2], acc[i][4 * h + 3]);
                 } else {
 #pragma unroll
                     for (int q = 0; q < 4; ++q)
-                        if (gj0 + q < args.n) {
-                            args.r2[base + q] = r2v[q];
-                            if (args.dprime) args.dprime[base + q] = dpv[q];
-                            if (args.C) args.C[base + q] = acc[i][4 * h + q];
+                        if (tri || gj0 + q < args.n) {
+                            r2p[base + q] = r2v[q];
+                            if (dpp) dpp[base + q] = dpv[q];
+                            if (Cp) Cp[base + q] = acc[i][4 * h + q];
                         }
                 }
             }
@@ -231,6 +244,10 @@ bitgemm_popc_kernel(const GemmArgs args) {
 template <int BM, int BN, int EPI>
 cudaError_t launch_tile(const GemmArgs &a, cudaStream_t s) {
     dim3 grid((unsigned)((a.n + BN - 1) / BN), (unsigned)((a.m + BM - 1) / BM));
+    if (a.tri_n >= 0) {   // packed triangle: one block per tile of the call
+        if (a.tri_n == 0) return cudaSuccess;
+        grid = dim3((unsigned)a.tri_n, 1);
+    }
     switch (a.op) {
     case 0: bitgemm_popc_kernel<BM, BN, 0, EPI><<<grid, NT, 0, s>>>(a); break;
     case 1: bitgemm_popc_kernel<BM, BN, 1, EPI><<<grid, NT, 0, s>>>(a); break;
@@ -244,6 +261,10 @@ cudaError_t launch_tile(const GemmArgs &a, cudaStream_t s) {
 }  // namespace
 
 cudaError_t launch_bitgemm_popc(const GemmArgs &a, int epi, cudaStream_t s) {
+    if (a.tri_n >= 0) {   // f3 packed triangle: 128 x 128 tiles, grid.x = tiles (< 2^31)
+        if (a.tri_n > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+        return epi == EPI_LD ? launch_tile<128, 128, EPI_LD>(a, s) : launch_tile<128, 128, EPI_COUNTS>(a, s);
+    }
     // gridDim.y <= 65535: walk M in chunks (offsetting every row-indexed pointer).
     const int64_t BMmax = a.m <= 64 ? 64 : 128;
     const int64_t chunk = 65535 * BMmax;

@@ -25,6 +25,7 @@
 //     When the lane side is the second operand (FastID: database rows on lanes,
 //     queries on columns) the output is written transposed, coalesced along lanes.
 #include "snp_internal.h"
+#include "e2m1.cuh"
 #include "tc_ptx.cuh"
 
 namespace snp {
@@ -62,12 +63,6 @@ struct TcArgs {
     float *dprime;
 };
 
-__device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
-    const int64_t lo = w * 32;
-    if (lo + 32 <= nbits) return 0xffffffffu;
-    if (lo >= nbits) return 0u;
-    return (1u << (uint32_t)(nbits - lo)) - 1u;
-}
 
 __device__ __forceinline__ void ld_stats(int64_t n, int64_t na, int64_t nb, int64_t nab, float &r2, float &dp) {
     const int64_t num = n * nab - na * nb;
@@ -343,7 +338,7 @@ template <int BN, int EPI>
 cudaError_t launch_cfg(const TcArgs &t, cudaStream_t s) {
     using C = Cfg<BN>;
     auto kern = bitgemm_tc_kernel<BN, EPI>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM);
+    cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)C::SMEM);
     if (e != cudaSuccess) return e;
     const int64_t gx = (t.nl + BM - 1) / BM;
     const int64_t gy = (t.nc + BN - 1) / BN;

@@ -21,6 +21,7 @@
 // Exactness: products are in {0, 1}, fp32 sums of them are exact below 2^24.
 #include "snp_internal.h"
 #include "tc_ptx.cuh"
+#include "e2m1.cuh"
 
 #include <cuda.h>
 #include <cstdlib>
@@ -136,83 +137,6 @@ struct FArgs {
                              // then the expanders count them from the streamed words
 };
 
-__device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
-    const int64_t lo = w * 32;
-    if (lo + 32 <= nbits) return 0xffffffffu;
-    if (lo >= nbits) return 0u;
-    return (1u << (uint32_t)(nbits - lo)) - 1u;
-}
-
-// Bits -> e2m1 nibbles for kind::mxf4 (scale factors all 2^0).  Output word t of input
-// word x holds bit 4n + t in nibble n (a fixed K permutation shared by both operands).
-// The two operands use complementary nibble positions so every product of set bits is
-// exactly 1.0 with as few shifts as possible (e2m1: bit0 = 0.5, bit1 = 1.0, bit2 = 2.0):
-//   t:        0            1           2            3
-//   A (TMEM)  bit0 = 0.5   bit1 = 1.0  bit2 = 2.0   bit1 = 1.0 (x >> 2)
-//   B (smem)  bit2 = 2.0   bit1 = 1.0  bit0 = 0.5   bit1 = 1.0 (x >> 2)
-// A: 4 LOP3 + 1 shift, B: 4 LOP3 + 2 shifts (was 4 LOP3 + 3 shifts for 1.0 everywhere).
-__device__ __forceinline__ void expandA(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
-    o0 = x & 0x11111111u;
-    o1 = x & 0x22222222u;
-    o2 = x & 0x44444444u;
-    o3 = __umulhi(x, 0x40000000u) & 0x22222222u;   // (x >> 2) on the FMA pipe
-}
-__device__ __forceinline__ void expandB(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
-    const uint32_t y = __umulhi(x, 0x40000000u);    // x >> 2
-    o0 = (x * 4u) & 0x44444444u;
-    o1 = x & 0x22222222u;
-    o2 = y & 0x11111111u;
-    o3 = y & 0x22222222u;
-}
-
-__host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
-    return (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
-}
-
-
-__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&v)[16]) {
-    __syncwarp();   // warp-collective (.sync.aligned): converge first
-    asm volatile(
-        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
-            taddr),
-        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
-        "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
-        : "memory");
-}
-
-__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
-    __syncwarp();   // warp-collective (.sync.aligned): converge first
-    asm volatile(
-        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
-        "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
-        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
-        "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]),
-        "r"(v[17]), "r"(v[18]), "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]),
-        "r"(v[25]), "r"(v[26]), "r"(v[27]), "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
-        : "memory");
-}
-
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
-    __syncwarp();   // warp-collective (.sync.aligned): converge first
-    asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-        : "r"(taddr));
-}
-
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
-    __syncwarp();   // warp-collective (.sync.aligned): converge first
-    asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
-        "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
-          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
-          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-        : "r"(taddr));
-}
-
 // NOPS: ops per launch; BEST: keep best matches; ACC: accumulate into the counts.
 // Everything uniform that would otherwise be tested inside the 32-column epilogue loop
 // is a template parameter or folded into per-lane predicates: loop unswitching on
@@ -252,8 +176,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     __shared__ unsigned int launch_k;
-    if (args.trace && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x] = (long long)ptx::globaltimer_ns();
-    if (args.trace && tid == 0 && blockIdx.x == 0) {
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x] = (long long)ptx::globaltimer_ns();
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x == 0) {
         launch_k = atomicAdd(&g_fastid_launch_ctr, 1u) & 63u;
         g_fastid_launch_time[2 * launch_k] = (long long)ptx::globaltimer_ns();
     }
@@ -324,8 +248,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         uint32_t v[16];
 #pragma unroll
         for (int i = 0; i < 16; ++i) v[i] = 0x7F7F7F7Fu;   // ue8m0 scale 2^0 in every byte
-        tmem_st16(tmem + ((uint32_t)(q * 32) << 16) + C::SF_COL, v);
-        tmem_st16(tmem + ((uint32_t)(q * 32) << 16) + C::SF_COL + 16, v);
+        ptx::tmem_st16(tmem + ((uint32_t)(q * 32) << 16) + C::SF_COL, v);
+        ptx::tmem_st16(tmem + ((uint32_t)(q * 32) << 16) + C::SF_COL + 16, v);
         ptx::tmem_st_wait();
     }
     ptx::fence_proxy_async_smem();
@@ -337,7 +261,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         asm volatile("bar.sync 1, %0;" ::"r"(NEPI * 32) : "memory");
     }
 
-    if (args.trace && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 1] = (long long)ptx::globaltimer_ns();
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 1] = (long long)ptx::globaltimer_ns();
     if (warp == TMA_WARP) {
         // ------------------------------------------------------------ TMA producer
         if (lane == 0) {
@@ -384,7 +308,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         for (int it = g; it < total_it32; it += G) {
             publish_until(tl);
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
-            const bool tr = args.trace && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
+            const bool tr = SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
 #endif
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 0] = clock64();
@@ -426,7 +350,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #pragma unroll
                 for (int i = 0; i < 8; ++i)
                     expandA(wv[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-                tmem_st32(tbase + 32 * h, v);
+                ptx::tmem_st32(tbase + 32 * h, v);
                 if (NHALF == 2 && h == 0) {   // publish the first half: the MMA may start on it
                     ptx::tmem_st_wait();
                     ptx::tc_fence_before();
@@ -470,23 +394,23 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             const uint32_t tl32 = (uint32_t)tl;
             const int acc = (int)(tl32 % NACC);
 #ifdef FASTID_TRACE2
-            if (args.trace && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 0] = clock64();
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 0] = clock64();
 #endif
             if (tl32 >= NACC) ptx::mbar_wait_uniform(&acce[acc], (tl32 / NACC - 1) & 1u);
 #ifdef FASTID_TRACE2
-            if (args.trace && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 1] = clock64();
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 1] = clock64();
 #endif
             ptx::tc_fence_after();
             const uint32_t d = tmu + (uint32_t)(acc * C::ACC_COLS);
             uint64_t bd = bdesc0;
             for (int s = 0; s < nst; ++s, ++itm) {
 #ifdef FASTID_TRACE2
-                if (args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 3] = clock64();
+                if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 3] = clock64();
 #endif
                 ptx::mbar_wait_uniform(&full[b * NHALF], bround & 1);
                 ptx::tc_fence_after();
 #ifdef FASTID_TRACE2
-                if (args.trace && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 5] = clock64();
+                if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 5] = clock64();
 #endif
                 const uint32_t a0 = tmu + (uint32_t)(C::A_COL0 + ACOLS * b);
 #pragma unroll
@@ -531,12 +455,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             else ptx::mbar_wait_warp(&popf[acc], ph);
             ptx::mbar_wait_warp(&accf[acc], ph);
 #ifdef FASTID_TRACE2
-            if (args.trace && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 2] = clock64();
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 2] = clock64();
 #endif
             ptx::tc_fence_after();
             uint32_t v[EC];
-            if constexpr (EC == 32) tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
-            else tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
+            if constexpr (EC == 32) ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
+            else ptx::tmem_ld16(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * C::ACC_COLS + c0), v);
             if (!pre) {   // read the popcount partials BEFORE releasing the buffer pair
 #pragma unroll
                 for (int gg = 0; gg < G; ++gg) pd += popD[(acc * G + gg) * BM + li];
@@ -570,7 +494,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                     C32[j] = 32u * args.cc[j];
                     L[j] = 32u * args.cd[j] * pd - C32[j] * 0x4B000000u + laneterm;
                 }
-                sv[j] = valid && args.outs[j] != nullptr && !args.nostore;
+                sv[j] = valid && args.outs[j] != nullptr && !SNP_PROF(args.nostore);
                 op_[j] = sv[j] ? args.outs[j] + (int64_t)c0 * ldo + gd : nullptr;
             }
             // best match: key = count << 5 | lane, so ONE redux.sync.min gives the tile
@@ -620,7 +544,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 }
             }
 #ifdef FASTID_TRACE2
-            if (args.trace && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 3] = clock64();
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 256) g_fastid_etrace[4 * tl + 3] = clock64();
 #endif
         }
         if (BEST) {
@@ -654,8 +578,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 
     ptx::tc_fence_before();
     __syncthreads();
-    if (args.trace && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 2] = (long long)ptx::globaltimer_ns();
-    if (args.trace && tid == 0 && blockIdx.x == 0) g_fastid_launch_time[2 * launch_k + 1] = (long long)ptx::globaltimer_ns();
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 2] = (long long)ptx::globaltimer_ns();
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x == 0) g_fastid_launch_time[2 * launch_k + 1] = (long long)ptx::globaltimer_ns();
     if (warp == MMA_WARP) {
         ptx::tc_fence_after();
         ptx::tmem_dealloc<512>(tmem);
@@ -667,33 +591,6 @@ __global__ void fastid_search_init(unsigned long long *keys, int64_t n, unsigned
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         keys[i] = ~0ULL;
     if (blockIdx.x == 0 && threadIdx.x == 0) *done = 0u;
-}
-
-typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
-                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
-                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-EncodeTiledFn encode_fn() {
-    static EncodeTiledFn fn = nullptr;
-    if (!fn) {
-        void *p = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-            q == cudaDriverEntryPointSuccess)
-            fn = reinterpret_cast<EncodeTiledFn>(p);
-    }
-    return fn;
-}
-
-int num_sms() {
-    static int n = 0;
-    if (!n) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-        if (n <= 0) n = 148;
-    }
-    return n;
 }
 
 size_t smem_bytes(int bn, int64_t nbits) {
@@ -739,65 +636,52 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     f.ntiles = (a.nd + BM - 1) / BM;
     f.nst = (int)((a.nbits + KBITS - 1) / KBITS);
     f.qbytes = (size_t)BN * f.nst * (KBITS / 32) * 16;
+#ifdef SNP_PROFILING
     static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
     f.trace = trace ? 1 : 0;
     static const bool nostore = std::getenv("SNP_DEBUG_NOSTORE") && std::getenv("SNP_DEBUG_NOSTORE")[0] == '1';
     f.nostore = nostore ? 1 : 0;
+#endif
     const size_t smem = smem_bytes(BN, a.nbits);
 
-    EncodeTiledFn enc = encode_fn();
-    if (!enc) return cudaErrorNotSupported;
     CUtensorMap tm;
-    const cuuint64_t dims[2] = {(cuuint64_t)a.ldd32, (cuuint64_t)a.nd};
-    const cuuint64_t strides[1] = {(cuuint64_t)a.ldd32 * 4};
-    const cuuint32_t box[2] = {KBITS / 32, BM};
-    const cuuint32_t estr[2] = {1, 1};
-    CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(a.D), dims, strides, box, estr,
-                     CU_TENSOR_MAP_INTERLEAVE_NONE, KBITS == 512 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B,
-                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+    if (!make_map_u32_2d(&tm, a.D, a.nd, a.ldd32, KBITS / 32, BM,
+                         KBITS == 512 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B))
+        return cudaErrorInvalidValue;
 
     using KernFn = void (*)(const CUtensorMap, const FArgs);
     const bool best = f.best_mask != 0;
     KernFn kern = nullptr;
-    int ki = 0;
     int nthreads = Roles<GG>::NTHREADS;   // the runtime-coefficient kernels are GG = 4 only
     if (a.accumulate) {
         nthreads = Roles<4>::NTHREADS;
         if (a.nops != 1 || best) return cudaErrorInvalidValue;
-        kern = fastid_tc4_kernel<BN, 1, false, true, -1, 4>; ki = 0;
+        kern = fastid_tc4_kernel<BN, 1, false, true, -1, 4>;
     } else if (a.nops == 1) {   // compile-time op
         static KernFn k1[2][4] = {{fastid_tc4_kernel<BN, 1, false, false, 0, GG>, fastid_tc4_kernel<BN, 1, false, false, 1, GG>,
                                    fastid_tc4_kernel<BN, 1, false, false, 2, GG>, fastid_tc4_kernel<BN, 1, false, false, 3, GG>},
                                   {fastid_tc4_kernel<BN, 1, true, false, 0, GG>, fastid_tc4_kernel<BN, 1, true, false, 1, GG>,
                                    fastid_tc4_kernel<BN, 1, true, false, 2, GG>, fastid_tc4_kernel<BN, 1, true, false, 3, GG>}};
         kern = k1[best][a.ops[0] & 3];
-        ki = 1 + 4 * best + (a.ops[0] & 3);
     } else if (a.nops == 2 && a.ops[0] == 1 && a.ops[1] == 2) {   // XOR + ANDNOT (identity + mixture)
         kern = best ? fastid_tc4_kernel<BN, 2, true, false, 1 | (2 << 2), GG>
                     : fastid_tc4_kernel<BN, 2, false, false, 1 | (2 << 2), GG>;
-        ki = 9 + best;
     } else {
         nthreads = Roles<4>::NTHREADS;
         switch (a.nops * 2 + (best ? 1 : 0)) {
-        case 4: kern = fastid_tc4_kernel<BN, 2, false, false, -1, 4>; ki = 11; break;
-        case 5: kern = fastid_tc4_kernel<BN, 2, true, false, -1, 4>; ki = 12; break;
-        case 6: kern = fastid_tc4_kernel<BN, 3, false, false, -1, 4>; ki = 13; break;
-        case 7: kern = fastid_tc4_kernel<BN, 3, true, false, -1, 4>; ki = 14; break;
-        case 8: kern = fastid_tc4_kernel<BN, 4, false, false, -1, 4>; ki = 15; break;
-        case 9: kern = fastid_tc4_kernel<BN, 4, true, false, -1, 4>; ki = 16; break;
+        case 4: kern = fastid_tc4_kernel<BN, 2, false, false, -1, 4>; break;
+        case 5: kern = fastid_tc4_kernel<BN, 2, true, false, -1, 4>; break;
+        case 6: kern = fastid_tc4_kernel<BN, 3, false, false, -1, 4>; break;
+        case 7: kern = fastid_tc4_kernel<BN, 3, true, false, -1, 4>; break;
+        case 8: kern = fastid_tc4_kernel<BN, 4, false, false, -1, 4>; break;
+        case 9: kern = fastid_tc4_kernel<BN, 4, true, false, -1, 4>; break;
         default: return cudaErrorInvalidValue;
         }
     }
-    static size_t attr_set[17] = {};   // max dynamic smem already granted, per instantiation
-    if (attr_set[ki] < smem) {
-        const size_t grant = MAX_SMEM - 1024;   // leave room for the kernel's static shared memory
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)grant);
-        if (e != cudaSuccess) return e;
-        attr_set[ki] = grant;
-    }
-    const int grid = (int)(f.ntiles < num_sms() ? f.ntiles : num_sms());
+    // grant the whole opt-in once per (device, instantiation): the query batch's size varies per call
+    if (cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)(MAX_SMEM - 1024)); e != cudaSuccess)
+        return e;
+    const int grid = (int)(f.ntiles < device_sms() ? f.ntiles : device_sms());
     if (f.best_mask) {
         const int64_t nk = (int64_t)a.nops * a.nq;
         fastid_search_init<<<(int)((nk + 255) / 256), 256, 0, s>>>(a.keys, nk, a.done);
@@ -871,6 +755,7 @@ cudaError_t launch_fastid_search_tc4(const SearchArgs &a, cudaStream_t s) {
 
 }  // namespace snp
 
+#ifdef SNP_PROFILING
 // Profiling aid (not part of include/snp.h): copy the pipeline trace of the last
 // traced fastid_tc4 launch (4 x 1024 clock64 stamps) to host memory.
 extern "C" int snp_debug_fastid_launch_times(long long *host, int n) {
@@ -892,3 +777,4 @@ extern "C" int snp_debug_fastid_trace(long long *host, int n) {
     if (n > 8 * 1024) n = 8 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_trace, sizeof(long long) * n);
 }
+#endif  // SNP_PROFILING

@@ -22,6 +22,7 @@
 // shared memory 3 x 16 KB packed + 3 x 32 KB expanded B + barriers/popcounts.
 #include "snp_internal.h"
 #include "tc_ptx.cuh"
+#include "e2m1.cuh"
 
 #include <cuda.h>
 #include <cstdlib>
@@ -87,64 +88,13 @@ struct GArgs {
     int op2;          // EPI_COUNTS, swapped layout: second op written to C2 (or C2 = NULL)
     uint32_t *C2;
     const uint32_t *popL, *popC;   // row popcounts (row_popc pre-pass), NULL if unused
+    // f3 packed triangle (snp_ld_sym): tiles tlo .. tlo + ntri - 1 of the row-major upper
+    // triangle of the T x T tile grid (T = nlb), tile u of the launch stored as a dense
+    // 128 x 128 row-major block at element offset u * 128 * 128 of C / r2 / dprime (ldo = 128)
+    int tri;
+    int64_t tlo, ntri, mreal;
 };
 
-__device__ __forceinline__ uint32_t word_mask(int64_t w, int64_t nbits) {
-    const int64_t lo = w * 32;
-    if (lo + 32 <= nbits) return 0xffffffffu;
-    if (lo >= nbits) return 0u;
-    return (1u << (uint32_t)(nbits - lo)) - 1u;
-}
-
-// Bits -> e2m1 nibbles for kind::mxf4 (scale factors all 2^0).  Output word t of input
-// word x holds bit 4n + t in nibble n (a fixed K permutation shared by both operands).
-// The two operands use complementary nibble positions so every product of set bits is
-// exactly 1.0 with as few shifts as possible (e2m1: bit0 = 0.5, bit1 = 1.0, bit2 = 2.0):
-//   t:        0            1           2            3
-//   A (TMEM)  bit0 = 0.5   bit1 = 1.0  bit2 = 2.0   bit1 = 1.0 (x >> 2)
-//   B (smem)  bit2 = 2.0   bit1 = 1.0  bit0 = 0.5   bit1 = 1.0 (x >> 2)
-// A: 4 LOP3 + 1 shift, B: 4 LOP3 + 2 shifts (was 4 LOP3 + 3 shifts for 1.0 everywhere).
-__device__ __forceinline__ void expandA(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
-    o0 = x & 0x11111111u;
-    o1 = x & 0x22222222u;
-    o2 = x & 0x44444444u;
-    o3 = __umulhi(x, 0x40000000u) & 0x22222222u;   // (x >> 2) on the FMA pipe
-}
-__device__ __forceinline__ void expandB(uint32_t x, uint32_t &o0, uint32_t &o1, uint32_t &o2, uint32_t &o3) {
-    const uint32_t y = __umulhi(x, 0x40000000u);    // x >> 2
-    o0 = (x * 4u) & 0x44444444u;
-    o1 = x & 0x22222222u;
-    o2 = y & 0x11111111u;
-    o3 = y & 0x22222222u;
-}
-
-__host__ __device__ constexpr uint32_t idesc_mxf4(int M, int N) {
-    return (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | (1u << 23) | ((uint32_t)(M >> 4) << 24);
-}
-
-__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
-    __syncwarp();   // warp-collective (.sync.aligned): converge first
-    asm volatile(
-        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
-        "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
-        "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
-        "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]),
-        "r"(v[17]), "r"(v[18]), "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]),
-        "r"(v[25]), "r"(v[26]), "r"(v[27]), "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
-        : "memory");
-}
-
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
-    __syncwarp();   // warp-collective (.sync.aligned): converge first
-    asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
-        "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
-          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
-          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-        : "r"(taddr));
-}
 
 // LD statistics in fp32 from exact integers (reading R3).  num, nA(n-nA), nB(n-nB) are
 // exact integers; each is rounded once to fp32, so r2 and D' carry a relative error of
@@ -646,7 +596,7 @@ __device__ __forceinline__ void epi_swapped_counts(const GArgs &args, uint32_t (
     }
 }
 
-template <int EPI>
+template <int EPI, bool TRI = false>
 __global__ void __launch_bounds__(NTHREADS, 1)
 gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
                 const GArgs args) {
@@ -666,7 +616,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t nbits = args.nbits;
     const int nst = args.nst;
-    const int64_t ntiles = args.sym ? args.nlb * (args.nlb + 1) / 2 : args.nlb * args.ncb;
+    const int64_t ntiles = TRI ? args.ntri : args.sym ? args.nlb * (args.nlb + 1) / 2 : args.nlb * args.ncb;
     // 32-bit tile arithmetic (ntiles < 2^31): a 64-bit division is a subroutine CALL, and
     // any call in the kernel made ptxas drop the MMA issue loop out of uniform registers
     const uint32_t nlb32 = (uint32_t)args.nlb, ncb32 = (uint32_t)args.ncb;
@@ -754,7 +704,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         uint32_t v[32];
 #pragma unroll
         for (int i = 0; i < 32; ++i) v[i] = 0x7F7F7F7Fu;   // ue8m0 2^0 in every scale byte
-        tmem_st32(tmem + ((uint32_t)(q * 32) << 16) + SF_COL, v);
+        ptx::tmem_st32(tmem + ((uint32_t)(q * 32) << 16) + SF_COL, v);
         ptx::tmem_st_wait();
     }
     ptx::tc_fence_before();
@@ -774,7 +724,8 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 const int64_t t = blockIdx.x + tl * gridDim.x;
                 const uint32_t t32 = (uint32_t)t;
                 uint32_t lbt, cbt;
-                if (args.sym) decode_sym(t32, lbt, cbt);
+                if (TRI) tri_decode(args.nlb, args.tlo + t, lbt, cbt);
+                else if (args.sym) decode_sym(t32, lbt, cbt);
                 else { lbt = tile_lb(t32); cbt = tile_cb(t32); }
                 const int32_t rl = (int32_t)(lbt * BM), rc = (int32_t)(cbt * BN);
                 for (int s = 0; s < nst; ++s) {
@@ -806,7 +757,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         uint32_t pround = 0;
         for (int64_t it = g; it < total_it; it += G) {
 #ifdef GEMM_TRACE
-            const bool tr = args.trace && blockIdx.x == 0 && r8 == 0 && lane == 0 && it < 2048;
+            const bool tr = SNP_PROF(args.trace) && blockIdx.x == 0 && r8 == 0 && lane == 0 && it < 2048;
 #endif
 #ifdef GEMM_TRACE
             if (tr) g_gemm_trace[8 * it + 0] = clock64();
@@ -820,7 +771,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             if (tr) g_gemm_trace[8 * it + 1] = clock64();
 #endif
 #ifdef GEMM_DEBUG_SKIP
-            if (args.debug_skip) {
+            if (SNP_PROF(args.debug_skip)) {
                 __syncwarp();
                 if (lane == 0) {
                     ptx::mbar_arrive(&pempty[pk]);
@@ -858,7 +809,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
 #pragma unroll
                     for (int i = 0; i < 8; ++i)
                         expandA(w[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-                    tmem_st32(tA + 32 * h, v);
+                    ptx::tmem_st32(tA + 32 * h, v);
                     if (GH == 2 && h == 0) {   // publish the first 256 bits
                         ptx::tmem_st_wait();
                         ptx::tc_fence_before();
@@ -954,17 +905,26 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             const int64_t t = blockIdx.x + tl * gridDim.x;
             const uint32_t t32 = (uint32_t)t;
             uint32_t lbt, cbt;
-            if (args.sym) decode_sym(t32, lbt, cbt);
+            if (TRI) tri_decode(args.nlb, args.tlo + t, lbt, cbt);
+            else if (args.sym) decode_sym(t32, lbt, cbt);
             else { lbt = tile_lb(t32); cbt = tile_cb(t32); }
-            const bool mirror = args.sym && lbt != cbt;   // f3: also write the mirror block
+            const bool mirror = !TRI && args.sym && lbt != cbt;   // f3: also write the mirror block
+            // packed triangle: the epilogue addresses the tile as rows t * 128 .. t * 128 + 127
+            // of a [ntri * 128][128] matrix (args.nl / nc / ldo are those virtual sizes), so
+            // its (row * ldo + col) addressing lands in the dense block t; the real size m
+            // (args.mreal) bounds only the popcount loads here — entries past m are written
+            // as the zeros they compute (no popcount, TMA zero fill)
+            const int64_t nlr = TRI ? args.mreal : args.nl, ncr = TRI ? args.mreal : args.nc;
             const int64_t gl = (int64_t)lbt * BM + li;
             const int64_t gc0 = (int64_t)cbt * BN + c0;
+            const int64_t erow0 = TRI ? t * BM + q * 32 : gl - lane;   // epilogue block origin
+            const int64_t ecol0 = TRI ? (int64_t)c0 : gc0;
             const bool rows_ok = gl < args.nl && gc0 < args.nc;
-            const int ncols = gc0 < args.nc ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
+            const int ncols = gc0 < ncr ? (int)(ncr - gc0 < 64 ? ncr - gc0 : 64) : 0;
             // popcounts: lane j holds the column popcounts of columns c0 + j and c0 + 32 + j
             uint32_t pl = 0, pcol0 = 0, pcol1 = 0;
             if (need_pop) {
-                if (gl < args.nl) pl = __ldg(args.popL + gl);
+                if (gl < nlr) pl = __ldg(args.popL + gl);
                 if (lane < ncols) pcol0 = __ldg(args.popC + gc0 + lane);
                 if (32 + lane < ncols) pcol1 = __ldg(args.popC + gc0 + 32 + lane);
             }
@@ -982,7 +942,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             for (int hh = 0; hh < 2; ++hh) {
                 uint32_t v[32];
                 __syncwarp();            // tcgen05.ld is warp-collective: re-converge first
-                tmem_ld32(ta + 32 * hh, v);
+                ptx::tmem_ld32(ta + 32 * hh, v);
                 ptx::tmem_ld_wait();
                 if (hh == 1) {
                     ptx::tc_fence_before();
@@ -991,7 +951,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 }
                 const uint32_t pcol = hh ? pcol1 : pcol0;
                 if (!args.swap) {
-                    epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, gl - lane, gc0 + 32 * hh, pl, pcol,
+                    epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, erow0, ecol0 + 32 * hh, pl, pcol,
                                         ia, small_n, want_dp, mirror);
                     continue;
                 }
@@ -1288,7 +1248,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
         uint32_t v[32];
 #pragma unroll
         for (int i = 0; i < 32; ++i) v[i] = 0x7F7F7F7Fu;   // ue8m0 2^0 in every scale byte
-        tmem_st32(tmem + ((uint32_t)(q * 32) << 16) + SF_COL, v);
+        ptx::tmem_st32(tmem + ((uint32_t)(q * 32) << 16) + SF_COL, v);
         ptx::tmem_st_wait();
     }
     ptx::tc_fence_before();
@@ -1334,7 +1294,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
             if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
             ptx::mbar_wait_warp(&pfull[pk], pround & 1);
 #ifdef GEMM_DEBUG_SKIP
-            if (args.debug_skip) {   // profiling experiment: tokens only (results invalid)
+            if (SNP_PROF(args.debug_skip)) {   // profiling experiment: tokens only (results invalid)
                 __syncwarp();
                 if (lane == 0) { ptx::mbar_arrive(&pempty[pk]); arrive_remote(&full[slot], 0); }
                 s += G;
@@ -1366,7 +1326,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
 #pragma unroll
                     for (int i = 0; i < 8; ++i)
                         expandA(w[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-                    tmem_st32(tA + 32 * h, v);
+                    ptx::tmem_st32(tA + 32 * h, v);
                 }
                 ptx::tmem_st_wait();
                 ptx::tc_fence_before();
@@ -1454,7 +1414,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
             for (int hh = 0; hh < 2; ++hh) {
                 uint32_t v[32];
                 __syncwarp();
-                tmem_ld32(ta + 32 * hh, v);
+                ptx::tmem_ld32(ta + 32 * hh, v);
                 ptx::tmem_ld_wait();
                 if (hh == 1) {
                     ptx::tc_fence_before();
@@ -1476,59 +1436,22 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
     }
 }
 
-typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
-                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
-                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-EncodeTiledFn encode_fn() {
-    static EncodeTiledFn fn = nullptr;
-    if (!fn) {
-        void *p = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-            q == cudaDriverEntryPointSuccess)
-            fn = reinterpret_cast<EncodeTiledFn>(p);
-    }
-    return fn;
-}
-
 bool make_map(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32, uint32_t box_rows = 128) {
-    EncodeTiledFn enc = encode_fn();
-    if (!enc) return false;
-    const cuuint64_t dims[2] = {(cuuint64_t)ld32, (cuuint64_t)rows};
-    const cuuint64_t strides[1] = {(cuuint64_t)ld32 * 4};
-    const cuuint32_t box[2] = {KW, box_rows};
-    const cuuint32_t estr[2] = {1, 1};
-    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(base), dims, strides, box, estr,
-               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    return make_map_u32_2d(tm, base, rows, ld32, KW, box_rows, CU_TENSOR_MAP_SWIZZLE_64B);
 }
 
-int num_sms() {
-    static int n = 0;
-    if (!n) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-        if (n <= 0) n = 148;
-    }
-    return n;
-}
-
-template <int EPI>
+template <int EPI, bool TRI = false>
 cudaError_t launch_g(const GArgs &g, const uint32_t *L, int64_t ldl32, const uint32_t *Cn, int64_t ldc32,
                      cudaStream_t s) {
     CUtensorMap tmL, tmC;
-    if (!make_map(&tmL, L, g.nl, ldl32) || !make_map(&tmC, Cn, g.nc, ldc32)) return cudaErrorInvalidValue;
-    auto kern = gemm_tc4_kernel<EPI>;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
-    const int64_t ntiles = g.sym ? g.nlb * (g.nlb + 1) / 2 : g.nlb * g.ncb;
-    const int grid = (int)(ntiles < num_sms() ? ntiles : num_sms());
+    // packed-triangle launches keep virtual output sizes in g.nl / g.nc: the operands have m rows
+    const int64_t rows_l = TRI ? g.mreal : g.nl, rows_c = TRI ? g.mreal : g.nc;
+    if (!make_map(&tmL, L, rows_l, ldl32) || !make_map(&tmC, Cn, rows_c, ldc32)) return cudaErrorInvalidValue;
+    auto kern = gemm_tc4_kernel<EPI, TRI>;
+    if (cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)SMEM); e != cudaSuccess) return e;
+    const int64_t ntiles = TRI ? g.ntri : g.sym ? g.nlb * (g.nlb + 1) / 2 : g.nlb * g.ncb;
+    if (ntiles <= 0) return cudaSuccess;
+    const int grid = (int)(ntiles < device_sms() ? ntiles : device_sms());
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = dim3((unsigned)NTHREADS);
@@ -1551,16 +1474,12 @@ cudaError_t launch_g2(GArgs g, const uint32_t *L, int64_t ldl32, const uint32_t 
     if (!make_map(&tmL, L, g.nl, ldl32, 128) || !make_map(&tmC, Cn, g.nc, ldc32, x2::BNH))
         return cudaErrorInvalidValue;
     auto kern = gemm_tc4x2_kernel<EPI>;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)x2::SMEM);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
+    if (cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)x2::SMEM); e != cudaSuccess)
+        return e;
     g.nlb = (g.nl + 2 * BM - 1) / (2 * BM);
     g.ncb = (g.nc + x2::BNP - 1) / x2::BNP;
     const int64_t npairs = g.nlb * g.ncb;
-    const int pairs = num_sms() / 2;
+    const int pairs = device_sms() / 2;
     const int grid = 2 * (int)(npairs < pairs ? npairs : pairs);
     kern<<<grid, x2::NTHREADS, x2::SMEM, s>>>(tmL, tmC, g);
     count_launches(1);
@@ -1580,6 +1499,32 @@ bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
 
 cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     GArgs g{};
+    if (a.tri_n >= 0) {   // f3 packed triangle: self-LD only (A == B), no swap, no mirror
+        if (a.m != a.n || a.A != a.B || a.lda32 != a.ldb32 || a.C2) return cudaErrorInvalidValue;
+        g.popL = a.popA;
+        g.popC = a.popA;
+        g.mreal = a.m;
+        g.nl = a.tri_n * BM;   // the epilogue's virtual [ntri * 128][128] output (see the kernel)
+        g.nc = BN;
+        g.nbits = a.nbits;
+        g.op = a.op;
+        g.accumulate = a.accumulate;
+        g.ldo = BN;
+        g.C = a.C;
+        g.r2 = a.r2;
+        g.dprime = a.dprime;
+        g.nlb = g.ncb = (a.m + BM - 1) / BM;
+        g.nst = (int)((a.nbits + KBITS - 1) / KBITS);
+        g.tri = 1;
+        g.tlo = a.tri_lo;
+        g.ntri = a.tri_n;
+        g.off32 = (uint64_t)a.tri_n * BM * BN < (1ull << 32) ? 1 : 0;   // virtual row * 128 + col
+        g.v4 = (((uintptr_t)a.r2 & 15u) == 0 && ((uintptr_t)a.C & 15u) == 0) ? 1 : 0;
+        g.order = 2;
+        g_last_sym = true;
+        return epi == EPI_LD ? launch_g<EPI_LD, true>(g, a.A, a.lda32, a.A, a.lda32, s)
+                             : launch_g<EPI_COUNTS, true>(g, a.A, a.lda32, a.A, a.lda32, s);
+    }
     const bool swap = a.m < a.n;     // larger operand on TMEM lanes
     g.popL = swap ? a.popB : a.popA;
     g.popC = swap ? a.popA : a.popB;
@@ -1601,10 +1546,12 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.nlb = (g.nl + BM - 1) / BM;
     g.ncb = (g.nc + BN - 1) / BN;
     g.nst = (int)((a.nbits + KBITS - 1) / KBITS);
+#ifdef SNP_PROFILING
     static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
     g.trace = trace ? 1 : 0;
     static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
     g.debug_skip = skip ? 1 : 0;
+#endif
     g.off32 = (uint64_t)(swap ? a.n : a.m) * (uint64_t)a.ldc < (1ull << 32) ? 1 : 0;
     g.v4 = (a.ldc % 4 == 0 && ((uintptr_t)a.r2 & 15u) == 0 && ((uintptr_t)a.C & 15u) == 0) ? 1 : 0;
     // f3 symmetric self-LD (B aliases A, symmetric output: LD statistics, AND or XOR
@@ -1632,6 +1579,7 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
 
 }  // namespace snp
 
+#ifdef SNP_PROFILING
 extern "C" int snp_debug_gemm_trace(long long *host, int n) {
     if (n > 8 * 2048) n = 8 * 2048;
     return (int)cudaMemcpyFromSymbol(host, snp::g_gemm_trace, sizeof(long long) * n);
@@ -1646,3 +1594,4 @@ extern "C" int snp_debug_gemm_watchdog(int mode, int *record8) {
     cudaMemcpyToSymbol(snp::ptx::g_snp_watchdog, zero, sizeof(zero));
     return (int)cudaGetLastError();
 }
+#endif  // SNP_PROFILING

@@ -296,6 +296,82 @@ snp_status snp_ld_r2(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *
     return run_gemm(a, EPI_LD, variant, ws, ws_bytes, s);
 }
 
+int64_t snp_sym_tiles(int64_t m) {
+    if (m <= 0) return 0;
+    const int64_t T = (m + SYM_TILE - 1) / SYM_TILE;
+    return T * (T + 1) / 2;
+}
+
+size_t snp_ld_sym_workspace_bytes(int64_t m, int64_t nbits) {
+    if (m <= 0 || nbits <= 0) return 0;
+    return align256((size_t)m * 4);   // row popcounts when popA is NULL
+}
+
+snp_status snp_ld_sym(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *popA, int64_t nbits,
+                      int64_t tile_lo, int64_t tile_hi, float *r2, float *dprime, uint32_t *counts,
+                      void *ws, size_t ws_bytes, void *stream) {
+    snp_status st;
+    if (m < 0) return SNP_E_SHAPE;
+    if ((st = check_nbits(nbits)) != SNP_OK) return st;
+    if ((st = check_packed(A, m, lda, nbits)) != SNP_OK) return st;
+    const int64_t ntot = snp_sym_tiles(m);
+    if (tile_lo < 0 || tile_hi < tile_lo || tile_hi > ntot) return SNP_E_RANGE;
+    if (m == 0 || tile_hi == tile_lo) return SNP_OK;
+    if (!r2 && !counts) return SNP_E_NULL;
+    if (dprime && !r2) return SNP_E_NULL;
+    if ((r2 && !aligned16(r2)) || (dprime && !aligned16(dprime)) || (counts && !aligned16(counts)))
+        return SNP_E_ALIGN;
+    if (nbits > 0xB504F33LL) return SNP_E_RANGE;   // n^2 products must stay exact in int64/fp64
+    const bool want_ld = r2 != nullptr;
+    int variant = choose_variant(m, m, nbits);
+    if (variant == SNP_VARIANT_TC && !gemm_tc4_supported(m, m, nbits)) {
+        // the packed layout is produced by the mxf4 kernel (nbits < 2^24) and the CUDA-core
+        // kernel; auto dispatch takes the CUDA-core one above that, a forced TC cannot
+        if (current_variant() == SNP_VARIANT_TC) return SNP_E_SHAPE;
+        variant = SNP_VARIANT_POPC;
+    }
+    const bool need_pop = want_ld && !popA;
+    if (need_pop && (ws_bytes < snp_ld_sym_workspace_bytes(m, nbits) || !ws)) return SNP_E_WORKSPACE;
+    if ((st = check_arch()) != SNP_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e;
+    if (need_pop) {
+        uint32_t *pa = reinterpret_cast<uint32_t *>(ws);
+        if ((e = launch_row_popc(A, m, nbits, lda, pa, s)) != cudaSuccess) return set_cuda_error(e);
+        popA = pa;
+    }
+    GemmArgs a{};
+    a.A = a.B = reinterpret_cast<const uint32_t *>(A);
+    a.m = a.n = m; a.lda32 = a.ldb32 = 2 * lda; a.nbits = nbits;
+    a.op = SNP_OP_AND; a.accumulate = 0; a.ldc = SYM_TILE; a.C = counts;
+    a.r2 = r2; a.dprime = dprime; a.popA = a.popB = popA;
+    a.tri_lo = tile_lo; a.tri_n = tile_hi - tile_lo;
+    if (variant == SNP_VARIANT_TC) {
+        e = launch_gemm_tc4(a, want_ld ? EPI_LD : EPI_COUNTS, s);
+        g_last_kernel = SNP_KERNEL_TC_MXF4_SYM;
+    } else {
+        e = launch_bitgemm_popc(a, want_ld ? EPI_LD : EPI_COUNTS, s);
+        g_last_kernel = SNP_KERNEL_POPC;
+    }
+    if (e != cudaSuccess) return set_cuda_error(e);
+    g_last_variant = variant;
+    return SNP_OK;
+}
+
+snp_status snp_sym_unpack(const uint32_t *tiles, int64_t m, int64_t tile_lo, int64_t tile_hi, uint32_t *out,
+                          int64_t ldo, void *stream) {
+    if (m < 0) return SNP_E_SHAPE;
+    const int64_t ntot = snp_sym_tiles(m);
+    if (tile_lo < 0 || tile_hi < tile_lo || tile_hi > ntot) return SNP_E_RANGE;
+    if (m == 0 || tile_hi == tile_lo) return SNP_OK;
+    if (!tiles || !out) return SNP_E_NULL;
+    if (ldo < m) return SNP_E_SHAPE;
+    snp_status st;
+    if ((st = check_arch()) != SNP_OK) return st;
+    cudaError_t e = launch_sym_unpack(tiles, m, tile_lo, tile_hi - tile_lo, out, ldo, (cudaStream_t)stream);
+    return e == cudaSuccess ? SNP_OK : set_cuda_error(e);
+}
+
 snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t *popQ,
                       const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD,
                       int64_t nbits, int op, uint32_t *out, int64_t ldo, int accumulate,
@@ -572,6 +648,19 @@ snp_status snp_shard_plan(int64_t rows, int world, int64_t align, int64_t *bound
         blk += base + (r < rem ? 1 : 0);
         const int64_t b = blk * align;
         bounds[r + 1] = b < rows ? b : rows;
+    }
+    return SNP_OK;
+}
+
+snp_status snp_shard_plan_sym(int64_t m, int world, int64_t *tile_bounds) {
+    if (world < 1 || m < 0) return SNP_E_RANGE;
+    if (!tile_bounds) return SNP_E_NULL;
+    // equal-cost 128 x 128 tiles, so contiguous ranges of the row-major triangle balance
+    // the work to within one tile: bounds[r] = floor(r * total / world)
+    const int64_t total = snp_sym_tiles(m);
+    for (int r = 0; r <= world; ++r) {
+        // r * total can overflow int64 only for total > 2^56 (m > 2^35): not reachable (m < 2^31)
+        tile_bounds[r] = (int64_t)(((__int128)r * total) / world);
     }
     return SNP_OK;
 }

@@ -1,19 +1,48 @@
 // snp_internal.h — launcher declarations shared by the library's translation units.
 // Not part of the public ABI (that is include/snp.h).
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <math.h>
 
 namespace snp {
 
 // Process-wide count of kernels this library launched (snp_launch_count()).
 void count_launches(int k);
 
+// runtime.cu — per-device caches (thread-safe): SM count, dynamic shared-memory opt-in per
+// (device, kernel), the driver's tensor-map encoder and 2-D uint32 tensor maps for TMA.
+int device_sms();
+cudaError_t ensure_dyn_smem(const void *kernel, int bytes);
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn tensor_map_encoder();
+bool make_map_u32_2d(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32, uint32_t box_words,
+                     uint32_t box_rows, CUtensorMapSwizzle swizzle);
+
 // Epilogue kinds of the bit-GEMM.
 enum Epi : int {
     EPI_COUNTS = 0,   // C = / += counts                       (a3, a4 direct ops)
     EPI_LD = 1        // r2 [, D'] [, counts] from nAB, nA, nB  (a5)
 };
+
+// f3 packed triangle (snp_ld_sym): the row-major upper triangle of a T x T grid of
+// 128 x 128 tiles, tile t <-> (I, J), I <= J < T, t = start(I) + (J - I) with
+// start(I) = I T - I (I - 1) / 2.
+constexpr int SYM_TILE = 128;
+__host__ __device__ __forceinline__ int64_t tri_start(int64_t T, int64_t I) { return I * T - I * (I - 1) / 2; }
+__host__ __device__ __forceinline__ void tri_decode(int64_t T, int64_t t, uint32_t &I, uint32_t &J) {
+    const double b = 2.0 * (double)T + 1.0;
+    int64_t i = (int64_t)((b - sqrt(b * b - 8.0 * (double)t)) * 0.5);   // estimate, then exact fix-up
+    if (i < 0) i = 0;
+    if (i > T - 1) i = T - 1;
+    while (i > 0 && tri_start(T, i) > t) --i;
+    while (i + 1 < T && tri_start(T, i + 1) <= t) ++i;
+    I = (uint32_t)i;
+    J = (uint32_t)(i + (t - tri_start(T, i)));
+}
 
 struct GemmArgs {
     const uint32_t *A;   // [m][lda32] packed rows viewed as uint32 words
@@ -31,6 +60,10 @@ struct GemmArgs {
     const uint32_t *popB;
     int op2 = 0;           // gemm_tc4, swapped layout (m < n) only: a second op from the same
     uint32_t *C2 = nullptr;  // AND count, written to C2 (NULL: one op)
+    // f3 packed triangle (self-LD, A == B, m == n): tri_n >= 0 computes tiles tri_lo ..
+    // tri_lo + tri_n - 1 only, tile u of the call stored dense at element u * 128 * 128
+    // of C / r2 / dprime (row-major, ldc = 128); no mirror.
+    int64_t tri_lo = 0, tri_n = -1;
 };
 
 // CUDA-core LOP3 + POPC variant (bitgemm_popc.cu).
@@ -43,6 +76,10 @@ cudaError_t launch_pack_popc(const uint8_t *g, int64_t rows, int64_t nbits, int6
                              uint64_t *packed, int64_t ldw, uint32_t *popc, cudaStream_t s);
 cudaError_t launch_row_popc(const uint64_t *x, int64_t rows, int64_t nbits, int64_t ldw,
                             uint32_t *popc, cudaStream_t s);
+
+// sym.cu — f3 packed triangle -> full symmetric matrix (4-byte elements).
+cudaError_t launch_sym_unpack(const uint32_t *tiles, int64_t m, int64_t tlo, int64_t ntiles, uint32_t *out,
+                              int64_t ldo, cudaStream_t s);
 
 // best.cu — scratch is best_index reinterpreted as packed (count<<32 | j) keys.
 cudaError_t launch_best(const uint32_t *counts, int64_t nq, int64_t nd, int64_t ldo,

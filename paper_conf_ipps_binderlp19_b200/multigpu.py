@@ -9,6 +9,10 @@ The path shards with ONE exchange step and no collective inside the hot loop:
   the lowest-global-index tie-break (reading R4).
 * LD: output row blocks are sharded; the packed matrix is broadcast from rank 0
   and rank r computes rows ``[b_r, b_{r+1})`` against all columns.
+* Symmetric self-LD (f3): the T(T+1)/2 upper-triangle 128 x 128 tiles are split into
+  contiguous, equal-count ranges (``snp_shard_plan_sym``); rank r computes its range
+  into the packed tile layout of ``snp_ld_sym`` — no tile twice, no mirrored-block
+  exchange, balanced within one tile.
 
 The compute callables default to the CUDA library; tests inject oracle-backed
 callables to exercise the same exchange logic with the gloo backend on CPU.
@@ -51,6 +55,13 @@ def pack_best(bc: torch.Tensor, bi: torch.Tensor) -> torch.Tensor:
     minimum over shards is the global best with the lowest-index tie-break (reading R4):
     ONE all-gather and ONE min replace two gathers and an argmin merge."""
     c = (bc.view(torch.int32) if bc.dtype == torch.uint32 else bc).to(torch.int64) & 0xFFFFFFFF
+    # a real count must stay below 2^23 so count << 40 keeps the sign bit clear; counts of
+    # longer profiles go through merge_best (two-tensor gather) instead
+    real = bi >= 0
+    if bool(((c >= (1 << (63 - KEY_IDX_BITS))) & real).any()):
+        raise ValueError("pack_best: count >= 2^23 does not fit the packed key; use merge_best")
+    if bool((bi >= (1 << KEY_IDX_BITS)).any()):
+        raise ValueError("pack_best: index >= 2^40 does not fit the packed key")
     key = (c << KEY_IDX_BITS) | bi.to(torch.int64)
     return torch.where(bi < 0, torch.full_like(key, KEY_NONE), key)
 
@@ -101,3 +112,26 @@ def ld_step(B: torch.Tensor, nbits: int, lo: int, hi: int, compute=None, group=N
     if world > 1:
         dist.broadcast(B.view(torch.int64) if B.dtype == torch.uint64 else B, src=0, group=group)
     return compute(B[lo:hi], B)
+
+
+def sym_tile_coords(m: int, t: int, tile: int = 128) -> tuple[int, int]:
+    """Tile t of the row-major upper triangle (include/snp.h, snp_ld_sym) -> (I, J), I <= J:
+    t = start(I) + (J - I), start(I) = I T - I (I - 1) / 2, T = ceil(m / tile)."""
+    T = -(-m // tile)
+    if not 0 <= t < T * (T + 1) // 2:
+        raise ValueError("tile index out of range")
+    i = 0
+    while i + 1 < T and (i + 1) * T - (i + 1) * i // 2 <= t:
+        i += 1
+    return i, i + t - (i * T - i * (i - 1) // 2)
+
+
+def ld_sym_step(B: torch.Tensor, nbits: int, tile_lo: int, tile_hi: int, compute=None, group=None):
+    """One sharded symmetric self-LD step: broadcast the packed matrix from rank 0, compute
+    this rank's packed-triangle tiles [tile_lo, tile_hi) (snp_shard_plan_sym)."""
+    from . import snp_ld_sym
+    compute = compute or (lambda B_, lo_, hi_: snp_ld_sym(B_, nbits, lo_, hi_, counts=True))
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    if world > 1:
+        dist.broadcast(B.view(torch.int64) if B.dtype == torch.uint64 else B, src=0, group=group)
+    return compute(B, tile_lo, tile_hi)

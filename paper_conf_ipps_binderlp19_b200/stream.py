@@ -57,8 +57,11 @@ def stream_search(Q: torch.Tensor, D_host: torch.Tensor, nbits: int, ops=("xor",
     Pbuf = [torch.empty(rows_max, dtype=torch.uint32, device=dev) for _ in range(nbuf)] if popD_host is not None else None
     # per-chunk results are written as uint32 counts / int64 indices, then widened
     cnt32 = torch.empty((nops, len(plan), nq), dtype=torch.uint32, device=dev)
-    ws = torch.empty(max(1, snp_fastid_search_workspace_bytes(nq, rows_max, nbits, nops)), dtype=torch.uint8,
-                     device=dev)
+    # the dispatcher's kernel choice (and so its scratch) depends on the chunk's row count: a
+    # ragged last chunk with few rows can take a path that needs more workspace than a full
+    # chunk, so size for every distinct chunk length
+    ws_need = max(snp_fastid_search_workspace_bytes(nq, rows, nbits, nops) for rows in {r1 - r0 for r0, r1 in plan})
+    ws = torch.empty(max(1, ws_need), dtype=torch.uint8, device=dev)
     comp = torch.cuda.current_stream(dev)
     copy = torch.cuda.Stream(dev)
     copy.wait_stream(comp)   # the buffers (and Q) were just allocated / produced on comp

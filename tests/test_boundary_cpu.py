@@ -179,3 +179,53 @@ def test_search_validation_before_launch(snplib):
     assert snplib.snp_fastid_search_workspace_bytes(4, 9, 100, 2) >= 2 * 4 * 8
     assert snplib.snp_fastid_search_workspace_bytes(4, 0, 100, 2) >= 2 * 4 * 8
     assert snplib.snp_fastid_search_workspace_bytes(0, 9, 100, 2) == 0
+
+
+@pytest.mark.parametrize("m,world", [(0, 1), (1, 1), (128, 3), (300, 2), (2048, 8), (32768, 8), (32768, 7),
+                                     (100_000, 5), (129, 8)])
+def test_shard_plan_sym_properties(snplib, m, world):
+    """e + f3: contiguous tile ranges covering every upper-triangle tile exactly once,
+    tile counts balanced within one, deterministic."""
+    T = -(-m // 128)
+    total = T * (T + 1) // 2
+    assert snplib.snp_sym_tiles(m) == total
+    b = snplib.snp_shard_plan_sym(m, world)
+    assert len(b) == world + 1 and b[0] == 0 and b[-1] == total
+    sizes = [b[r + 1] - b[r] for r in range(world)]
+    assert all(x >= 0 for x in sizes)
+    assert max(sizes) - min(sizes) <= 1
+    assert b == snplib.snp_shard_plan_sym(m, world)
+
+
+def test_shard_plan_sym_errors(snplib):
+    L = snplib.lib()
+    arr = (ctypes.c_int64 * 4)()
+    assert L.snp_shard_plan_sym(100, 0, ctypes.cast(arr, ctypes.c_void_p)) == E_RANGE
+    assert L.snp_shard_plan_sym(-1, 2, ctypes.cast(arr, ctypes.c_void_p)) == E_RANGE
+    assert L.snp_shard_plan_sym(100, 2, None) == E_NULL
+    assert L.snp_sym_tiles(-3) == 0
+
+
+def test_sym_tile_enumeration_is_a_bijection():
+    """The row-major upper-triangle order of snp_ld_sym: every (I <= J) exactly once, in
+    order, with the closed-form start(I) = I T - I (I - 1) / 2."""
+    from paper_conf_ipps_binderlp19_b200.multigpu import sym_tile_coords
+    for m in (1, 128, 129, 300, 2048, 5000):
+        T = -(-m // 128)
+        coords = [sym_tile_coords(m, t) for t in range(T * (T + 1) // 2)]
+        assert coords == [(i, j) for i in range(T) for j in range(i, T)]
+
+
+def test_ld_sym_validation(snplib):
+    """snp_ld_sym rejects bad tile ranges and missing outputs before any launch."""
+    L = snplib.lib()
+    fake = 1 << 20   # an aligned non-NULL address: validation fails before it is touched
+    assert L.snp_ld_sym(fake, 300, 8, None, 300, 0, 7, fake, None, None, fake, 4096, None) == E_RANGE
+    assert L.snp_ld_sym(fake, 300, 8, None, 300, 3, 2, fake, None, None, fake, 4096, None) == E_RANGE
+    assert L.snp_ld_sym(fake, 300, 8, None, 300, -1, 2, fake, None, None, fake, 4096, None) == E_RANGE
+    assert L.snp_ld_sym(fake, 300, 8, None, 300, 0, 6, None, None, None, fake, 4096, None) == E_NULL
+    assert L.snp_ld_sym(fake, 300, 8, None, 300, 0, 6, None, fake, fake, fake, 4096, None) == E_NULL  # D' needs r2
+    assert L.snp_ld_sym(fake, 300, 8, None, 300, 2, 2, fake, None, None, None, 0, None) == OK          # empty range
+    assert L.snp_ld_sym(fake + 8, 300, 8, None, 300, 0, 6, fake, None, None, fake, 4096, None) == E_ALIGN
+    assert L.snp_sym_unpack(fake, 300, 0, 7, fake, 300, None) == E_RANGE
+    assert L.snp_sym_unpack(fake, 300, 0, 6, fake, 299, None) == E_SHAPE

@@ -572,6 +572,25 @@ def test_stream_search_chunks(snp, with_pop):
         assert np.array_equal(res[j][1].cpu().numpy(), ri), op
 
 
+@pytest.mark.parametrize("nq,nd,chunk", [(40, 1536 + 128, 1536), (64, 4 * 1024 + 100, 1024), (100, 2048 + 40, 2048)])
+def test_stream_search_ragged_small_last_chunk(snp, nq, nd, chunk):
+    """f2 with a last chunk so short (< 4 nq rows, or < 256 rows past 64 queries) that the
+    dispatcher leaves the fused kernel for a path with a larger workspace: the scratch is
+    sized for every distinct chunk length, so the stream completes and matches the oracle."""
+    from paper_conf_ipps_binderlp19_b200.stream import stream_search
+    nbits = 900
+    db = snpgen.fastid_db(72, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(72, nq, nd, nbits)
+    q[1] = db[nd - 3]                                  # exact copy in the short last chunk
+    D_host = pack_dev(snp, db).cpu().pin_memory()
+    res = stream_search(pack_dev(snp, q), D_host, nbits, ("xor", "andnot"), chunk_rows=chunk)
+    torch.cuda.synchronize()
+    for j, op in enumerate(("xor", "andnot")):
+        rb, ri = oracle.best(oracle.counts(q, db, op))
+        assert np.array_equal(res[j][0].cpu().numpy().astype(np.uint32), rb), op
+        assert np.array_equal(res[j][1].cpu().numpy(), ri), op
+
+
 def test_search_general_kernel_forced(snp, monkeypatch):
     """More than 64 queries at few bits with the 64-query slicing disabled: the general
     kernel's paired-op pass (counts of two ops from one AND count) + best pass."""
@@ -670,3 +689,63 @@ def test_ld_unaligned_output_rows(snp, self_ld):
             assert (r2b[:, m:].cpu().numpy() == -1.0).all()
             if dpb is not None:
                 check_r2(dpb[:, :m].cpu().numpy(), dp_ref)
+
+
+def _sym_blocks_ref(g, m):
+    r2, dp, n = oracle.ld(g, g)
+    return r2, dp, n
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("m,nbits", [(300, 1025), (128, 64), (129, 700), (2300, 1025), (1, 5)])
+def test_ld_sym_packed_tiles(snp, variant, m, nbits):
+    """f3 packed triangle: every tile of the row-major upper triangle equals the oracle's
+    block (counts bit-exact, r2 / D' within 1e-6 relative, exactly 0 where the oracle is 0);
+    entries of ragged tiles past m are 0; snp_sym_unpack rebuilds the full matrices."""
+    from paper_conf_ipps_binderlp19_b200.multigpu import sym_tile_coords
+    g = snpgen.ld_genotypes(63, np.arange(m), nbits, structure=True)
+    A = pack_dev(snp, g, garbage_seed=5)
+    _variant(snp, variant)
+    try:
+        r2, dp, cnt = snp.snp_ld_sym(A, nbits, r2=True, dprime=True, counts=True)
+        kern = snp.snp_last_kernel()
+    finally:
+        _variant(snp, "auto")
+    assert kern == ("tc_mxf4_sym" if variant == "tc" else "popc")
+    r2_ref, dp_ref, n_ref = oracle.ld(g, g)
+    R2, DP, C = r2.cpu().numpy(), dp.cpu().numpy(), u32(cnt)
+    for t in range(snp.snp_sym_tiles(m)):
+        I, J = sym_tile_coords(m, t)
+        rs, cs = slice(128 * I, min(m, 128 * I + 128)), slice(128 * J, min(m, 128 * J + 128))
+        h, w = rs.stop - rs.start, cs.stop - cs.start
+        assert np.array_equal(C[t, :h, :w], n_ref[rs, cs]), (t, I, J)
+        check_r2(R2[t, :h, :w], r2_ref[rs, cs])
+        check_r2(DP[t, :h, :w], dp_ref[rs, cs])
+        for X in (R2, DP):
+            assert (X[t, h:, :] == 0).all() and (X[t, :, w:] == 0).all()
+        assert (C[t, h:, :] == 0).all() and (C[t, :, w:] == 0).all()
+    full = snp.snp_sym_unpack(cnt, m)
+    assert np.array_equal(u32(full), n_ref)
+    fr2 = snp.snp_sym_unpack(r2, m)
+    check_r2(fr2.cpu().numpy(), r2_ref)
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_ld_sym_tile_ranges_match_whole(snp, variant):
+    """One rank's share: tiles [lo, hi) of an uneven plan equal the same tiles of the whole
+    call (counts-only and r2-only forms), for every rank of a 3-way plan."""
+    m, nbits = 700, 513
+    g = snpgen.ld_genotypes(64, np.arange(m), nbits, structure=True)
+    A = pack_dev(snp, g)
+    _variant(snp, variant)
+    try:
+        r2w, _, cw = snp.snp_ld_sym(A, nbits, counts=True)
+        b = snp.snp_shard_plan_sym(m, 3)
+        for r in range(3):
+            _, _, c = snp.snp_ld_sym(A, nbits, b[r], b[r + 1], r2=False, counts=True)
+            r2, _, _ = snp.snp_ld_sym(A, nbits, b[r], b[r + 1])
+            assert torch.equal(c, cw[b[r]:b[r + 1]]), r
+            assert torch.equal(r2, r2w[b[r]:b[r + 1]]), r
+    finally:
+        _variant(snp, "auto")
+    assert np.array_equal(u32(snp.snp_sym_unpack(cw, m)), oracle.ld(g, g)[2])

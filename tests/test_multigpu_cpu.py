@@ -143,3 +143,79 @@ def test_pack_best_keys():
     u = torch.tensor([0x7FFFFF, 0], dtype=torch.int32).view(torch.uint32)   # uint32 counts
     c, i = unpack_best(pack_best(u, torch.tensor([3, 4])))
     assert c.tolist() == [0x7FFFFF, 0] and i.tolist() == [3, 4]
+
+
+def test_pack_best_rejects_counts_that_overflow_the_key():
+    """count << 40 must keep the sign bit clear: counts >= 2^23 (possible for profiles of
+    more than 2^23 SNPs) are rejected instead of silently winning the min as negatives."""
+    from paper_conf_ipps_binderlp19_b200.multigpu import pack_best
+    with pytest.raises(ValueError):
+        pack_best(torch.tensor([1 << 23]), torch.tensor([0]))
+    with pytest.raises(ValueError):
+        pack_best(torch.tensor([1]), torch.tensor([1 << 40]))
+    pack_best(torch.tensor([(1 << 23) - 1, 0xFFFFFFFF]), torch.tensor([0, -1]))   # empty shard is fine
+
+
+def _sym_worker(rank, world, port, q):
+    try:
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        from paper_conf_ipps_binderlp19_b200 import multigpu, snp_shard_plan_sym
+        m, nbits = 300, 130
+        g = snpgen.ld_genotypes(79, np.arange(m), nbits, structure=True)
+        B = torch.from_numpy(oracle.pack(g, 4).view(np.int64)) if rank == 0 else torch.zeros((m, 4), dtype=torch.int64)
+        b = snp_shard_plan_sym(m, world)
+        lo, hi = b[rank], b[rank + 1]
+
+        def tiles_compute(B_, lo_, hi_):
+            # oracle-backed tiles in the packed layout: tile u = block (I, J), zeros past m
+            gg = oracle.unpack(B_.numpy().view(np.uint64), nbits)
+            out = np.zeros((hi_ - lo_, 128, 128), dtype=np.float64)
+            for u, t in enumerate(range(lo_, hi_)):
+                I, J = multigpu.sym_tile_coords(m, t)
+                r2, _, _ = oracle.ld(gg[128 * I:128 * I + 128], gg[128 * J:128 * J + 128])
+                out[u, :r2.shape[0], :r2.shape[1]] = r2
+            return out
+
+        mine = multigpu.ld_sym_step(B, nbits, lo, hi, compute=tiles_compute)
+        got = [None] * world
+        dist.all_gather_object(got, (lo, hi, mine))
+        full = np.full((m, m), np.nan)
+        seen = set()
+        for lo_, hi_, tl in got:
+            for u, t in enumerate(range(lo_, hi_)):
+                assert t not in seen
+                seen.add(t)
+                I, J = multigpu.sym_tile_coords(m, t)
+                blk = tl[u][:min(128, m - 128 * I), :min(128, m - 128 * J)]
+                full[128 * I:128 * I + blk.shape[0], 128 * J:128 * J + blk.shape[1]] = blk
+                full[128 * J:128 * J + blk.shape[1], 128 * I:128 * I + blk.shape[0]] = blk.T
+        r2_ref, _, _ = oracle.ld(g, g)
+        q.put((rank, bool(np.array_equal(full, r2_ref)), len(seen), hi - lo))
+        dist.destroy_process_group()
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, "error", traceback.format_exc()))
+
+
+def test_two_rank_gloo_symmetric_ld_plan():
+    """f3 + e: the triangle-balanced plan over 2 ranks — each rank computes only its tile
+    range (oracle-backed tiles in the packed layout); together the ranks cover every upper-
+    triangle tile once and the mirrored union equals the oracle's full r2 matrix."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sym_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for r in res:
+        assert r[1] != "error", r[2]
+        rank, ok, nseen, mine = r
+        assert ok, f"rank {rank}: reconstructed symmetric matrix != oracle"
+        assert nseen == 6                      # T = 3 tiles per side: 6 upper-triangle tiles
+        assert mine == 3                       # balanced: 3 + 3

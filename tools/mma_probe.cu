@@ -2,6 +2,7 @@
 // one issuing thread, back-to-back MMAs on garbage operands, clock64 around them).
 // Used to pick the tensor-core kernel shapes.  Not part of the library.
 #include <cstdio>
+#include <cstdlib>
 #include <cstdint>
 #include <cuda_runtime.h>
 #include "../paper_conf_ipps_binderlp19_b200/csrc/tc_ptx.cuh"
@@ -73,6 +74,11 @@ void run(const char *name) {
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     long long h[148]; cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
     cudaError_t err = cudaGetLastError();
+    if (err != cudaSuccess) {
+        printf("%-14s M=%3d N=%3d  FAILED: %s\n", name, M, N, cudaGetErrorString(err));
+        fflush(stdout);
+        exit(1);   // a sticky error poisons every later launch
+    }
     double cyc = (double)h[0] / iters;
     const int K = (MODE <= 1) ? 64 : 32;
     double macs = (double)M * N * K * iters * 148;
@@ -82,6 +88,7 @@ void run(const char *name) {
 }
 
 int main() {
+    setvbuf(stdout, nullptr, _IONBF, 0);
     run<0, 64>("mxf4 SS"); run<0, 128>("mxf4 SS"); run<0, 256>("mxf4 SS");
     run<1, 64>("mxf4 TS"); run<1, 128>("mxf4 TS"); run<1, 256>("mxf4 TS");
     run<2, 64>("i8 SS"); run<2, 128>("i8 SS"); run<2, 256>("i8 SS");
