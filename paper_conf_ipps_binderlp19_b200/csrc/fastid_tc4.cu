@@ -33,6 +33,8 @@ namespace snp {
 // [2] before full arrive, [3] MMA after full wait.  Enabled by SNP_TRACE=1.
 __device__ long long g_fastid_trace[8 * 1024];
 __device__ long long g_fastid_etrace[4 * 256];   // FASTID_TRACE2: per tile, CTA 0
+__device__ long long g_fastid_wtrace[4 * 1024];
+__device__ long long g_fastid_wtrace2[32 * 1024]; // FASTID_TRACE2: per stage and warp qa: 8 stamps  // FASTID_TRACE2: per stage, full-arrive clock of warps qa = 0..3
 __device__ long long g_fastid_cta_time[3 * 1024];
 __device__ long long g_fastid_launch_time[2 * 64];   // CTA 0: start / end globaltimer per launch
 __device__ unsigned int g_fastid_launch_ctr;   // per CTA: start, main loop start, end (globaltimer ns)
@@ -58,6 +60,16 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 // (popcounts counted in-kernel) but 185 -> 191 us with 2 groups, so only for GG = 4.
 #ifndef FASTID_HALF
 #define FASTID_HALF 4   // the GG that uses half-stage barriers (0: none)
+#endif
+// tcgen05 instructions issued from one SM sub-partition execute in order, so the TMEM
+// stores (tcgen05.st) of the expander warp that shares the MMA warp's sub-partition queue
+// behind every MMA already issued — measured: that lane quarter finished each stage
+// 1 350 - 1 560 cycles after the other three (scripts/trace_fastid2.py), which throttled
+// the pipeline to 600 - 760 cycles per 400-cycle stage.  With FASTID_ISSUE_AHEAD the MMA
+// warp issues stage s only after that warp has ISSUED its stores for stage s + 1, so they
+// are queued ahead of MMA(s) instead of behind it.
+#ifndef FASTID_ISSUE_AHEAD
+#define FASTID_ISSUE_AHEAD 1
 #endif
 #ifndef FASTID_NACC
 #define FASTID_NACC 2   // TMEM accumulators (the MMA may run NACC - 1 tiles ahead of the epilogue)
@@ -88,8 +100,13 @@ struct Roles {
     static constexpr int G = GG;
     static constexpr int NEXP = 4 * GG;
     static constexpr int EPI_WARP0 = NEXP;
+#ifndef FASTID_MMA_FIRST
     static constexpr int TMA_WARP = NEXP + NEPI;
     static constexpr int MMA_WARP = NEXP + NEPI + 1;
+#else   // experiment: MMA issuer on SMSP (NEXP + NEPI) % 4, TMA producer on the next one
+    static constexpr int TMA_WARP = NEXP + NEPI + 1;
+    static constexpr int MMA_WARP = NEXP + NEPI;
+#endif
     static constexpr int NTHREADS = (NEXP + NEPI + 2) * 32;
 };
 constexpr size_t MAX_SMEM = 232448;     // 227 KB opt-in
@@ -169,7 +186,8 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     uint64_t *accf = empty + NS;             // [NACC]
     uint64_t *acce = accf + NACC;            // [NACC]
     uint64_t *popf = acce + NACC;            // [NACC]
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(popf + NACC);
+    uint64_t *issued = popf + NACC;          // [NS] MMA-sub-partition expander -> MMA: stores issued
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(issued + NS);
     uint32_t *popQ = tmem_slot + 4;          // [BN]
     uint32_t *popD = popQ + BN;              // [2 acc][G][BM]
     uint32_t *popQ32 = popD + NACC * G * BM; // [BN] 32 * popQ (epilogue key term)
@@ -201,6 +219,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             ptx::mbar_init(&acce[i], NEPI);
             ptx::mbar_init(&popf[i], NEXP);
         }
+        for (int i = 0; i < NS; ++i) ptx::mbar_init(&issued[i], 1);
         ptx::fence_mbar_init();
     }
     if (warp == TMA_WARP && lane == 0) ptx::prefetch_tensormap(&tmD);
@@ -310,16 +329,29 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             const bool tr = SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && qa == 0 && it < 1024;
 #endif
+#ifdef FASTID_TRACE2
+            const bool trw = SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && it < 1024;
+            long long *tw2 = g_fastid_wtrace2 + 32 * it + 8 * qa;
+#endif
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 0] = clock64();
+#ifdef FASTID_TRACE2
+            if (trw) tw2[0] = clock64();
+#endif
 #endif
             ptx::mbar_wait_warp(&pfull[p], pround & 1);
 #ifdef FASTID_TRACE2
             if (tr) g_fastid_trace[8 * it + 4] = clock64();
+#ifdef FASTID_TRACE2
+            if (trw) tw2[4] = clock64();
+#endif
 #endif
             if (bround > 0) ptx::mbar_wait_warp(&empty[b], (bround - 1) & 1);
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 1] = clock64();
+#ifdef FASTID_TRACE2
+            if (trw) tw2[1] = clock64();
+#endif
 #endif
             // 64-byte row of the stage; TMA 64B swizzle: 16-byte chunk c of row r sits at
             // chunk c ^ ((r >> 1) & 3)  (conflict-free LDS.128 across the warp)
@@ -343,6 +375,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             }
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive(&pempty[p]);
+#ifdef FASTID_TRACE2
+            if (tr) g_fastid_trace[8 * it + 6] = clock64();
+#ifdef FASTID_TRACE2
+            if (trw) tw2[6] = clock64();
+#endif
+#endif
             const uint32_t tbase = tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + ACOLS * b);
 #pragma unroll
             for (int h = 0; h < KW / 8; ++h) {
@@ -358,11 +396,27 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                     if (lane == 0) ptx::mbar_arrive(&full[b * NHALF]);
                 }
             }
+#ifdef FASTID_TRACE2
+            if (tr) g_fastid_trace[8 * it + 7] = clock64();
+#ifdef FASTID_TRACE2
+            if (trw) tw2[7] = clock64();
+#endif
+#endif
+            if (FASTID_ISSUE_AHEAD && qa == (MMA_WARP & 3)) {
+                __syncwarp();   // every lane's tcgen05.st of this stage is issued
+                if (lane == 0) ptx::mbar_arrive(&issued[b]);
+            }
             ptx::tmem_st_wait();
             ptx::tc_fence_before();
             __syncwarp();
 #if defined(FASTID_TRACE) || defined(FASTID_TRACE2)
             if (tr) g_fastid_trace[8 * it + 2] = clock64();
+#ifdef FASTID_TRACE2
+            if (trw) tw2[2] = clock64();
+#endif
+#endif
+#ifdef FASTID_TRACE2
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && it < 1024) g_fastid_wtrace[4 * it + qa] = clock64();
 #endif
             if (lane == 0) ptx::mbar_arrive(&full[b * NHALF + NHALF - 1]);
             s += G;
@@ -408,6 +462,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 3] = clock64();
 #endif
                 ptx::mbar_wait_uniform(&full[b * NHALF], bround & 1);
+                if (FASTID_ISSUE_AHEAD && itm + 1 < total_it) {
+                    // the next stage's stores on this sub-partition go ahead of these MMAs
+                    const int bn = b + 1 == NS ? 0 : b + 1;
+                    const uint32_t rn = b + 1 == NS ? bround + 1 : bround;
+                    ptx::mbar_wait_uniform(&issued[bn], rn & 1);
+                }
                 ptx::tc_fence_after();
 #ifdef FASTID_TRACE2
                 if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 5] = clock64();
@@ -771,6 +831,16 @@ extern "C" int snp_debug_fastid_cta_times(long long *host, int n) {
 extern "C" int snp_debug_fastid_etrace(long long *host, int n) {
     if (n > 4 * 256) n = 4 * 256;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_etrace, sizeof(long long) * n);
+}
+
+extern "C" int snp_debug_fastid_wtrace2(long long *host, int n) {
+    if (n > 32 * 1024) n = 32 * 1024;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_wtrace2, sizeof(long long) * n);
+}
+
+extern "C" int snp_debug_fastid_wtrace(long long *host, int n) {
+    if (n > 4 * 1024) n = 4 * 1024;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_wtrace, sizeof(long long) * n);
 }
 
 extern "C" int snp_debug_fastid_trace(long long *host, int n) {

@@ -33,6 +33,16 @@ namespace snp {
 // [0] expander before waits, [1] after waits, [2] after packed LDS, [3] half 0 published,
 // [4] half 1 published, [5] MMA got half 0, [6] MMA got half 1, [7] MMA commit issued.
 __device__ long long g_gemm_trace[8 * 2048];
+// Per-CTA timeline (build with -DSNP_PROFILING -DGEMM_TRACE3, read with snp_debug_gemm_cta):
+// globaltimer ns at [0] entry, [1] setup done, [2] griddepcontrol.wait returned, [3] first
+// packed stage arrived (expander 0), [4] first accumulator ready (epilogue warp 0), [5] last
+// tile stored (epilogue warp 0), [6] exit barrier passed.
+__device__ long long g_gemm_cta[8 * 1024];
+#ifdef GEMM_TRACE3
+#define GEMM_T3(k, cond) do { if ((cond) && blockIdx.x < 1024) g_gemm_cta[8 * blockIdx.x + (k)] = (long long)ptx::globaltimer_ns(); } while (0)
+#else
+#define GEMM_T3(k, cond) do { } while (0)
+#endif
 
 namespace {
 
@@ -614,6 +624,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acce + 2);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    GEMM_T3(0, tid == 0);
     const int64_t nbits = args.nbits;
     const int nst = args.nst;
     const int64_t ntiles = TRI ? args.ntri : args.sym ? args.nlb * (args.nlb + 1) / 2 : args.nlb * args.ncb;
@@ -710,10 +721,12 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     ptx::tc_fence_before();
     __syncthreads();
     ptx::tc_fence_after();
+    GEMM_T3(1, tid == 0);
     // programmatic dependent launch: the setup above overlapped the previous kernel (the
     // row-popcount pre-pass); its results are visible after this wait, and nothing global
     // was read or written before it
     asm volatile("griddepcontrol.wait;" ::: "memory");
+    GEMM_T3(2, tid == 0);
 
     if (warp == TMA_WARP) {
         // ------------------------------------------------------------ TMA producer
@@ -767,6 +780,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             // release use u+1 first rules out parity aliasing on pfull (same parity as u)
             if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
             ptx::mbar_wait_warp(&pfull[pk], pround & 1);
+            GEMM_T3(3, it == 0 && warp == 0 && lane == 0);
 #ifdef GEMM_TRACE
             if (tr) g_gemm_trace[8 * it + 1] = clock64();
 #endif
@@ -929,6 +943,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 if (32 + lane < ncols) pcol1 = __ldg(args.popC + gc0 + 32 + lane);
             }
             ptx::mbar_wait_warp(&accf[acc], ph);
+            GEMM_T3(4, tl == 0 && e == 0 && lane == 0);
             ptx::tc_fence_after();
             const bool full_vec = ncols == 64 && !args.swap;
             const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * ACC_COLS + c0);
@@ -1044,8 +1059,10 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         }
     }
 
+    GEMM_T3(5, warp == EPI_WARP0 && lane == 0);
     ptx::tc_fence_before();
     __syncthreads();
+    GEMM_T3(6, tid == 0);
     if (warp == MMA_WARP) {
         ptx::tc_fence_after();
         ptx::tmem_dealloc<512>(tmem);
@@ -1580,6 +1597,11 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
 }  // namespace snp
 
 #ifdef SNP_PROFILING
+extern "C" int snp_debug_gemm_cta(long long *host, int n) {
+    if (n > 8 * 1024) n = 8 * 1024;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_gemm_cta, sizeof(long long) * n);
+}
+
 extern "C" int snp_debug_gemm_trace(long long *host, int n) {
     if (n > 8 * 2048) n = 8 * 2048;
     return (int)cudaMemcpyFromSymbol(host, snp::g_gemm_trace, sizeof(long long) * n);
