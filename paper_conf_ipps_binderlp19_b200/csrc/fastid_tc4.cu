@@ -65,11 +65,13 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 // stores (tcgen05.st) of the expander warp that shares the MMA warp's sub-partition queue
 // behind every MMA already issued — measured: that lane quarter finished each stage
 // 1 350 - 1 560 cycles after the other three (scripts/trace_fastid2.py), which throttled
-// the pipeline to 600 - 760 cycles per 400-cycle stage.  With FASTID_ISSUE_AHEAD the MMA
-// warp issues stage s only after that warp has ISSUED its stores for stage s + 1, so they
-// are queued ahead of MMA(s) instead of behind it.
+// the pipeline to 600 - 760 cycles per 400-cycle stage (the TMA warp's sub-partition shows
+// a smaller lag of the same kind).  With FASTID_ISSUE_AHEAD the MMA warp issues stage s only
+// after that warp has ISSUED its stores for stage s + 1, so they are queued ahead of MMA(s):
+// measured, the lag halves (~800 cycles) but the MMA then waits on the look-ahead, FastID-1M
+// 0.192 -> 0.200 ms, so it is off.
 #ifndef FASTID_ISSUE_AHEAD
-#define FASTID_ISSUE_AHEAD 1
+#define FASTID_ISSUE_AHEAD 0
 #endif
 #ifndef FASTID_NACC
 #define FASTID_NACC 2   // TMEM accumulators (the MMA may run NACC - 1 tiles ahead of the epilogue)
