@@ -251,8 +251,10 @@ typedef enum {
     SNP_KERNEL_TC_I8 = 2,       /* tcgen05 kind::i8 on u8-expanded operands        */
     SNP_KERNEL_TC_MXF4 = 3,     /* tcgen05 kind::mxf4 on e2m1-expanded operands    */
     SNP_KERNEL_FASTID_MXF4 = 4, /* kind::mxf4, resident queries, TMA-streamed DB   */
-    SNP_KERNEL_TC_MXF4_SYM = 5  /* kind::mxf4 self-LD, upper-triangle tiles + mirror (f3):
+    SNP_KERNEL_TC_MXF4_SYM = 5, /* kind::mxf4 self-LD, upper-triangle tiles + mirror (f3):
                                    executes about half of the M*N*nbits comparisons */
+    SNP_KERNEL_POPC_STREAM = 6  /* CUDA-core FastID for nq <= 4: TMA-streamed database,
+                                   LOP3 + POPC, all ops and best matches in one pass   */
 } snp_kernel;
 int snp_last_kernel(void);
 

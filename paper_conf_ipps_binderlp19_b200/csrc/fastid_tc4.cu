@@ -55,6 +55,9 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 #ifndef FASTID_NS
 #define FASTID_NS 4
 #endif
+#ifndef FASTID_NS32
+#define FASTID_NS32 6   // TMEM A stages of the 32-wide-query instantiations (GG = 2)
+#endif
 // Per-half-stage full barriers (the MMA starts on the first 256 bits while the expanders
 // write the second half): measured on FastID-1M, 207 -> 195 us with 4 expander groups
 // (popcounts counted in-kernel) but 185 -> 191 us with 2 groups, so only for GG = 4.
@@ -115,8 +118,13 @@ constexpr size_t MAX_SMEM = 232448;     // 227 KB opt-in
 
 template <int BN>
 struct FCfg {
-    static constexpr int NS = FASTID_NS;            // TMEM A stages of 64 columns (multiple of G)
-    static_assert(NS % 4 == 0 && NP % 4 == 0, "rings must be multiples of the group count");
+    // TMEM A stages of 64 columns (a multiple of the expander group count).  A 32-wide
+    // query batch frees 64 accumulator columns for two more stages: the lane quarter that
+    // shares the MMA warp's sub-partition runs ~3.5 stages behind the others (its TMEM
+    // stores queue behind the issued MMAs, scripts/trace_fastid2.py), and deeper staging
+    // keeps the MMA fed while it catches up.
+    static constexpr int NS = FASTID_NS != 4 ? FASTID_NS : (BN == 32 ? FASTID_NS32 : 4);
+    static_assert(NS % 2 == 0 && NP % 4 == 0, "rings must be multiples of the group count");
     static constexpr int ACC_COLS = BN;
     static constexpr int A_COL0 = NACC * ACC_COLS;
     static constexpr int SF_COL = A_COL0 + NS * ACOLS;
@@ -779,8 +787,10 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
 // (configs[4] sweep: 1..32 queries x 20M x 8192 SNPs took the general kernel + best pass
 // at 9-12 ms against a 3.1 ms database read).
 int fastid_bn(int64_t m, int64_t nbits) {
-    if (m <= 64 && smem_bytes(64, nbits) <= MAX_SMEM - 1024) return 64;
+    // <= 32 queries: the 32-wide batch (N = 32 MMAs cost the same as N = 64, the epilogue
+    // half, and TMEM room for 6 A stages instead of 4)
     if (m <= 32 && smem_bytes(32, nbits) <= MAX_SMEM - 1024) return 32;
+    if (m <= 64 && smem_bytes(64, nbits) <= MAX_SMEM - 1024) return 64;
     return 0;
 }
 

@@ -99,6 +99,19 @@ int choose_variant(int64_t m, int64_t n, int64_t nbits) {
     return tc_supported(m, n, nbits) ? SNP_VARIANT_TC : SNP_VARIANT_POPC;
 }
 
+// a7: the CUDA-core streaming kernel serves the few-query FastID shapes (nq <= STREAM_NQ in
+// AUTO, from the measured configs[4] sweep; any nq <= 4 when the CUDA-core variant is forced)
+constexpr int64_t STREAM_NQ = 3;   // profiles/round2/sweep_stream2.txt: 1-3 queries win everywhere
+bool use_stream(int64_t nq, int64_t nd, int64_t nbits) {
+    const char *e = std::getenv("SNP_FASTID_STREAM");   // "0": never (A/B measurement hook)
+    if (e && e[0] == '0') return false;
+    if (!fastid_stream_supported(nq, nd, nbits)) return false;
+    const int v = current_variant();
+    if (v == SNP_VARIANT_POPC) return true;
+    if (v == SNP_VARIANT_TC) return false;
+    return nq <= STREAM_NQ;
+}
+
 size_t pops_bytes(int64_t m, int64_t n) { return align256((size_t)m * 4) + align256((size_t)n * 4); }
 
 // Which tensor-core kernel serves a shape (mirrors run_gemm's choice).
@@ -180,6 +193,7 @@ size_t snp_ld_workspace_bytes(int64_t m, int64_t n, int64_t nbits) {
 
 size_t snp_fastid_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op) {
     if (nq <= 0 || nd <= 0 || nbits <= 0) return 0;
+    if (use_stream(nq, nd, nbits)) return 0;
     if (choose_variant(nq, nd, nbits) != SNP_VARIANT_TC) return 0;
     if (op != SNP_OP_AND && tc_kernel_for(nq, nd, nbits, EPI_COUNTS) == SNP_KERNEL_TC_MXF4)
         return pops_bytes(nq, nd);   // row popcounts for the general kernel's identities
@@ -397,6 +411,18 @@ snp_status snp_fastid(const uint64_t *Q, int64_t nq, int64_t ldq, const uint32_t
     a.m = nq; a.n = nd; a.lda32 = 2 * ldq; a.ldb32 = 2 * ldd; a.nbits = nbits;
     a.op = op; a.accumulate = accumulate ? 1 : 0; a.ldc = ldo; a.C = out;
     a.popA = popQ; a.popB = popD;
+    if (use_stream(nq, nd, nbits)) {
+        SearchArgs sa{};
+        sa.Q = a.A; sa.nq = nq; sa.ldq32 = a.lda32;
+        sa.D = a.B; sa.nd = nd; sa.ldd32 = a.ldb32;
+        sa.popD = popD; sa.nbits = nbits;
+        sa.nops = 1; sa.ops[0] = op; sa.counts[0] = out; sa.ldo = ldo; sa.accumulate = a.accumulate;
+        cudaError_t e = launch_fastid_stream(sa, s);
+        if (e != cudaSuccess) return set_cuda_error(e);
+        g_last_variant = SNP_VARIANT_POPC;
+        g_last_kernel = SNP_KERNEL_POPC_STREAM;
+        return SNP_OK;
+    }
     if (variant == SNP_VARIANT_TC) {
         // given popcounts are used as they are (the FastID kernel skips counting the
         // streamed database words); NULL ones are derived in-kernel or by a pre-pass
@@ -466,6 +492,7 @@ extern "C" {
 size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int nops) {
     if (nq <= 0 || nbits <= 0 || nops < 1 || nops > 4) return 0;
     if (nd < 0) return 0;
+    if (nd > 0 && use_stream(nq, nd, nbits)) return fastid_stream_ws_bytes(nq, nops);
     if (search_fused(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(nq, nops);
     if (search_sliced(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(search_slice_width(nq, nd, nbits), nops);
     size_t b = align256((size_t)nops * nq * 8);
@@ -534,6 +561,15 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
         a.counts[j] = counts ? counts[j] : nullptr;
         a.best_count[j] = best_count ? best_count[j] : nullptr;
         a.best_index[j] = best_index ? best_index[j] : nullptr;
+    }
+    if (nd > 0 && use_stream(nq, nd, nbits)) {
+        // few queries: one CUDA-core pass over the database for every op (fastid_stream.cu)
+        a.keys = reinterpret_cast<unsigned long long *>(ws);
+        a.done = reinterpret_cast<unsigned int *>((char *)ws + align256((size_t)nops * nq * 8));
+        if ((e = launch_fastid_stream(a, s)) != cudaSuccess) return set_cuda_error(e);
+        g_last_variant = SNP_VARIANT_POPC;
+        g_last_kernel = SNP_KERNEL_POPC_STREAM;
+        return SNP_OK;
     }
     if (search_fused(nq, nd, nbits)) {
         // one pass over the database for every op (fastid_tc4.cu)

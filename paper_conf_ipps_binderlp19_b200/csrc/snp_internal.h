@@ -128,6 +128,12 @@ cudaError_t launch_fastid_tc4(const GemmArgs &a, int epi, cudaStream_t s);
 size_t fastid_search_tc4_ws_bytes(int64_t nq, int nops);
 cudaError_t launch_fastid_search_tc4(const SearchArgs &a, cudaStream_t s);
 
+// CUDA-core streaming FastID kernel for nq <= 4 (fastid_stream.cu): database TMA-streamed,
+// LOP3 + POPC per word and query, counts and best matches of up to 4 ops in one pass.
+bool fastid_stream_supported(int64_t nq, int64_t nd, int64_t nbits);
+size_t fastid_stream_ws_bytes(int64_t nq, int nops);
+cudaError_t launch_fastid_stream(const SearchArgs &a, cudaStream_t s);
+
 // best.cu building blocks for the chunked search path: keys (count << 32 | j) are
 // initialised to ~0, min-merged per count block (j offset by jbase), then finalised.
 cudaError_t launch_best_init(unsigned long long *keys, int64_t n, cudaStream_t s);

@@ -749,3 +749,58 @@ def test_ld_sym_tile_ranges_match_whole(snp, variant):
     finally:
         _variant(snp, "auto")
     assert np.array_equal(u32(snp.snp_sym_unpack(cw, m)), oracle.ld(g, g)[2])
+
+
+STREAM_SHAPES = [(1, 1, 1), (1, 300, 63), (2, 257, 512), (3, 5000, 513), (4, 4100, 4097), (4, 70000, 2048),
+                 (2, 1000, 20000), (1, 256, 130000)]
+
+
+@pytest.mark.parametrize("nq,nd,nbits", STREAM_SHAPES)
+@pytest.mark.parametrize("pre", [False, True], ids=["popD_inkernel", "popD_given"])
+def test_fastid_stream_all_ops_counts_and_best(snp, nq, nd, nbits, pre):
+    """CUDA-core streaming kernel (nq <= 4): every op's counts and best matches from one
+    database pass vs the oracle, ragged 256-row tiles and K tails, garbage in the padding,
+    database popcounts given or counted in-kernel; snp_fastid (single op) and accumulate."""
+    db = snpgen.fastid_db(81, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(81, nq, nd, nbits)
+    if nd > 10:
+        q[0] = db[nd // 2]                                 # an exact match (count 0)
+    D = pack_dev(snp, db, garbage_seed=3)
+    Q = pack_dev(snp, q, garbage_seed=4)
+    pd = snp.snp_row_popc(D, nbits) if pre else None
+    ops = ("and", "xor", "andnot", "notand")
+    # AUTO takes the streaming kernel for <= 3 queries (a7); the forced CUDA-core variant for <= 4
+    _variant(snp, "auto" if nq <= 3 else "popc")
+    try:
+        counts, best = snp.snp_fastid_search(Q, D, nbits, ops, index_base=7, popD=pd)
+        assert snp.snp_last_kernel() == "popc_stream"
+        out = snp.snp_fastid(Q, D, nbits, "xor", popD=pd)
+        assert snp.snp_last_kernel() == "popc_stream"
+        snp.snp_fastid(Q, D, nbits, "xor", out=out, popD=pd, accumulate=True)
+    finally:
+        _variant(snp, "auto")
+    for j, op in enumerate(ops):
+        ref = oracle.counts(q, db, op)
+        assert np.array_equal(u32(counts[j]), ref), op
+        rb, ri = oracle.best(ref, 7)
+        assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), op
+    assert np.array_equal(u32(out), 2 * oracle.counts(q, db, "xor"))
+
+
+def test_fastid_stream_ties_lowest_index(snp):
+    """Equal minimum counts in many tiles and CTAs: the lowest database index wins (R4)."""
+    nq, nd, nbits = 3, 300_000, 256
+    db = snpgen.fastid_db(82, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(82, nq, nd, nbits)
+    for r in (299_999, 150_000, 40_001, 40_000, 77_777):
+        db[r] = q[1]                                       # exact copies of query 1 everywhere
+    D, Q = pack_dev(snp, db), pack_dev(snp, q)
+    _variant(snp, "popc")
+    try:
+        _, best = snp.snp_fastid_search(Q, D, nbits, ("xor",), counts=False)
+        assert snp.snp_last_kernel() == "popc_stream"
+    finally:
+        _variant(snp, "auto")
+    assert int(best[0][0][1]) == 0 and int(best[0][1][1]) == 40_000
+    rb, ri = oracle.best(oracle.counts(q, db, "xor"))
+    assert np.array_equal(u32(best[0][0]), rb) and np.array_equal(best[0][1].cpu().numpy(), ri)
