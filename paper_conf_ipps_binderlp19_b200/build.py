@@ -29,7 +29,7 @@ def sources():
 
 
 def _inputs():
-    return sources() + sorted(glob.glob(os.path.join(CSRC, "*.h"))) + [HEADER, __file__]
+    return sources() + sorted(glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh"))) + [HEADER, __file__]
 
 
 def stale() -> bool:

@@ -27,6 +27,17 @@
 #include <cuda.h>
 #include <cstdlib>
 
+// Output stores: evict-first streaming stores (st.global.cs) by default — an LD output is
+// written once and must not push the packed operands out of L2; -DGEMM_STORE_WB keeps them
+// as ordinary write-back stores (measurement variant).
+#ifdef GEMM_STORE_WB
+#define STG_OUT "st.global"
+#define STG_OUT_FN(p, v) (void)(*(p) = (v))
+#else
+#define STG_OUT "st.global.cs"
+#define STG_OUT_FN(p, v) __stcs((p), (v))
+#endif
+
 namespace snp {
 
 // Pipeline trace of CTA 0 (profiling aid, SNP_TRACE=1): per iteration it < 2048,
@@ -38,10 +49,13 @@ __device__ long long g_gemm_trace[8 * 2048];
 // packed stage arrived (expander 0), [4] first accumulator ready (epilogue warp 0), [5] last
 // tile stored (epilogue warp 0), [6] exit barrier passed.
 __device__ long long g_gemm_cta[8 * 1024];
+__device__ long long g_gemm_cta2[8 * 1024];   // epilogue warp 0, first tile: [2 hh] after TMEM load, [2 hh + 1] after block
 #ifdef GEMM_TRACE3
 #define GEMM_T3(k, cond) do { if ((cond) && blockIdx.x < 1024) g_gemm_cta[8 * blockIdx.x + (k)] = (long long)ptx::globaltimer_ns(); } while (0)
+#define GEMM_T3B(k, cond) do { if ((cond) && blockIdx.x < 1024) g_gemm_cta2[8 * blockIdx.x + (k)] = (long long)ptx::globaltimer_ns(); } while (0)
 #else
 #define GEMM_T3(k, cond) do { } while (0)
+#define GEMM_T3B(k, cond) do { } while (0)
 #endif
 
 namespace {
@@ -158,12 +172,12 @@ __device__ __forceinline__ uint32_t acc_count(uint32_t v, bool small) {
 
 // predicated evict-first stores (no branch around them: shuffles stay converged)
 __device__ __forceinline__ void st_cs_pred_f32(float *p, float v, uint32_t ok) {
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(p), "f"(v),
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p " STG_OUT ".f32 [%0], %1;\n\t}" ::"l"(p), "f"(v),
                  "r"(ok)
                  : "memory");
 }
 __device__ __forceinline__ void st_cs_pred_u32(uint32_t *p, uint32_t v, uint32_t ok) {
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p " STG_OUT ".u32 [%0], %1;\n\t}" ::"l"(p), "r"(v),
                  "r"(ok)
                  : "memory");
 }
@@ -212,11 +226,11 @@ __device__ __forceinline__ void epi_mirror(const GArgs &args, const uint32_t (&c
             const float fn = (float)num;
             const float r2v = fminf(__fmul_rn(__fmul_rn(fn, ia), __fmul_rn(fn, ib)), 1.0f);
             const uint32_t okr = (ok_i && u < ncol) ? 1u : 0u, okc = (okr && has_c) ? 1u : 0u;
-            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p " STG_OUT ".f32 [%0], %1;\n\t}" ::"l"(
                              r2b + off),
                          "f"(r2v), "r"(okr)
                          : "memory");
-            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p " STG_OUT ".u32 [%0], %1;\n\t}" ::"l"(
                              cb + off),
                          "r"(c[u]), "r"(okc)
                          : "memory");
@@ -234,7 +248,7 @@ __device__ __forceinline__ void epi_mirror(const GArgs &args, const uint32_t (&c
         if (EPI == EPI_COUNTS) {
             const uint32_t x = args.op == 0 ? cu : pl + pb - 2u * cu;   // AND or XOR (symmetric)
             if (args.accumulate) args.C[o] += x;
-            else __stcs(args.C + o, x);
+            else STG_OUT_FN(args.C + o, x);
         } else {
             float r2v, dpv = 0.f;
             if (small_n) {
@@ -250,9 +264,9 @@ __device__ __forceinline__ void epi_mirror(const GArgs &args, const uint32_t (&c
             } else {
                 ld_stats_f32(n, (int64_t)pl, (int64_t)pb, (int64_t)cu, r2v, dpv);
             }
-            __stcs(args.r2 + o, r2v);
-            if (want_dp) __stcs(args.dprime + o, dpv);
-            if (args.C) __stcs(args.C + o, cu);
+            STG_OUT_FN(args.r2 + o, r2v);
+            if (want_dp) STG_OUT_FN(args.dprime + o, dpv);
+            if (args.C) STG_OUT_FN(args.C + o, cu);
         }
     }
 }
@@ -346,7 +360,7 @@ __device__ __forceinline__ void copy_out_v4(const uint32_t *tw, int lane, uint32
         const int r = 4 * it + rsub;
         uint4 x = *reinterpret_cast<const uint4 *>(tw + r * 32 + ((cchunk ^ (r & 7)) << 2));
         uint4 *d = reinterpret_cast<uint4 *>(dst + off0 + (uint32_t)r * ld32 + 4u * (uint32_t)cchunk);
-        __stcs(d, x);
+        STG_OUT_FN(d, x);
     }
 }
 __device__ __forceinline__ void epi_ld_fast_v4(const GArgs &args, const uint32_t (&c)[32], uint32_t *tw, int lane,
@@ -468,7 +482,7 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
             const uint32_t x = op == 0 ? c : op == 1 ? plr + pcol - 2u * c : op == 2 ? plr - c : pcol - c;
             if (colok) {
                 if (acc) *cp += x;
-                else __stcs(cp, x);
+                else STG_OUT_FN(cp, x);
             }
             cp += ldo;
         }
@@ -501,11 +515,11 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
             const float r2v = fminf(__fmul_rn(__fmul_rn(fn, iar), __fmul_rn(fn, ib)), 1.0f);
             // predicated evict-first stores (outputs are written once; the packed operands
             // stay in L2): no branch, so the shuffles stay in a converged straight line
-            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.f32 [%0], %1;\n\t}" ::"l"(
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p " STG_OUT ".f32 [%0], %1;\n\t}" ::"l"(
                              r2b + off),
                          "f"(r2v), "r"(okr)
                          : "memory");
-            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.cs.u32 [%0], %1;\n\t}" ::"l"(
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p " STG_OUT ".u32 [%0], %1;\n\t}" ::"l"(
                              cb + off),
                          "r"(c), "r"(okc)
                          : "memory");
@@ -528,8 +542,8 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
             const float fn = (float)num;
             const float r2v = fminf(__fmul_rn(__fmul_rn(fn, iar), __fmul_rn(fn, ib)), 1.0f);
             if (colok) {
-                __stcs(rp, r2v);   // outputs are written once: evict-first keeps the packed
-                if (cp) __stcs(cp, (uint32_t)c);   // operands resident in L2
+                STG_OUT_FN(rp, r2v);   // outputs are written once: evict-first keeps the packed
+                if (cp) STG_OUT_FN(cp, (uint32_t)c);   // operands resident in L2
             }
             rp += ldo;
             if (cp) cp += ldo;
@@ -558,9 +572,9 @@ __device__ __forceinline__ void epi_transposed(const GArgs &args, uint32_t (&c)[
         } else {
             ld_stats_f32(n, (int64_t)plr, (int64_t)pb, (int64_t)cr, r2v, dpv);
         }
-        __stcs(args.r2 + o, r2v);
-        if (want_dp) __stcs(args.dprime + o, dpv);
-        if (args.C) __stcs(args.C + o, cr);
+        STG_OUT_FN(args.r2 + o, r2v);
+        if (want_dp) STG_OUT_FN(args.dprime + o, dpv);
+        if (args.C) STG_OUT_FN(args.C + o, cr);
     }
 }
 
@@ -595,12 +609,12 @@ __device__ __forceinline__ void epi_swapped_counts(const GArgs &args, uint32_t (
         const uint32_t x1 = cc1 * c + (cq1 * pq + b1);
         if (ok) {
             if (acc) *o1 += x1;
-            else __stcs(o1, x1);
+            else STG_OUT_FN(o1, x1);
         }
         o1 += ldo;
         if (two) {
             const uint32_t x2 = cc2 * c + (cq2 * pq + b2);
-            if (ok) __stcs(o2, x2);
+            if (ok) STG_OUT_FN(o2, x2);
             o2 += ldo;
         }
     }
@@ -959,6 +973,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 __syncwarp();            // tcgen05.ld is warp-collective: re-converge first
                 ptx::tmem_ld32(ta + 32 * hh, v);
                 ptx::tmem_ld_wait();
+                GEMM_T3B(2 * hh, tl == 0 && e == 0 && lane == 0);
                 if (hh == 1) {
                     ptx::tc_fence_before();
                     __syncwarp();
@@ -968,6 +983,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 if (!args.swap) {
                     epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, erow0, ecol0 + 32 * hh, pl, pcol,
                                         ia, small_n, want_dp, mirror);
+                    GEMM_T3B(2 * hh + 1, tl == 0 && e == 0 && lane == 0);
                     continue;
                 }
                 if (EPI == EPI_COUNTS) {
@@ -1004,7 +1020,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                                                  : op == 2 ? pq - c[k] : pd - c[k];
                                 uint32_t *o = Cb + (gc0 + u0 + k) * ldo + gl;
                                 if (args.accumulate) *o += r;
-                                else __stcs(o, r);
+                                else STG_OUT_FN(o, r);
                             }
                         }
                     } else {
@@ -1597,6 +1613,11 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
 }  // namespace snp
 
 #ifdef SNP_PROFILING
+extern "C" int snp_debug_gemm_cta2(long long *host, int n) {
+    if (n > 8 * 1024) n = 8 * 1024;
+    return (int)cudaMemcpyFromSymbol(host, snp::g_gemm_cta2, sizeof(long long) * n);
+}
+
 extern "C" int snp_debug_gemm_cta(long long *host, int n) {
     if (n > 8 * 1024) n = 8 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_gemm_cta, sizeof(long long) * n);

@@ -87,3 +87,89 @@ def stream_search(Q: torch.Tensor, D_host: torch.Tensor, nbits: int, ops=("xor",
         buf.record_stream(copy)
     bc[:, :len(plan)] = cnt32.view(torch.int32).to(torch.int64) & 0xFFFFFFFF
     return [merge_best(bc[j], bi[j]) for j in range(nops)]
+
+
+def ld_block_plan(m: int, block_tiles: int) -> list[tuple[int, int, int, int]]:
+    """Row blocks of block_tiles tile rows in the order they are streamed (last first), each
+    with the packed-triangle tile range it completes: (I0, I1, tile_lo, tile_hi).  Tile row I
+    holds tiles (I, J), J >= I, so it needs only row blocks >= I — all of which arrive no
+    later than block I (host logic, covered by tests on CPU)."""
+    T = -(-m // 128)
+
+    def start(I):      # first tile of tile row I (row-major upper triangle)
+        return I * T - I * (I - 1) // 2
+    return [(b0, min(T, b0 + block_tiles), start(b0), start(min(T, b0 + block_tiles)))
+            for b0 in range(0, T, block_tiles)][::-1]
+
+
+def stream_ld_sym(A_host: torch.Tensor, nbits: int, block_tiles: int = 16, r2: bool = True, counts: bool = True,
+                  dprime: bool = False, out_host: dict | None = None, device=None):
+    """f2 for LD — end-to-end symmetric self-LD from a packed matrix in pinned host memory
+    (the paper's end-to-end mode, §VI.A: input and output transfers double-buffered
+    and overlapped with the kernels; Fig. 6).
+
+    Row blocks of ``block_tiles`` x 128 SNPs are copied host -> device on a copy stream in
+    REVERSE order; tile row I of the packed upper triangle (``snp_ld_sym``) needs only row
+    blocks >= I, so as soon as block b has arrived (all later ones arrived before it) its
+    tile rows are computed on the compute stream while block b - 1 is in flight.  Row
+    popcounts are counted per block as it lands.  With ``out_host`` (dict of pinned host
+    tensors 'r2' / 'counts' / 'dprime' shaped like the device outputs) each block's tiles are
+    copied back on a second copy stream while the next block computes.
+
+    Returns dict of device outputs ([snp_sym_tiles(m)][128][128]) and the device matrix."""
+    from . import snp_ld_sym, snp_row_popc, snp_sym_tiles
+    if A_host.is_cuda or not A_host.is_pinned():
+        raise ValueError("A_host must be a pinned CPU tensor")
+    if block_tiles < 1:
+        raise ValueError("block_tiles >= 1")
+    dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+    m = A_host.shape[0]
+    T = -(-m // 128)
+    ntot = snp_sym_tiles(m)
+    A = torch.empty(A_host.shape, dtype=A_host.dtype, device=dev)
+    pop = torch.empty(m, dtype=torch.uint32, device=dev)
+    outs = {}
+    if r2:
+        outs["r2"] = torch.empty((ntot, 128, 128), dtype=torch.float32, device=dev)
+    if dprime:
+        outs["dprime"] = torch.empty((ntot, 128, 128), dtype=torch.float32, device=dev)
+    if counts:
+        outs["counts"] = torch.empty((ntot, 128, 128), dtype=torch.uint32, device=dev)
+    if not outs:
+        raise ValueError("nothing requested")
+    comp = torch.cuda.current_stream(dev)
+    h2d, d2h = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+    h2d.wait_stream(comp)
+    d2h.wait_stream(comp)
+
+    plan = ld_block_plan(m, block_tiles)
+    blocks = [(I0, I1) for I0, I1, _, _ in plan]
+    arrived = []
+    for I0, I1 in blocks:                       # all H2D copies queued up front, last block first
+        r0, r1 = I0 * 128, min(m, I1 * 128)
+        with torch.cuda.stream(h2d):
+            A[r0:r1].copy_(A_host[r0:r1], non_blocking=True)
+            ev = torch.cuda.Event()
+            ev.record(h2d)
+        arrived.append(ev)
+    for (I0, I1, lo, hi), ev in zip(plan, arrived):
+        r0, r1 = I0 * 128, min(m, I1 * 128)
+        comp.wait_event(ev)
+        snp_row_popc(A[r0:r1], nbits, out=pop[r0:r1])
+        snp_ld_sym(A, nbits, lo, hi, popA=pop, r2=outs.get("r2", False)[lo:hi] if r2 else False,
+                   dprime=outs["dprime"][lo:hi] if dprime else None,
+                   counts=outs["counts"][lo:hi] if counts else None)
+        if out_host is not None:
+            done = torch.cuda.Event()
+            done.record(comp)
+            d2h.wait_event(done)
+            with torch.cuda.stream(d2h):
+                for k, t in outs.items():
+                    if k in out_host:
+                        out_host[k][lo:hi].copy_(t[lo:hi], non_blocking=True)
+    comp.wait_stream(d2h)
+    comp.wait_stream(h2d)
+    for t in [A, pop, *outs.values()]:
+        t.record_stream(h2d)
+        t.record_stream(d2h)
+    return outs, A

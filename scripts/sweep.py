@@ -14,6 +14,8 @@ ap.add_argument("--M", default="1,2,4,8,16,32,64,128,256,1024,4096,8192")
 ap.add_argument("--N", default="1000000,4000000")
 ap.add_argument("--K", default="2048,4096,8192,16384")
 ap.add_argument("--max-popc-s", type=float, default=0.4)
+ap.add_argument("--tight", action="store_true", help="packed rows of ceil(nbits/64) (even) words, no padding")
+ap.add_argument("--counts", action="store_true", help="also write the count matrix (else best only)")
 a = ap.parse_args()
 torch.cuda.set_device(0)
 POPC_RATE = 1.2e14          # comparisons/s, measured (~86% of the POPC pipe peak)
@@ -31,20 +33,22 @@ def timeit(fn, reps=5):
 
 rows = []
 for K in [int(x) for x in a.K.split(",")]:
-    w = snp.snp_words(K)
+    w = snp.snp_words(K) if not a.tight else ((K + 63) // 64 + 1) // 2 * 2
     for N in [int(x) for x in a.N.split(",")]:
         D = torch.randint(-2**62, 2**62, (N, w), dtype=torch.int64, device="cuda").view(torch.uint64)
         pd = snp.snp_row_popc(D, K)
         for M in [int(x) for x in a.M.split(",")]:
             Q = torch.randint(-2**62, 2**62, (M, w), dtype=torch.int64, device="cuda").view(torch.uint64)
-            rec = {"M": M, "N": N, "nbits": K, "cmp": M * N * K}
+            rec = {"M": M, "N": N, "nbits": K, "cmp": M * N * K, "ldw": w, "counts": bool(a.counts),
+                   "bytes": N * w * 8 + (M * N * 4 if a.counts else 0)}
             for v in ("tc", "popc"):
                 if v == "popc" and M * N * K / POPC_RATE > a.max_popc_s:
                     rec[v + "_ms"] = None
                     continue
                 snp.snp_set_variant(v)
                 ws = torch.empty(snp.snp_fastid_search_workspace_bytes(M, N, K, 1), dtype=torch.uint8, device="cuda")
-                ms = timeit(lambda: snp.snp_fastid_search(Q, D, K, ("xor",), counts=False, best=True, ws=ws, popD=pd))
+                outc = [torch.empty((M, N), dtype=torch.uint32, device="cuda")] if a.counts else False
+                ms = timeit(lambda: snp.snp_fastid_search(Q, D, K, ("xor",), counts=outc, best=True, ws=ws, popD=pd))
                 rec[v + "_ms"] = ms
                 rec[v + "_kernel"] = snp.snp_last_kernel()
                 del ws
@@ -57,6 +61,6 @@ for K in [int(x) for x in a.K.split(",")]:
             del Q
         del D, pd
         torch.cuda.empty_cache()
-print("M\\tN\\tnbits\\ttc_ms\\tpopc_ms\\twinner\\ttc Tcmp/s", file=sys.stderr)
+print("M\\tN\\tnbits\\ttc_ms\\tpopc_ms\\twinner\\ttc Tcmp/s\\tbest GB/s", file=sys.stderr)
 for r in rows:
-    print(f"{r['M']}\t{r['N']}\t{r['nbits']}\t{r['tc_ms']:.3f}\t{r['popc_ms'] if r['popc_ms'] is None else round(r['popc_ms'], 3)}\t{r['winner']}\t{r['tc_cmp_per_s']/1e12:.0f}", file=sys.stderr)
+    print(f"{r['M']}\t{r['N']}\t{r['nbits']}\t{r['tc_ms']:.3f}\t{r['popc_ms'] if r['popc_ms'] is None else round(r['popc_ms'], 3)}\t{r['winner']}\t{r['tc_cmp_per_s']/1e12:.0f}\t{r['bytes'] / min(x for x in (r['tc_ms'], r['popc_ms']) if x) / 1e6:.0f}", file=sys.stderr)

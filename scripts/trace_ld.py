@@ -35,3 +35,10 @@ names = ["entry", "setup done", "gdc.wait done", "1st stage in", "1st acc ready"
 for k, nm in enumerate(names):
     x = (t[:, k] - t0) / 1e3
     print(f"{nm:18s} min {x.min():7.2f}  med {np.median(x):7.2f}  max {x.max():7.2f} us")
+
+b2 = (ctypes.c_longlong * 8192)()
+snp.lib().snp_debug_gemm_cta2(b2, 8192)
+u = np.array(b2, dtype=np.int64).reshape(1024, 8)[:grid, :4].astype(np.float64)
+for k, nm in enumerate(["TMEM ld half 0", "block half 0 done", "TMEM ld half 1", "block half 1 done"]):
+    x = (u[:, k] - t0) / 1e3
+    print(f"{nm:18s} min {x.min():7.2f}  med {np.median(x):7.2f}  max {x.max():7.2f} us")

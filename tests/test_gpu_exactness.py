@@ -149,6 +149,7 @@ sys.path.insert(0, ".")
 import oracle, snpgen
 import paper_conf_ipps_binderlp19_b200 as snp
 torch.cuda.set_device(0)
+snp.snp_set_variant("tc")          # the tensor variant (AUTO streams <= 3 queries on CUDA cores)
 rng = np.random.default_rng(7)
 def rows(r, k, p):
     return (rng.random((r, k), dtype=np.float32) < p).astype(np.uint8)

@@ -804,3 +804,57 @@ def test_fastid_stream_ties_lowest_index(snp):
     assert int(best[0][0][1]) == 0 and int(best[0][1][1]) == 40_000
     rb, ri = oracle.best(oracle.counts(q, db, "xor"))
     assert np.array_equal(u32(best[0][0]), rb) and np.array_equal(best[0][1].cpu().numpy(), ri)
+
+
+@pytest.mark.parametrize("with_host_out", [False, True])
+def test_stream_ld_sym_end_to_end(snp, with_host_out):
+    """f2 for LD: packed matrix in pinned host memory streamed in reverse row blocks, tile
+    rows computed as their blocks land, outputs optionally copied back block by block;
+    counts / r2 equal the oracle's (through snp_sym_unpack) and the resident snp_ld_sym."""
+    from paper_conf_ipps_binderlp19_b200.stream import stream_ld_sym
+    m, nbits = 900, 1100
+    g = snpgen.ld_genotypes(66, np.arange(m), nbits, structure=True)
+    A_dev = pack_dev(snp, g)
+    A_host = A_dev.cpu().pin_memory()
+    nt = snp.snp_sym_tiles(m)
+    host = ({"r2": torch.empty((nt, 128, 128), dtype=torch.float32).pin_memory(),
+             "counts": torch.empty((nt, 128, 128), dtype=torch.int32).pin_memory()} if with_host_out else None)
+    outs, _ = stream_ld_sym(A_host, nbits, block_tiles=2, out_host=host)
+    torch.cuda.synchronize()
+    r2_ref, _, n_ref = oracle.ld(g, g)
+    assert np.array_equal(u32(snp.snp_sym_unpack(outs["counts"], m)), n_ref)
+    check_r2(snp.snp_sym_unpack(outs["r2"], m).cpu().numpy(), r2_ref)
+    r2w, _, cw = snp.snp_ld_sym(A_dev, nbits, counts=True)
+    assert torch.equal(cw, outs["counts"]) and torch.equal(r2w, outs["r2"])
+    if host is not None:
+        assert np.array_equal(host["counts"].numpy().view(np.uint32), u32(cw))
+        assert torch.equal(host["r2"], r2w.cpu())
+
+
+@pytest.mark.parametrize("ldw", [2, 4, 6])
+@pytest.mark.parametrize("nq", [1, 3, 32, 100])
+def test_narrow_rows_short_profiles(snp, ldw, nq):
+    """The paper's FastID profiles are 128-1024 SNPs (Fig. 8): packed rows as
+    narrow as 2 words (16 bytes, no padding to the recommended 64) are valid input for every
+    op, the fused search and LD; results vs the oracle."""
+    nbits = 64 * ldw - 5
+    nd = 3000
+    db = snpgen.fastid_db(83, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(83, nq, nd, nbits)
+    D = pack_dev(snp, db, ldw=ldw, garbage_seed=1)
+    Q = pack_dev(snp, q, ldw=ldw, garbage_seed=2)
+    counts, best = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), index_base=2)
+    for j, op in enumerate(("xor", "andnot")):
+        ref = oracle.counts(q, db, op)
+        assert np.array_equal(u32(counts[j]), ref), (op, snp.snp_last_kernel())
+        rb, ri = oracle.best(ref, 2)
+        assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), op
+    assert np.array_equal(u32(snp.snp_fastid(Q, D, nbits, "and")), oracle.counts(q, db, "and"))
+    g = snpgen.ld_genotypes(84, np.arange(300), nbits, structure=True)
+    A = pack_dev(snp, g, ldw=ldw)
+    r2, _, cnt = snp.snp_ld_r2(A, A, nbits, counts=True)
+    r2_ref, _, n_ref = oracle.ld(g, g)
+    assert np.array_equal(u32(cnt), n_ref)
+    check_r2(r2.cpu().numpy(), r2_ref)
+    _, _, ct = snp.snp_ld_sym(A, nbits, r2=False, counts=True)
+    assert np.array_equal(u32(snp.snp_sym_unpack(ct, 300)), n_ref)

@@ -219,3 +219,24 @@ def test_two_rank_gloo_symmetric_ld_plan():
         assert ok, f"rank {rank}: reconstructed symmetric matrix != oracle"
         assert nseen == 6                      # T = 3 tiles per side: 6 upper-triangle tiles
         assert mine == 3                       # balanced: 3 + 3
+
+
+@pytest.mark.parametrize("m,bt", [(1, 1), (128, 4), (700, 2), (2048, 16), (32768, 16), (5000, 3)])
+def test_stream_ld_block_plan(m, bt):
+    """f2 for LD host logic: blocks streamed last-first; together their tile ranges cover
+    every packed-triangle tile exactly once, in contiguous pieces; every tile of a block's
+    range needs only rows of that block or of blocks streamed before it."""
+    from paper_conf_ipps_binderlp19_b200.multigpu import sym_tile_coords
+    from paper_conf_ipps_binderlp19_b200.stream import ld_block_plan
+    T = -(-m // 128)
+    plan = ld_block_plan(m, bt)
+    assert [p[0] for p in plan] == sorted([p[0] for p in plan], reverse=True)
+    covered = sorted((lo, hi) for _, _, lo, hi in plan)
+    assert covered[0][0] == 0 and covered[-1][1] == T * (T + 1) // 2
+    assert all(a[1] == b[0] for a, b in zip(covered, covered[1:]))
+    arrived_from = T
+    for I0, I1, lo, hi in plan:
+        arrived_from = I0                      # rows >= 128 * I0 are on the device now
+        for t in ([lo, hi - 1] if hi - lo > 2 else range(lo, hi)):
+            I, J = sym_tile_coords(m, t)
+            assert I0 <= I < I1 and J >= arrived_from
