@@ -542,13 +542,19 @@ def setup_ld_tri(wl, rank, world, dev):
             if host:
                 G.copy_(Ghost, non_blocking=True)                           # e2e H2D
             snp.snp_pack_popc(G, nbits=nbits, out=B, popc=pop)             # a1 + a2
-        if world > 1:
-            import torch.distributed as dist
-            dist.broadcast(B.view(torch.int64), src=0)
-            dist.broadcast(pop.view(torch.int32), src=0)
         if kev is not None:
             kev[0].record(s)
-        compute()
+        if world > 1:
+            # packed matrix broadcast in row blocks (last first), each rank's tiles computed as
+            # the blocks they read land (SURVEY §8e overlap); popcounts counted per block
+            from paper_conf_ipps_binderlp19_b200 import multigpu
+            multigpu.ld_sym_step_overlapped(
+                B, nbits, lo, hi, block_tiles=16,
+                compute=lambda B_, a, b_: snp.snp_ld_sym(B_, nbits, a, b_, popA=pop, r2=r2[a - lo:b_ - lo],
+                                                         counts=cnt[a - lo:b_ - lo]),
+                popc=(None if rank == 0 else lambda r0, r1: snp.snp_row_popc(B[r0:r1], nbits, out=pop[r0:r1])))
+        else:
+            compute()
         if kev is not None:
             kev[1].record(s)
         if host:   # e2e: D2H of the step's result statistic (r2 of the first pair)

@@ -77,9 +77,33 @@ __global__ void pack_popc_kernel(const uint8_t *__restrict__ g, int64_t rows, in
     const int lane = threadIdx.x & 31;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t fullw = nbits / 64;            // words entirely inside nbits
     for (int64_t r = warp; r < rows; r += nwarps) {
         uint32_t c = 0;
-        for (int64_t w = lane; w < ldw; w += 32) {
+        int64_t w = lane;
+        if (VEC) {
+            // two full words per lane per round, all 8 loads issued before any is consumed
+            // (memory-level parallelism: the LD step's first kernel is latency-bound otherwise)
+            for (; w + 32 < fullw; w += 64) {
+                const uint4 *p0 = reinterpret_cast<const uint4 *>(g + r * ldg + w * 64);
+                const uint4 *p1 = reinterpret_cast<const uint4 *>(g + r * ldg + (w + 32) * 64);
+                uint4 v0[4], v1[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) { v0[q] = __ldg(p0 + q); v1[q] = __ldg(p1 + q); }
+                uint64_t a = 0, b = 0;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    a |= (uint64_t)nonzero_bits8(((uint64_t)v0[q].y << 32) | v0[q].x) << (16 * q);
+                    a |= (uint64_t)nonzero_bits8(((uint64_t)v0[q].w << 32) | v0[q].z) << (16 * q + 8);
+                    b |= (uint64_t)nonzero_bits8(((uint64_t)v1[q].y << 32) | v1[q].x) << (16 * q);
+                    b |= (uint64_t)nonzero_bits8(((uint64_t)v1[q].w << 32) | v1[q].z) << (16 * q + 8);
+                }
+                packed[r * ldw + w] = a;
+                packed[r * ldw + w + 32] = b;
+                c += __popcll(a) + __popcll(b);
+            }
+        }
+        for (; w < ldw; w += 32) {
             const int64_t k0 = w * 64;
             uint64_t word = 0;
             if (k0 < nbits) {

@@ -79,7 +79,12 @@ bool make_map_u32_2d(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_
     const cuuint32_t box[2] = {box_words, box_rows};
     const cuuint32_t estr[2] = {1, 1};
     return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<uint32_t *>(base), dims, strides, box, estr,
-               CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle,
+#ifdef SNP_TMA_L2_PROMO_NONE
+               CU_TENSOR_MAP_L2_PROMOTION_NONE,   // measurement variant
+#else
+               CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+#endif
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 

@@ -135,3 +135,36 @@ def ld_sym_step(B: torch.Tensor, nbits: int, tile_lo: int, tile_hi: int, compute
     if world > 1:
         dist.broadcast(B.view(torch.int64) if B.dtype == torch.uint64 else B, src=0, group=group)
     return compute(B, tile_lo, tile_hi)
+
+
+def ld_sym_step_overlapped(B: torch.Tensor, nbits: int, tile_lo: int, tile_hi: int, block_tiles: int = 16,
+                           compute=None, popc=None, group=None):
+    """Symmetric self-LD step with the packed-matrix broadcast chunked and overlapped with the
+    tiles ("chunk the broadcast into column blocks and overlap it with compute").
+
+    Row blocks of ``block_tiles`` x 128 SNPs are broadcast from rank 0 LAST block first
+    (stream.ld_block_plan); tile row I of the packed triangle needs only row blocks >= I, so
+    after each block lands this rank computes the part of its range [tile_lo, tile_hi) that
+    block completes, while the next block is in flight (NCCL ops are asynchronous on their
+    own stream; each compute waits only for the blocks it reads).  Row popcounts of a block
+    are counted locally as it lands (``popc(block_rows)``) instead of being broadcast.
+
+    compute(B, lo, hi) -> result for tiles [lo, hi); returns the list of (lo, hi, result)."""
+    from .stream import ld_block_plan
+    if compute is None:
+        from . import snp_ld_sym
+        compute = lambda B_, lo_, hi_: snp_ld_sym(B_, nbits, lo_, hi_, counts=True)   # noqa: E731
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    out = []
+    for I0, I1, blo, bhi in ld_block_plan(B.shape[0], block_tiles):
+        r0, r1 = I0 * 128, min(B.shape[0], I1 * 128)
+        if world > 1:
+            work = dist.broadcast((B.view(torch.int64) if B.dtype == torch.uint64 else B)[r0:r1], src=0,
+                                  group=group, async_op=True)
+            work.wait()          # orders this block's consumers after its arrival (stream-ordered on NCCL)
+        if popc is not None:
+            popc(r0, r1)
+        lo, hi = max(tile_lo, blo), min(tile_hi, bhi)
+        if lo < hi:
+            out.append((lo, hi, compute(B, lo, hi)))
+    return out

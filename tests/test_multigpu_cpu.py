@@ -240,3 +240,67 @@ def test_stream_ld_block_plan(m, bt):
         for t in ([lo, hi - 1] if hi - lo > 2 else range(lo, hi)):
             I, J = sym_tile_coords(m, t)
             assert I0 <= I < I1 and J >= arrived_from
+
+
+def _sym_overlap_worker(rank, world, port, q):
+    try:
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        from paper_conf_ipps_binderlp19_b200 import multigpu, snp_shard_plan_sym
+        m, nbits = 700, 130
+        g = snpgen.ld_genotypes(80, np.arange(m), nbits, structure=True)
+        B = torch.from_numpy(oracle.pack(g, 4).view(np.int64)) if rank == 0 else torch.zeros((m, 4), dtype=torch.int64)
+        b = snp_shard_plan_sym(m, world)
+        lo, hi = b[rank], b[rank + 1]
+        seen_rows = []
+
+        def tiles_compute(B_, lo_, hi_):
+            gg = oracle.unpack(B_.numpy().view(np.uint64), nbits)
+            res = {}
+            for t in range(lo_, hi_):
+                I, J = multigpu.sym_tile_coords(m, t)
+                # every row this tile reads must have arrived already
+                assert all(min(seen_rows) <= 128 * x for x in (I, J))
+                res[t] = oracle.ld(gg[128 * I:128 * I + 128], gg[128 * J:128 * J + 128])[2]
+            return res
+
+        parts = multigpu.ld_sym_step_overlapped(B, nbits, lo, hi, block_tiles=2, compute=tiles_compute,
+                                                popc=lambda r0, r1: seen_rows.append(r0))
+        mine = {}
+        for plo, phi, res in parts:
+            assert lo <= plo < phi <= hi
+            mine.update(res)
+        got = [None] * world
+        dist.all_gather_object(got, mine)
+        full = np.full((m, m), -1, dtype=np.int64)
+        for d in got:
+            for t, blk in d.items():
+                I, J = multigpu.sym_tile_coords(m, t)
+                full[128 * I:128 * I + blk.shape[0], 128 * J:128 * J + blk.shape[1]] = blk
+                full[128 * J:128 * J + blk.shape[1], 128 * I:128 * I + blk.shape[0]] = blk.T
+        _, _, n_ref = oracle.ld(g, g)
+        q.put((rank, bool(np.array_equal(full, n_ref)), sorted(mine) == list(range(lo, hi))))
+        dist.destroy_process_group()
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, "error", traceback.format_exc()))
+
+
+def test_two_rank_gloo_symmetric_ld_overlapped_broadcast():
+    """e + f3: the packed matrix broadcast in row blocks (last first) overlapped with the
+    tiles each block completes; every rank computes exactly its tile range, no tile reads a
+    row that has not arrived, and the union equals the oracle's full count matrix."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sym_overlap_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for r in res:
+        assert r[1] != "error", r[2]
+        assert r[1] and r[2], r
