@@ -748,17 +748,17 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     CUtensorMap tm;
     if (!make_map_u32_2d(&tm, a.D, a.nd, a.ldd32, KBITS / 32, BM,
                          KBITS == 1024 ? CU_TENSOR_MAP_SWIZZLE_128B
-                         : KBITS == 512 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B))
+                         : KBITS == 512 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B, a.dcols32))
         return cudaErrorInvalidValue;
 
     using KernFn = void (*)(const CUtensorMap, const FArgs);
     const bool best = f.best_mask != 0;
     KernFn kern = nullptr;
     int nthreads = Roles<GG>::NTHREADS;   // the runtime-coefficient kernels are GG = 4 only
-    if (a.accumulate) {
+    if (a.accumulate) {   // K-chunked searches add each chunk's counts (one or two ops per pass)
         nthreads = Roles<4>::NTHREADS;
-        if (a.nops != 1 || best) return cudaErrorInvalidValue;
-        kern = fastid_tc4_kernel<BN, 1, false, true, -1, 4>;
+        if (a.nops > 2 || best) return cudaErrorInvalidValue;
+        kern = a.nops == 1 ? fastid_tc4_kernel<BN, 1, false, true, -1, 4> : fastid_tc4_kernel<BN, 2, false, true, -1, 4>;
     } else if (a.nops == 1) {   // compile-time op
         static KernFn k1[2][4] = {{fastid_tc4_kernel<BN, 1, false, false, 0, GG>, fastid_tc4_kernel<BN, 1, false, false, 1, GG>,
                                    fastid_tc4_kernel<BN, 1, false, false, 2, GG>, fastid_tc4_kernel<BN, 1, false, false, 3, GG>},

@@ -71,10 +71,10 @@ EncodeTiledFn tensor_map_encoder() {
 }
 
 bool make_map_u32_2d(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32, uint32_t box_words,
-                     uint32_t box_rows, CUtensorMapSwizzle swizzle) {
+                     uint32_t box_rows, CUtensorMapSwizzle swizzle, int64_t cols32) {
     EncodeTiledFn enc = tensor_map_encoder();
     if (!enc) return false;
-    const cuuint64_t dims[2] = {(cuuint64_t)ld32, (cuuint64_t)rows};
+    const cuuint64_t dims[2] = {(cuuint64_t)(cols32 > 0 ? cols32 : ld32), (cuuint64_t)rows};
     const cuuint64_t strides[1] = {(cuuint64_t)ld32 * 4};
     const cuuint32_t box[2] = {box_words, box_rows};
     const cuuint32_t estr[2] = {1, 1};

@@ -484,6 +484,24 @@ int64_t search_slice_width(int64_t nq, int64_t nd, int64_t nbits) {
     return 0;
 }
 bool search_sliced(int64_t nq, int64_t nd, int64_t nbits) { return search_slice_width(nq, nd, nbits) != 0; }
+// Long profiles with <= 64 queries whose expanded batch does not fit the FastID kernel's shared
+// memory: the profiles are cut into K chunks (multiples of 1024 bits) that fit, each chunk one
+// pass of the FastID kernel over the database's chunk columns that ADDS its counts (every op is
+// linear in the chunk-local AND count and popcounts, so the sums are exact); the
+// database is read once in total instead of going to the general kernel.  Returns the chunk
+// size in bits, or 0 when the path does not apply.
+int64_t search_kchunk_bits(int64_t nq, int64_t nd, int64_t nbits) {
+    const char *e = std::getenv("SNP_SEARCH_KCHUNK");   // "0": never (A/B measurement hook)
+    if (e && e[0] == '0') return 0;
+    // measured (profiles/round2/sweep_kchunk.txt, best-only 4M x 16384): 8 queries 3.43 -> 2.09 ms,
+    // 16 about 8 % faster, 32 equal, 64 four times slower (the per-chunk count read-modify-write
+    // grows with the query count) than the general kernel: used up to 16 queries
+    if (nd <= 0 || nq < 1 || nq > 16 || nbits <= 1024 || choose_variant(nq, nd, nbits) != SNP_VARIANT_TC) return 0;
+    if (fastid_tc4_supported(nq, nd, nbits) || search_slice_width(nq, nd, nbits)) return 0;
+    for (int64_t cb = (nbits - 1) / 1024 * 1024; cb >= 1024; cb -= 1024)
+        if (fastid_tc4_supported(nq, nd, cb)) return cb;
+    return 0;
+}
 
 }  // namespace
 
@@ -495,6 +513,9 @@ size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, 
     if (nd > 0 && use_stream(nq, nd, nbits)) return fastid_stream_ws_bytes(nq, nops);
     if (search_fused(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(nq, nops);
     if (search_sliced(nq, nd, nbits)) return fastid_search_tc4_ws_bytes(search_slice_width(nq, nd, nbits), nops);
+    if (search_kchunk_bits(nq, nd, nbits))   // keys + per-op count chunks (for ops without stored counts)
+        return align256((size_t)nops * nq * 8) + (size_t)nops * align256((size_t)nq * search_chunk_rows(nq, nd) * 4) +
+               fastid_search_tc4_ws_bytes(nq, nops);
     size_t b = align256((size_t)nops * nq * 8);
     if (nd == 0) return b;
     b += align256((size_t)nq * search_chunk_rows(nq, nd) * 4);
@@ -597,6 +618,71 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
             b.done = reinterpret_cast<unsigned int *>((char *)ws + align256((size_t)nops * SLICE_Q * 8));
             if ((e = launch_fastid_search_tc4(b, s)) != cudaSuccess) return set_cuda_error(e);
         }
+        g_last_variant = SNP_VARIANT_TC;
+        g_last_kernel = SNP_KERNEL_FASTID_MXF4;
+        return SNP_OK;
+    }
+
+    if (const int64_t KC = search_kchunk_bits(nq, nd, nbits)) {
+        // K-chunked FastID kernel passes (see search_kchunk_bits): counts of every op land in
+        // the caller's matrix, or — for ops without stored counts — in workspace count chunks
+        // over database row blocks; best matches by best.cu from the summed counts
+        unsigned long long *keys = reinterpret_cast<unsigned long long *>(ws);
+        char *p = (char *)ws + align256((size_t)nops * nq * 8);
+        const int64_t ch = search_chunk_rows(nq, nd);
+        uint32_t *tmp[4];
+        for (int j = 0; j < nops; ++j) {
+            tmp[j] = reinterpret_cast<uint32_t *>(p);
+            p += align256((size_t)nq * ch * 4);
+        }
+        for (int j = 0; j < nops; ++j)
+            if (a.best_count[j] && (e = launch_best_init(keys + (int64_t)j * nq, nq, s)) != cudaSuccess)
+                return set_cuda_error(e);
+        bool all_stored = true;
+        for (int j = 0; j < nops; ++j) all_stored = all_stored && a.counts[j] != nullptr;
+        // database row blocks: the whole database when every op's counts are stored, else
+        // blocks of ch rows through the workspace chunks (ops with stored counts write in place)
+        const int64_t rstep = all_stored ? nd : ch;
+        for (int64_t r0 = 0; r0 < nd; r0 += rstep) {
+            const int64_t rows = nd - r0 < rstep ? nd - r0 : rstep;
+            for (int j0 = 0; j0 < nops; j0 += 2) {
+                // one pass for two ops whose counts go to the same kind of buffer, else one per op
+                const int nj = nops - j0 >= 2 ? 2 : 1;
+                const bool pair = nj == 2 && ((a.counts[j0] != nullptr) == (a.counts[j0 + 1] != nullptr));
+                for (int g0 = j0; g0 < j0 + nj; g0 += pair ? 2 : 1) {
+                    const int ng = pair ? 2 : 1;
+                    const bool in_place = a.counts[g0] != nullptr;
+                    for (int64_t k0 = 0; k0 < nbits; k0 += KC) {
+                        SearchArgs c{};
+                        c.Q = a.Q + k0 / 32; c.nq = nq; c.ldq32 = a.ldq32;
+                        c.D = a.D + r0 * a.ldd32 + k0 / 32; c.nd = rows; c.ldd32 = a.ldd32;
+                        c.dcols32 = a.ldd32 - k0 / 32;         // the rows' remaining words: no over-read
+                        c.popD = nullptr;                      // chunk-local popcounts, counted in-kernel
+                        c.nbits = nbits - k0 < KC ? nbits - k0 : KC;
+                        c.nops = ng;
+                        c.accumulate = k0 > 0 ? 1 : 0;
+                        c.ldo = in_place ? ldo : ch;
+                        for (int jj = 0; jj < ng; ++jj) {
+                            c.ops[jj] = ops[g0 + jj];
+                            c.counts[jj] = in_place ? a.counts[g0 + jj] + r0 : tmp[g0 + jj];
+                        }
+                        if ((e = launch_fastid_search_tc4(c, s)) != cudaSuccess) return set_cuda_error(e);
+                    }
+                }
+            }
+            for (int j = 0; j < nops; ++j) {
+                if (!a.best_count[j]) continue;
+                const uint32_t *cj = a.counts[j] ? a.counts[j] + r0 : tmp[j];
+                if ((e = launch_best_reduce(cj, nq, rows, a.counts[j] ? ldo : ch, r0, keys + (int64_t)j * nq, s)) !=
+                    cudaSuccess)
+                    return set_cuda_error(e);
+            }
+        }
+        for (int j = 0; j < nops; ++j)
+            if (a.best_count[j] &&
+                (e = launch_best_finalize(keys + (int64_t)j * nq, nq, index_base, a.best_count[j], a.best_index[j], s)) !=
+                    cudaSuccess)
+                return set_cuda_error(e);
         g_last_variant = SNP_VARIANT_TC;
         g_last_kernel = SNP_KERNEL_FASTID_MXF4;
         return SNP_OK;

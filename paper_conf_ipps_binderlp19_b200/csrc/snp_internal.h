@@ -19,8 +19,10 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t
                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 EncodeTiledFn tensor_map_encoder();
+// cols32 > 0: the rows hold only cols32 words from `base` (a column window of a wider matrix,
+// elements past it read as zero); 0: ld32
 bool make_map_u32_2d(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32, uint32_t box_words,
-                     uint32_t box_rows, CUtensorMapSwizzle swizzle);
+                     uint32_t box_rows, CUtensorMapSwizzle swizzle, int64_t cols32 = 0);
 
 // Epilogue kinds of the bit-GEMM.
 enum Epi : int {
@@ -93,6 +95,7 @@ struct SearchArgs {
     int64_t nq, ldq32;
     const uint32_t *D;   // [nd][ldd32] database
     int64_t nd, ldd32;
+    int64_t dcols32 = 0; // > 0: D is a column window of dcols32 words (K-chunked searches)
     const uint32_t *popD;     // [nd] database row popcounts or NULL (derived in-kernel)
     int64_t nbits;
     int nops;

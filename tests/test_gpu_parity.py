@@ -858,3 +858,30 @@ def test_narrow_rows_short_profiles(snp, ldw, nq):
     check_r2(r2.cpu().numpy(), r2_ref)
     _, _, ct = snp.snp_ld_sym(A, nbits, r2=False, counts=True)
     assert np.array_equal(u32(snp.snp_sym_unpack(ct, 300)), n_ref)
+
+
+@pytest.mark.parametrize("nq,nbits", [(8, 20000), (16, 13000), (12, 30000), (5, 33000)])
+@pytest.mark.parametrize("mode", ["counts", "best_only", "mixed"])
+def test_search_kchunked_long_profiles(snp, nq, nbits, mode, monkeypatch):
+    """<= 64 queries whose expanded batch does not fit the FastID kernel: K-chunked passes that
+    add their counts (one DB read in total); every op's counts and best matches vs the oracle,
+    with counts stored, best-only (workspace count chunks over row blocks) and mixed."""
+    monkeypatch.setenv("SNP_SEARCH_CHUNK_ROWS", "1024")      # several row blocks at this size
+    nd = 2600
+    db = snpgen.fastid_db(85, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(85, nq, nd, nbits)
+    q[0] = db[2100]
+    D = pack_dev(snp, db, garbage_seed=6)
+    Q = pack_dev(snp, q, garbage_seed=7)
+    ops = ("and", "xor", "andnot", "notand")
+    counts = {"counts": True, "best_only": False,
+              "mixed": [torch.empty((nq, nd), dtype=torch.uint32, device=DEV), None, None,
+                        torch.empty((nq, nd), dtype=torch.uint32, device=DEV)]}[mode]
+    c, best = snp.snp_fastid_search(Q, D, nbits, ops, counts=counts, index_base=4)
+    assert snp.snp_last_kernel() == "fastid_mxf4"
+    for j, op in enumerate(ops):
+        ref = oracle.counts(q, db, op)
+        if c[j] is not None:
+            assert np.array_equal(u32(c[j]), ref), (op, mode)
+        rb, ri = oracle.best(ref, 4)
+        assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), (op, mode)
