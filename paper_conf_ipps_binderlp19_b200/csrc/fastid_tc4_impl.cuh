@@ -224,7 +224,15 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     }
     const int64_t nbits = args.nbits;
     const int nst = args.nst;
+#ifndef FASTID_CONTIG_TILES
+    // tile tl of this CTA is blockIdx.x + tl * gridDim.x (the CTAs sweep the database together)
     const int64_t my_tiles = args.ntiles > blockIdx.x ? (args.ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const int64_t tile0 = blockIdx.x, tstep = gridDim.x;
+#else
+    // measurement variant: each CTA takes one contiguous block of tiles
+    const int64_t tile0 = args.ntiles * blockIdx.x / gridDim.x, tstep = 1;
+    const int64_t my_tiles = args.ntiles * (blockIdx.x + 1) / gridDim.x - tile0;
+#endif
     const int64_t total_it = my_tiles * nst;
     const int64_t full32 = nbits / 32;
 
@@ -313,7 +321,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             int p = 0;
             uint32_t round = 0;   // how many times the ring has wrapped
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
-                const int64_t t = blockIdx.x + tl * gridDim.x;
+                const int64_t t = tile0 + tl * tstep;
                 const int32_t row0 = (int32_t)(t * BM);
                 for (int s = 0; s < nst; ++s) {
                     if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
@@ -539,7 +547,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)((uint32_t)tl % NACC);
             const uint32_t ph = ((uint32_t)tl / NACC) & 1u;
-            const int64_t t = blockIdx.x + tl * gridDim.x;
+            const int64_t t = tile0 + tl * tstep;
             const bool pre = args.popDg != nullptr;
             const int64_t gd_l = t * BM + li;   // this lane's local database row
             uint32_t pd = 0;
