@@ -601,12 +601,20 @@ __device__ __forceinline__ void epi_swapped_counts(const GArgs &args, uint32_t (
     const uint32_t b1 = cd1 * pl, b2 = cd2 * pl;   // database-row terms (this lane)
     uint32_t *o1 = args.C + col0 * ldo + gl;
     uint32_t *o2 = two ? args.C2 + col0 * ldo + gl : nullptr;
+#ifdef GEMM_DEBUG_NOSTORE
+    uint32_t sink = 0;
+#endif
 #pragma unroll
     for (int u = 0; u < 32; ++u) {
         const uint32_t pq = __shfl_sync(0xffffffffu, pcol, u);   // query popcount of column u
         const uint32_t c = acc_count(v[u], small);
         const bool ok = rowok && u < ncols;
         const uint32_t x1 = cc1 * c + (cq1 * pq + b1);
+#ifdef GEMM_DEBUG_NOSTORE   // profiling experiment: the epilogue without its stores (results invalid)
+        sink ^= x1;
+        if (two) sink ^= cc2 * c + (cq2 * pq + b2);
+        continue;
+#endif
         if (ok) {
             if (acc) *o1 += x1;
             else STG_OUT_FN(o1, x1);
@@ -618,6 +626,9 @@ __device__ __forceinline__ void epi_swapped_counts(const GArgs &args, uint32_t (
             o2 += ldo;
         }
     }
+#ifdef GEMM_DEBUG_NOSTORE
+    if (sink == 0x9e3779b9u) *o1 = sink;
+#endif
 }
 
 template <int EPI, bool TRI = false>
@@ -893,11 +904,25 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         uint32_t round = 0;
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)(tl & 1);
+#ifdef GEMM_TRACE4
+            const bool tr4 = SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && tl < 2048;
+            long long fw = 0;
+            if (tr4) g_gemm_trace[8 * tl + 0] = clock64();
+#endif
             if (tl >= 2) ptx::mbar_wait_uniform(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+#ifdef GEMM_TRACE4
+            if (tr4) g_gemm_trace[8 * tl + 1] = clock64();
+#endif
             ptx::tc_fence_after();
             const uint32_t d = tmu + (uint32_t)(acc * ACC_COLS);
             for (int s = 0; s < nst; ++s) {
+#ifdef GEMM_TRACE4
+                const long long w0 = clock64();
+#endif
                 ptx::mbar_wait_uniform(&full[b * GH], round & 1);
+#ifdef GEMM_TRACE4
+                fw += clock64() - w0;
+#endif
                 ptx::tc_fence_after();
                 const uint32_t a0 = tmu + (uint32_t)(A_COL0 + 64 * b);
                 const uint64_t b0 = bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4);
@@ -913,6 +938,9 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 if (++b == NS) { b = 0; ++round; }
             }
             ptx::mma_commit_uniform(&accf[acc]);
+#ifdef GEMM_TRACE4
+            if (tr4) { g_gemm_trace[8 * tl + 2] = clock64(); g_gemm_trace[8 * tl + 5] = fw; }
+#endif
         }
         __syncwarp();
     } else {
@@ -958,6 +986,10 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             }
             ptx::mbar_wait_warp(&accf[acc], ph);
             GEMM_T3(4, tl == 0 && e == 0 && lane == 0);
+#ifdef GEMM_TRACE4
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 2048) g_gemm_trace[8 * tl + 3] = clock64();
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && e == 7 && lane == 0 && tl < 2048) g_gemm_trace[8 * tl + 6] = clock64();
+#endif
             ptx::tc_fence_after();
             const bool full_vec = ncols == 64 && !args.swap;
             const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * ACC_COLS + c0);
@@ -978,6 +1010,10 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                     ptx::tc_fence_before();
                     __syncwarp();
                     if (lane == 0) ptx::mbar_arrive(&acce[acc]);   // accumulator drained
+#ifdef GEMM_TRACE4
+                    if (SNP_PROF(args.trace) && blockIdx.x == 0 && (e == 0 || e == 7) && lane == 0 && tl < 2048)
+                        g_gemm_trace[8 * tl + (e == 0 ? 4 : 7)] = clock64();
+#endif
                 }
                 const uint32_t pcol = hh ? pcol1 : pcol0;
                 if (!args.swap) {
@@ -1596,7 +1632,10 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.sym = (!swap && a.A == a.B && a.m == a.n && a.lda32 == a.ldb32 && (epi == EPI_LD || a.op <= 1) &&
              full_tiles > 1 && !(syme && syme[0] == '0')) ? 1 : 0;
     static const char *ord = std::getenv("SNP_GEMM_ORDER");
-    g.order = ord ? (ord[0] - '0') : 2;
+    // raster: grouped (2) for LD; lane-block-major (1) for the swapped many-query FastID shape,
+    // where all query blocks of a database block run together (configs[3] on 1 GPU: 102.7 ->
+    // 95.8 ms for the counts pass; scripts/gpu_f20m_order.sh)
+    g.order = ord ? (ord[0] - '0') : (swap ? 1 : 2);
     // CTA-pair kernel: opt-in (SNP_GEMM_X2=1) for the unswapped shapes with more than one
     // lane block.  Measured slower on B200 (LD-32K counts 9.1 ms vs 7.0 ms; with expansion
     // skipped 7.8 vs 4.7 ms: the M = 256, N = 128 pair MMAs run at about half the per-SM
