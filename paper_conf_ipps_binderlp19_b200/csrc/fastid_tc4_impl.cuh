@@ -422,8 +422,12 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 #endif
 #endif
             const uint32_t tbase = tmem + ((uint32_t)(qa * 32) << 16) + (uint32_t)(C::A_COL0 + ACOLS * b);
+            // the last stage of a short profile: only the 256-bit groups that hold bits < nbits
+            // are expanded (the MMA issues only the K-steps that cover them)
+            const int hmax = (int)((nbits - w0 * 32 + 255) / 256) < KW / 8 ? (int)((nbits - w0 * 32 + 255) / 256) : KW / 8;
 #pragma unroll
             for (int h = 0; h < KW / 8; ++h) {
+                if (NHALF == 1 && h >= hmax) break;
                 uint32_t v[32];
 #pragma unroll
                 for (int i = 0; i < 8; ++i)
@@ -474,6 +478,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         // tmem was read from shared memory (a per-thread value to ptxas); a warp reduction
         // lands it in a uniform register so everything derived from it stays uniform.
         constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
+        const int kmax_last = (int)((nbits - (int64_t)(nst - 1) * KBITS + 63) / 64);   // 1 .. KBITS / 64
         const uint32_t tmu = __reduce_or_sync(0xffffffffu, tmem);
         const uint32_t sfa = tmu + C::SF_COL, sfb = tmu + C::SF_COL + 16;
         const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(qsm), BN * 16, 128);
@@ -513,12 +518,16 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 if (SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && itm < 1024) g_fastid_trace[8 * itm + 5] = clock64();
 #endif
                 const uint32_t a0 = tmu + (uint32_t)(C::A_COL0 + ACOLS * b);
+                // K-steps of this stage that hold bits < nbits (the rest would multiply zeros:
+                // a 128-SNP profile issues 2 MMAs per tile instead of KBITS / 64)
+                const int kmax = s == nst - 1 ? kmax_last : KBITS / 64;
 #pragma unroll
                 for (int k = 0; k < KBITS / 64; ++k) {
                     if (NHALF == 2 && k == KBITS / 128) {   // second half of the stage
                         ptx::mbar_wait_uniform(&full[b * NHALF + 1], bround & 1);
                         ptx::tc_fence_after();
                     }
+                    if (NHALF == 1 && k >= kmax) break;
                     ptx::mma_mxf4_ts(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa,
                                      sfb);
                 }

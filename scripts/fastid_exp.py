@@ -26,5 +26,6 @@ res["1op counts+best"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor",), 
 res["1op counts"] = t(lambda: snp.snp_fastid(Q, D, nbits, "xor", out=outs[0]))
 res["1op counts popD"] = t(lambda: snp.snp_fastid(Q, D, nbits, "xor", out=outs[0], popD=pd))
 res["1op best only"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor",), counts=False, best=True))
+res["2ops counts only popD"] = t(lambda: snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=outs, best=False, popD=pd))
 rd = nd * w * 8
 print(json.dumps({k: {"us": 1e3 * v, "GBps_read_only": rd / v / 1e6} for k, v in res.items()}), flush=True)
