@@ -223,6 +223,29 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
                              uint32_t *const *best_count, int64_t *const *best_index,
                              int64_t index_base, void *ws, size_t ws_bytes, void *stream);
 
+/* f1, threshold form — every (query, database row) pair with count <= tau for op (the
+ * forensic decision of P:L58 "no set bits in the result signifies a positive match", with a
+ * tolerance: tau = 0 lists exact matches; P:L62 larger counts are less likely).
+ *   matches:     device array of `capacity` snp_match (16-byte aligned); the first `capacity`
+ *                matches found are stored, in UNSPECIFIED order (the set is exact).
+ *   match_count: device uint64 (8-byte aligned), set to the TOTAL number of matches (it may
+ *                exceed capacity: the caller can re-run with a larger list).
+ *   index:       index_base + database row.
+ * The database is processed in row chunks through workspace counts
+ * (snp_fastid_threshold_workspace_bytes), each chunk by snp_fastid's kernels and one
+ * compaction pass.  nq <= 65535; SNP_E_NULL for a NULL match_count (or matches with
+ * capacity > 0). */
+typedef struct {
+    uint32_t query;   /* query row                          */
+    uint32_t count;   /* popc(Q_query op D_row) <= tau       */
+    int64_t index;    /* index_base + database row           */
+} snp_match;
+size_t snp_fastid_threshold_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op);
+snp_status snp_fastid_threshold(const uint64_t *Q, int64_t nq, int64_t ldq, const uint64_t *D, int64_t nd,
+                                int64_t ldd, const uint32_t *popD, int64_t nbits, int op, uint32_t tau,
+                                int64_t index_base, snp_match *matches, int64_t capacity, uint64_t *match_count,
+                                void *ws, size_t ws_bytes, void *stream);
+
 /* e — multi-GPU row partition (host only, no device access): rows [0, rows)
  * split into `world` contiguous ranges bounds[r] .. bounds[r+1] (bounds is a
  * HOST array of world+1 int64), each boundary a multiple of `align` (except

@@ -21,7 +21,8 @@ __all__ = [
     "SnpError", "OPS", "VARIANTS", "snp_words", "snp_ld_workspace_bytes",
     "snp_fastid_workspace_bytes", "snp_pack", "snp_pack_popc", "snp_row_popc", "snp_ld_counts",
     "snp_ld_r2", "snp_fastid", "snp_fastid_best", "snp_fastid_search",
-    "snp_fastid_search_workspace_bytes", "snp_shard_plan", "snp_shard_plan_sym", "snp_sym_tiles",
+    "snp_fastid_search_workspace_bytes", "snp_fastid_threshold", "snp_fastid_threshold_workspace_bytes",
+    "snp_shard_plan", "snp_shard_plan_sym", "snp_sym_tiles",
     "snp_ld_sym_workspace_bytes", "snp_ld_sym", "snp_sym_unpack", "snp_set_variant",
     "snp_last_variant", "snp_last_kernel", "snp_launch_count", "status_string",
 ]
@@ -280,6 +281,36 @@ def snp_fastid_search(Q: torch.Tensor, D: torch.Tensor, nbits: int, ops=("xor", 
                                   int(index_base), _ptr(ws), 0 if ws is None else ws.numel(), _stream(stream)),
           "snp_fastid_search")
     return counts, best
+
+
+def snp_fastid_threshold_workspace_bytes(nq: int, nd: int, nbits: int, op="xor") -> int:
+    return int(lib().snp_fastid_threshold_workspace_bytes(int(nq), int(nd), int(nbits), _op(op)))
+
+
+def snp_fastid_threshold(Q: torch.Tensor, D: torch.Tensor, nbits: int, op="xor", tau: int = 0,
+                         capacity: int = 1 << 16, index_base: int = 0, popD=None, ws=None, stream=None):
+    """f1 threshold form: every (query, database row) with count <= tau.
+
+    Returns (query, count, index, total): int64 / uint32-in-int64 / int64 device tensors of the
+    stored matches (at most `capacity`, unspecified order) and the total number of matches
+    (host int; > capacity means the list was truncated)."""
+    _dev_tensor(Q, "Q", _WORD_DTYPES)
+    _dev_tensor(D, "D", _WORD_DTYPES)
+    _dev_tensor(popD, "popD", _U32)
+    opi = _op(op)
+    nq, nd = Q.shape[0], D.shape[0]
+    dev = Q.device
+    m = torch.empty((max(1, int(capacity)), 2), dtype=torch.int64, device=dev)   # 16-byte snp_match
+    total = torch.zeros(1, dtype=torch.int64, device=dev)
+    if ws is None:
+        ws = _workspace(snp_fastid_threshold_workspace_bytes(nq, nd, nbits, opi), dev)
+    check(lib().snp_fastid_threshold(_ptr(Q), nq, _ld(Q), _ptr(D), nd, _ld(D), _ptr(popD), int(nbits), opi,
+                                     int(tau), int(index_base), _ptr(m), int(capacity), _ptr(total), _ptr(ws),
+                                     0 if ws is None else ws.numel(), _stream(stream)), "snp_fastid_threshold")
+    n = int(total.item())
+    k = min(n, int(capacity))
+    w0 = m[:k, 0]
+    return w0 & 0xFFFFFFFF, (w0 >> 32) & 0xFFFFFFFF, m[:k, 1], n
 
 
 def snp_shard_plan(rows: int, world: int, align: int = 128) -> list[int]:

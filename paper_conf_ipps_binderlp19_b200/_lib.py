@@ -29,6 +29,9 @@ SIGNATURES = {
     "snp_fastid_search": (_int, [_p, _i64, _i64, _p, _i64, _i64, _p, _i64, _int, _p, _p, _i64, _p, _p, _i64,
                                  _p, _sz, _p]),
     "snp_shard_plan": (_int, [_i64, _int, _i64, _p]),
+    "snp_fastid_threshold_workspace_bytes": (_sz, [_i64, _i64, _i64, _int]),
+    "snp_fastid_threshold": (_int, [_p, _i64, _i64, _p, _i64, _i64, _p, _i64, _int, ctypes.c_uint32, _i64, _p, _i64,
+                                    _p, _p, _sz, _p]),
     "snp_shard_plan_sym": (_int, [_i64, _int, _p]),
     "snp_sym_tiles": (_i64, [_i64]),
     "snp_ld_sym_workspace_bytes": (_sz, [_i64, _i64]),

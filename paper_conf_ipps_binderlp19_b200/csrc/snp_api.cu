@@ -774,6 +774,51 @@ snp_status snp_shard_plan(int64_t rows, int world, int64_t align, int64_t *bound
     return SNP_OK;
 }
 
+size_t snp_fastid_threshold_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int op) {
+    if (nq <= 0 || nd <= 0 || nbits <= 0) return 0;
+    const int64_t ch = search_chunk_rows(nq, nd);
+    return align256((size_t)nq * ch * 4) + snp_fastid_workspace_bytes(nq, ch, nbits, op) + 256;
+}
+
+snp_status snp_fastid_threshold(const uint64_t *Q, int64_t nq, int64_t ldq, const uint64_t *D, int64_t nd,
+                                int64_t ldd, const uint32_t *popD, int64_t nbits, int op, uint32_t tau,
+                                int64_t index_base, snp_match *matches, int64_t capacity, uint64_t *match_count,
+                                void *ws, size_t ws_bytes, void *stream) {
+    snp_status st;
+    if (nq < 0 || nd < 0 || capacity < 0) return SNP_E_SHAPE;
+    if (op < SNP_OP_AND || op > SNP_OP_NOTAND) return SNP_E_OP;
+    if ((st = check_nbits(nbits)) != SNP_OK) return st;
+    if ((st = check_packed(Q, nq, ldq, nbits)) != SNP_OK) return st;
+    if ((st = check_packed(D, nd, ldd, nbits)) != SNP_OK) return st;
+    if (!match_count || (capacity > 0 && !matches)) return SNP_E_NULL;
+    if (((uintptr_t)match_count & 7u) || ((uintptr_t)matches & 15u)) return SNP_E_ALIGN;
+    if (nq > 65535) return SNP_E_RANGE;
+    if ((st = check_arch()) != SNP_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = cudaMemsetAsync(match_count, 0, sizeof(uint64_t), s);
+    if (e != cudaSuccess) return set_cuda_error(e);
+    if (nq == 0 || nd == 0) return SNP_OK;
+    const size_t need = snp_fastid_threshold_workspace_bytes(nq, nd, nbits, op);
+    if (ws_bytes < need || !ws) return SNP_E_WORKSPACE;
+    // the database in row chunks: counts of one chunk into workspace (snp_fastid's dispatch:
+    // the streaming, FastID or general kernel), then one compaction pass over the chunk
+    const int64_t ch = search_chunk_rows(nq, nd);
+    uint32_t *chunk = reinterpret_cast<uint32_t *>(ws);
+    char *ws2 = (char *)ws + align256((size_t)nq * ch * 4);
+    const size_t ws2_bytes = ws_bytes - align256((size_t)nq * ch * 4);
+    for (int64_t j0 = 0; j0 < nd; j0 += ch) {
+        const int64_t rows = nd - j0 < ch ? nd - j0 : ch;
+        if ((st = snp_fastid(Q, nq, ldq, nullptr, D + j0 * ldd, rows, ldd, popD ? popD + j0 : nullptr, nbits, op,
+                             chunk, ch, 0, ws2, ws2_bytes, stream)) != SNP_OK)
+            return st;
+        if ((e = launch_threshold_compact(chunk, nq, rows, ch, index_base + j0, tau,
+                                          reinterpret_cast<ThresholdMatch *>(matches), capacity,
+                                          reinterpret_cast<unsigned long long *>(match_count), s)) != cudaSuccess)
+            return set_cuda_error(e);
+    }
+    return SNP_OK;
+}
+
 snp_status snp_shard_plan_sym(int64_t m, int world, int64_t *tile_bounds) {
     if (world < 1 || m < 0) return SNP_E_RANGE;
     if (!tile_bounds) return SNP_E_NULL;

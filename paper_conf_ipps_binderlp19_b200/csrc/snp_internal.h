@@ -137,6 +137,16 @@ bool fastid_stream_supported(int64_t nq, int64_t nd, int64_t nbits);
 size_t fastid_stream_ws_bytes(int64_t nq, int nops);
 cudaError_t launch_fastid_stream(const SearchArgs &a, cudaStream_t s);
 
+// threshold.cu — f1 threshold form: (query, count, global index) of every count <= tau.
+struct ThresholdMatch {
+    uint32_t query;
+    uint32_t count;
+    int64_t index;
+};
+cudaError_t launch_threshold_compact(const uint32_t *counts, int64_t nq, int64_t rows, int64_t ldo, int64_t index0,
+                                     uint32_t tau, ThresholdMatch *out, int64_t capacity, unsigned long long *total,
+                                     cudaStream_t s);
+
 // best.cu building blocks for the chunked search path: keys (count << 32 | j) are
 // initialised to ~0, min-merged per count block (j offset by jbase), then finalised.
 cudaError_t launch_best_init(unsigned long long *keys, int64_t n, cudaStream_t s);

@@ -885,3 +885,28 @@ def test_search_kchunked_long_profiles(snp, nq, nbits, mode, monkeypatch):
             assert np.array_equal(u32(c[j]), ref), (op, mode)
         rb, ri = oracle.best(ref, 4)
         assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), (op, mode)
+
+
+@pytest.mark.parametrize("nq,nd,nbits,tau", [(3, 5000, 700, 0), (40, 3000, 1000, 400), (70, 2000, 4097, 1700),
+                                             (1, 1, 64, 64)])
+@pytest.mark.parametrize("op", ["xor", "andnot"])
+def test_fastid_threshold_matches(snp, nq, nd, nbits, tau, op, monkeypatch):
+    """f1 threshold form: the set of (query, row, count) with count <= tau equals the oracle's,
+    across database row chunks (small chunks forced), with index_base; truncation keeps the
+    total count."""
+    monkeypatch.setenv("SNP_SEARCH_CHUNK_ROWS", "768")
+    db = snpgen.fastid_db(86, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(86, nq, nd, nbits)
+    if nd > 10:
+        q[0] = db[nd - 5]
+    Q, D = pack_dev(snp, q, garbage_seed=8), pack_dev(snp, db, garbage_seed=9)
+    qi, cnt, idx, total = snp.snp_fastid_threshold(Q, D, nbits, op, tau=tau, capacity=nq * nd, index_base=10)
+    ref = oracle.counts(q, db, op)
+    rq, rd = np.nonzero(ref <= tau)
+    assert total == len(rq)
+    got = sorted(zip(qi.cpu().tolist(), (idx - 10).cpu().tolist(), cnt.cpu().tolist()))
+    want = sorted(zip(rq.tolist(), rd.tolist(), ref[rq, rd].tolist()))
+    assert got == want
+    if total > 3:
+        _, _, idx2, total2 = snp.snp_fastid_threshold(Q, D, nbits, op, tau=tau, capacity=3)
+        assert total2 == total and idx2.numel() == 3
