@@ -89,6 +89,12 @@ snp_status check_nbits(int64_t nbits) {
     return SNP_OK;
 }
 
+// Some tensor-core kernel serves the shape: the persistent kind::mxf4 kernels (any m, n below
+// 2^31 rows, nbits < 2^24) or the kind::i8 kernel (its grid bounds the smaller dimension).
+bool tc_any_supported(int64_t m, int64_t n, int64_t nbits) {
+    return fastid_tc4_supported(m, n, nbits) || gemm_tc4_supported(m, n, nbits) || tc_supported(m, n, nbits);
+}
+
 // Variant choice per shape (a7).  Measured dispatch: the tensor-core variant wins
 // whenever it supports the shape (>= 15x the POPC roof); the POPC
 // variant covers everything else and is kept as the forced/reference variant.
@@ -96,7 +102,7 @@ int choose_variant(int64_t m, int64_t n, int64_t nbits) {
     const int v = current_variant();
     if (v == SNP_VARIANT_POPC) return SNP_VARIANT_POPC;
     if (v == SNP_VARIANT_TC) return SNP_VARIANT_TC;
-    return tc_supported(m, n, nbits) ? SNP_VARIANT_TC : SNP_VARIANT_POPC;
+    return tc_any_supported(m, n, nbits) ? SNP_VARIANT_TC : SNP_VARIANT_POPC;
 }
 
 // a7: the CUDA-core streaming kernel serves the few-query FastID shapes (nq <= STREAM_NQ in
@@ -129,7 +135,7 @@ int tc_kernel_for(int64_t m, int64_t n, int64_t nbits, int epi) {
 snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes, cudaStream_t s) {
     cudaError_t e;
     if (variant == SNP_VARIANT_TC) {
-        if (!tc_supported(a.m, a.n, a.nbits)) return SNP_E_SHAPE;
+        if (!tc_any_supported(a.m, a.n, a.nbits)) return SNP_E_SHAPE;
         // kind::mxf4 (2x the int8 rate, half the expanded bytes) unless K is too long
         // for exact fp32 accumulation or SNP_TC_KIND=i8 asks for the int8 kernel.
         const int kern = tc_kernel_for(a.m, a.n, a.nbits, epi);
