@@ -224,14 +224,29 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     }
     const int64_t nbits = args.nbits;
     const int nst = args.nst;
-#ifndef FASTID_CONTIG_TILES
+#if defined(FASTID_TILE_GROUP)
+    // measurement variant: groups of FASTID_TILE_GROUP adjacent tiles per CTA, the CTAs sweeping
+    // the database together group by group
+    constexpr int64_t TG = FASTID_TILE_GROUP;
+    const int64_t ngroups = (args.ntiles + TG - 1) / TG;
+    const int64_t my_groups = ngroups > blockIdx.x ? (ngroups - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    int64_t my_tiles = my_groups * TG;
+    if (my_groups > 0) {   // the last group may be ragged
+        const int64_t lastg = blockIdx.x + (my_groups - 1) * gridDim.x;
+        const int64_t rem = args.ntiles - lastg * TG;
+        my_tiles -= TG - (rem < TG ? rem : TG);
+    }
+#define FASTID_TILE(tl) (((tl) / TG) * gridDim.x * TG + (int64_t)blockIdx.x * TG + (tl) % TG)
+#elif !defined(FASTID_CONTIG_TILES)
     // tile tl of this CTA is blockIdx.x + tl * gridDim.x (the CTAs sweep the database together)
     const int64_t my_tiles = args.ntiles > blockIdx.x ? (args.ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
     const int64_t tile0 = blockIdx.x, tstep = gridDim.x;
+#define FASTID_TILE(tl) (tile0 + (tl) * tstep)
 #else
     // measurement variant: each CTA takes one contiguous block of tiles
     const int64_t tile0 = args.ntiles * blockIdx.x / gridDim.x, tstep = 1;
     const int64_t my_tiles = args.ntiles * (blockIdx.x + 1) / gridDim.x - tile0;
+#define FASTID_TILE(tl) (tile0 + (tl) * tstep)
 #endif
     const int64_t total_it = my_tiles * nst;
     const int64_t full32 = nbits / 32;
@@ -321,7 +336,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
             int p = 0;
             uint32_t round = 0;   // how many times the ring has wrapped
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
-                const int64_t t = tile0 + tl * tstep;
+                const int64_t t = FASTID_TILE(tl);
                 const int32_t row0 = (int32_t)(t * BM);
                 for (int s = 0; s < nst; ++s) {
                     if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
@@ -556,7 +571,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         for (int64_t tl = 0; tl < my_tiles; ++tl) {
             const int acc = (int)((uint32_t)tl % NACC);
             const uint32_t ph = ((uint32_t)tl / NACC) & 1u;
-            const int64_t t = tile0 + tl * tstep;
+            const int64_t t = FASTID_TILE(tl);
             const bool pre = args.popDg != nullptr;
             const int64_t gd_l = t * BM + li;   // this lane's local database row
             uint32_t pd = 0;
