@@ -86,6 +86,39 @@ def ld_cases():
         check(f"many-query {op}", u32(counts[j]), oracle.counts(q, db, op))
 
 
+def round2_kernels():
+    # CUDA-core streaming FastID (nq <= 3 in AUTO, <= 4 forced), all ops + best, popD both ways
+    for nq, nd, nbits in [(1, 700, 700), (3, 520, 1000), (2, 300, 64)]:
+        db = snpgen.fastid_db(13, np.arange(nd), nbits)
+        q, _ = snpgen.fastid_queries(13, nq, nd, nbits)
+        D, Q = snp.snp_pack(dev(db)), snp.snp_pack(dev(q))
+        for pre in (None, snp.snp_row_popc(D, nbits)):
+            counts, best = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot", "and"), popD=pre, index_base=1)
+            for j, op in enumerate(("xor", "andnot", "and")):
+                check(f"stream {op} {nq}x{nd}x{nbits} k={snp.snp_last_kernel()}", u32(counts[j]), oracle.counts(q, db, op))
+    # packed-triangle self-LD (tensor TRI instantiation and CUDA-core), unpack
+    for variant in ("auto", "popc"):
+        snp.snp_set_variant(variant)
+        g = snpgen.ld_genotypes(14, np.arange(300), 777, structure=True)
+        A = snp.snp_pack(dev(g))
+        r2, dp, cnt = snp.snp_ld_sym(A, 777, r2=True, dprime=True, counts=True)
+        check(f"ld_sym {variant} k={snp.snp_last_kernel()}", u32(snp.snp_sym_unpack(cnt, 300)), oracle.ld(g, g)[2])
+        _, _, c2 = snp.snp_ld_sym(A, 777, 1, 5, r2=False, counts=True)
+        check(f"ld_sym range {variant}", u32(c2), u32(cnt[1:5]))
+    snp.snp_set_variant("auto")
+    # K-chunked long-profile search (<= 16 queries that do not fit the resident batch)
+    nq, nd, nbits = 6, 600, 20000
+    db = snpgen.fastid_db(15, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(15, nq, nd, nbits)
+    counts, _ = snp.snp_fastid_search(snp.snp_pack(dev(q)), snp.snp_pack(dev(db)), nbits, ("xor", "andnot"))
+    check("kchunk xor", u32(counts[0]), oracle.counts(q, db, "xor"))
+    # threshold list
+    qi, cnt, idx, total = snp.snp_fastid_threshold(snp.snp_pack(dev(q)), snp.snp_pack(dev(db)), nbits, "xor",
+                                                   tau=9000, capacity=nq * nd)
+    ref = oracle.counts(q, db, "xor")
+    check("threshold total", np.array([total]), np.array([int((ref <= 9000).sum())]))
+
+
 def small_kernels():
     g = snpgen.fastid_db(8, np.arange(333), 1000)
     P, pc = snp.snp_pack_popc(dev(g))
@@ -103,6 +136,7 @@ if __name__ == "__main__":
     small_kernels()
     if os.environ.get("SNP_TC_KIND") != "i8":
         fastid_cases()
+        round2_kernels()
     ld_cases()
     snp.snp_set_variant("popc")
     small_kernels()
