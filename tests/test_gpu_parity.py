@@ -910,3 +910,56 @@ def test_fastid_threshold_matches(snp, nq, nd, nbits, tau, op, monkeypatch):
     if total > 3:
         _, _, idx2, total2 = snp.snp_fastid_threshold(Q, D, nbits, op, tau=tau, capacity=3)
         assert total2 == total and idx2.numel() == 3
+
+
+def test_fuzz_round2_paths(snp):
+    """Seeded random shapes through the round-2 paths vs the oracle: the CUDA-core streaming
+    kernel (1-4 queries), K-chunked long profiles (<= 16 queries), packed-triangle tile ranges,
+    and threshold lists."""
+    from paper_conf_ipps_binderlp19_b200.multigpu import sym_tile_coords
+    rng = np.random.default_rng(2025)
+    for _ in range(4):
+        nq, nd, nbits = int(rng.integers(1, 5)), int(rng.integers(1, 3000)), int(rng.integers(1, 6000))
+        db = snpgen.fastid_db(97, np.arange(nd), nbits)
+        q, _ = snpgen.fastid_queries(97, nq, nd, nbits)
+        _variant(snp, "popc")
+        try:
+            counts, best = snp.snp_fastid_search(pack_dev(snp, q, garbage_seed=1), pack_dev(snp, db, garbage_seed=2),
+                                                 nbits, ("xor", "notand"), index_base=3)
+        finally:
+            _variant(snp, "auto")
+        for j, op in enumerate(("xor", "notand")):
+            ref = oracle.counts(q, db, op)
+            assert np.array_equal(u32(counts[j]), ref), (nq, nd, nbits, op)
+            rb, ri = oracle.best(ref, 3)
+            assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri)
+    for _ in range(3):
+        nq, nd, nbits = int(rng.integers(2, 17)), int(rng.integers(200, 1500)), int(rng.integers(14000, 40000))
+        db = snpgen.fastid_db(98, np.arange(nd), nbits)
+        q, _ = snpgen.fastid_queries(98, nq, nd, nbits)
+        counts, _ = snp.snp_fastid_search(pack_dev(snp, q, garbage_seed=3), pack_dev(snp, db, garbage_seed=4), nbits,
+                                          ("andnot",))
+        assert np.array_equal(u32(counts[0]), oracle.counts(q, db, "andnot")), (nq, nd, nbits)
+    for _ in range(3):
+        m, nbits = int(rng.integers(1, 700)), int(rng.integers(1, 3000))
+        g = snpgen.ld_genotypes(99, np.arange(m), nbits, structure=True)
+        A = pack_dev(snp, g, garbage_seed=5)
+        T = snp.snp_sym_tiles(m)
+        lo = int(rng.integers(0, T))
+        hi = int(rng.integers(lo + 1, T + 1))
+        r2, _, cnt = snp.snp_ld_sym(A, nbits, lo, hi, counts=True)
+        r2_ref, _, n_ref = oracle.ld(g, g)
+        for u, t in enumerate(range(lo, hi)):
+            I, J = sym_tile_coords(m, t)
+            rs, cs = slice(128 * I, min(m, 128 * I + 128)), slice(128 * J, min(m, 128 * J + 128))
+            assert np.array_equal(u32(cnt[u])[:rs.stop - rs.start, :cs.stop - cs.start], n_ref[rs, cs]), (m, nbits, t)
+            check_r2(r2[u].cpu().numpy()[:rs.stop - rs.start, :cs.stop - cs.start], r2_ref[rs, cs])
+    nq, nd, nbits = 9, 2500, 333
+    db = snpgen.fastid_db(100, np.arange(nd), nbits)
+    q, _ = snpgen.fastid_queries(100, nq, nd, nbits)
+    qi, cnt, idx, total = snp.snp_fastid_threshold(pack_dev(snp, q), pack_dev(snp, db), nbits, "xor", tau=150,
+                                                   capacity=nq * nd)
+    ref = oracle.counts(q, db, "xor")
+    rq, rd = np.nonzero(ref <= 150)
+    assert total == len(rq)
+    assert sorted(zip(qi.cpu().tolist(), idx.cpu().tolist())) == sorted(zip(rq.tolist(), rd.tolist()))
