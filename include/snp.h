@@ -262,7 +262,13 @@ snp_status snp_shard_plan(int64_t rows, int world, int64_t align, int64_t *bound
 snp_status snp_shard_plan_sym(int64_t m, int world, int64_t *tile_bounds);
 
 /* Variant override (SNP_VARIANT_AUTO restores the dispatch table).  The
- * environment variable SNP_FORCE_VARIANT=popc|tc sets the initial value. */
+ * environment variable SNP_FORCE_VARIANT=popc|tc sets the initial value.
+ * Other environment variables only steer the kernel CHOICE for A/B measurements (never the
+ * results): SNP_FASTID_STREAM=0 (no CUDA-core streaming kernel), SNP_FASTID_KBITS=512|1024
+ * (FastID tensor-kernel stage size), SNP_SEARCH_KCHUNK=0 / SNP_SEARCH_SLICES=0 (no K-chunked
+ * or query-sliced searches), SNP_FASTID_KERNEL=0, SNP_TC_KIND=i8, SNP_GEMM_SYM=0,
+ * SNP_GEMM_ORDER=0|1|2, SNP_GEMM_X2=1; SNP_SEARCH_CHUNK_ROWS sets the workspace row-chunk size
+ * (tests).  Each is covered by the parity tests. */
 snp_status snp_set_variant(int variant);
 /* Variant used by the most recent successful compute call on this thread. */
 int snp_last_variant(void);
