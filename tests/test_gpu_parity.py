@@ -963,3 +963,34 @@ def test_fuzz_round2_paths(snp):
     rq, rd = np.nonzero(ref <= 150)
     assert total == len(rq)
     assert sorted(zip(qi.cpu().tolist(), idx.cpu().tolist())) == sorted(zip(rq.tolist(), rd.tolist()))
+
+
+def test_cfg2_fastid_1m_full_oracle(snp):
+    """configs[1] in full (SURVEY §8d "cfg 1 and 2: full oracle"): every one of the 2 x 64 x 1M
+    XOR / ANDNOT counts of the bench's search call (database popcounts given, the fused FastID
+    kernel) equals the bit-by-bit CPU oracle, database regenerated on the host in row chunks
+    from the same seeded generator; best matches equal the oracle's argmin over all rows."""
+    nq, nd, nbits, seed = 64, 1_000_000, 4096, 1002
+    D = _gen_dev_fastid(seed, nd, nbits)
+    q, _ = snpgen.fastid_queries(seed, nq, nd, nbits)
+    Q = snp.snp_pack(to_dev(q))
+    counts, best = snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), popD=snp.snp_row_popc(D, nbits))
+    assert snp.snp_last_kernel() == "fastid_mxf4"
+    got = [c.cpu().numpy().view(np.uint32) for c in counts]
+    del counts, D
+    torch.cuda.empty_cache()
+    ref_best = [np.full(nq, 0xFFFFFFFF, dtype=np.int64), np.zeros(nq, dtype=np.int64)], \
+               [np.full(nq, 0xFFFFFFFF, dtype=np.int64), np.zeros(nq, dtype=np.int64)]
+    step = 125_000
+    for r0 in range(0, nd, step):
+        db = snpgen.fastid_db(seed, np.arange(r0, min(nd, r0 + step)), nbits)
+        for j, op in enumerate(("xor", "andnot")):
+            ref = oracle.counts(q, db, op)
+            assert np.array_equal(got[j][:, r0:r0 + ref.shape[1]], ref), (op, r0)
+            m, a = ref.min(1).astype(np.int64), ref.argmin(1) + r0
+            better = m < ref_best[j][0]
+            ref_best[j][1][better] = a[better]
+            ref_best[j][0][better] = m[better]
+    for j in range(2):
+        assert np.array_equal(best[j][0].cpu().numpy().astype(np.int64), ref_best[j][0])
+        assert np.array_equal(best[j][1].cpu().numpy(), ref_best[j][1])
