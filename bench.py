@@ -517,9 +517,10 @@ def setup_ld_tri(wl, rank, world, dev):
     full_host = ((torch.empty(r2.shape, dtype=torch.float32).pin_memory(),
                   torch.empty(cnt.shape, dtype=torch.uint32).pin_memory()) if out_bytes <= (1 << 30) else None)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    ldws = torch.empty(max(1, snp.snp_ld_sym_workspace_bytes(m, nbits)), dtype=torch.uint8, device=dev)
 
     def compute():
-        snp.snp_ld_sym(B, nbits, lo, hi, popA=pop, r2=r2, counts=cnt)          # a3 + a5 (f3 tiles)
+        snp.snp_ld_sym(B, nbits, lo, hi, popA=pop, r2=r2, counts=cnt, ws=ldws)  # a3 + a5 (f3 tiles)
 
     # end to end at N = 1 (the paper's mode): the matrix packed on the host (as the
     # paper's CPU packer leaves it) in pinned memory, streamed in row blocks overlapped with
@@ -766,13 +767,13 @@ def run_ours(args):
         # executed work is the rank's tiles (kernel_cmp); the effective rate counts the
         # m * m * nbits comparisons of the full symmetric matrix those tiles represent
         kcmp_eff = wlrun["cmp_all"] // world
-    elif kernel == "tc_mxf4_sym":
+    elif kernel in ("tc_mxf4_sym", "tc_mxf4_sym_pair"):
         # f3 symmetric self-LD executes only the upper-triangle 128 x 128 tiles (SURVEY §8d:
         # roofline on the executed work, M*N*nbits reported as the effective rate)
         T = -(-wl["m"] // 128)
         kcmp = T * (T + 1) // 2 * 128 * 128 * wl["nbits"]
     tops = 2 * kcmp / (kern_ms / 1e3) / 1e12
-    if kernel in ("tc_mxf4", "tc_mxf4_sym", "fastid_mxf4"):
+    if kernel in ("tc_mxf4", "tc_mxf4_sym", "tc_mxf4_sym_pair", "tc_mxf4_pair", "fastid_mxf4"):
         roof = {"bound": "tensor", "achieved": tops, "peak": peaks["f4_tops"], "unit": "TOPS",
                 "peak_src": f"fp4 dense = 4 x bf16 burst ({peaks['src']} MEASURED_PEAKS.json)"}
     elif kernel == "tc_i8":

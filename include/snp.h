@@ -282,8 +282,11 @@ typedef enum {
     SNP_KERNEL_FASTID_MXF4 = 4, /* kind::mxf4, resident queries, TMA-streamed DB   */
     SNP_KERNEL_TC_MXF4_SYM = 5, /* kind::mxf4 self-LD, upper-triangle tiles + mirror (f3):
                                    executes about half of the M*N*nbits comparisons */
-    SNP_KERNEL_POPC_STREAM = 6  /* CUDA-core FastID for nq <= 4: TMA-streamed database,
+    SNP_KERNEL_POPC_STREAM = 6, /* CUDA-core FastID for nq <= 4: TMA-streamed database,
                                    LOP3 + POPC, all ops and best matches in one pass   */
+    SNP_KERNEL_TC_MXF4_SYM_PAIR = 7, /* the whole f3 triangle on CTA pairs (tcgen05
+                                   cta_group::2, M = 256 pair tiles; snp_ld_sym)       */
+    SNP_KERNEL_TC_MXF4_PAIR = 8 /* kind::mxf4 on CTA pairs, general layout (opt-in)    */
 } snp_kernel;
 int snp_last_kernel(void);
 

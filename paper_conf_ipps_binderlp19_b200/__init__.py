@@ -396,7 +396,8 @@ def snp_launch_count() -> int:
     return int(lib().snp_launch_count())
 
 
-KERNELS = {0: "none", 1: "popc", 2: "tc_i8", 3: "tc_mxf4", 4: "fastid_mxf4", 5: "tc_mxf4_sym", 6: "popc_stream"}
+KERNELS = {0: "none", 1: "popc", 2: "tc_i8", 3: "tc_mxf4", 4: "fastid_mxf4", 5: "tc_mxf4_sym", 6: "popc_stream",
+           7: "tc_mxf4_sym_pair", 8: "tc_mxf4_pair"}
 
 
 def snp_last_kernel() -> str:

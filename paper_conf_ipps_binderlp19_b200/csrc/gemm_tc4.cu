@@ -25,6 +25,7 @@
 #include "e2m1.cuh"
 
 #include <cuda.h>
+#include <cstdio>
 #include <cstdlib>
 
 // Output stores: evict-first streaming stores (st.global.cs) by default — an LD output is
@@ -63,7 +64,10 @@ namespace {
 constexpr int BM = 128, BN = 128;
 constexpr int KBITS = 512;
 constexpr int KW = KBITS / 32;                 // 16 packed words per row per stage
-constexpr int NS = 3;                          // expanded slots (TMEM A stage + smem B stage)
+#ifndef GEMM_NS
+#define GEMM_NS 3
+#endif
+constexpr int NS = GEMM_NS;                    // expanded slots (TMEM A stage + smem B stage)
 #ifndef GEMM_NP
 #define GEMM_NP 6
 #endif
@@ -631,7 +635,7 @@ __device__ __forceinline__ void epi_swapped_counts(const GArgs &args, uint32_t (
 #endif
 }
 
-template <int EPI, bool TRI = false>
+template <int EPI, bool TRI = false, bool BPRE = false>
 __global__ void __launch_bounds__(NTHREADS, 1)
 gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
                 const GArgs args) {
@@ -714,10 +718,11 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
     if (tid == 0) {
         for (int i = 0; i < NP; ++i) {
             ptx::mbar_init(&pfull[i], 1);
-            ptx::mbar_init(&pempty[i], 8);
+            ptx::mbar_init(&pempty[i], BPRE ? 4 : 8);   // BPRE: only the A warps read the ring
         }
         for (int i = 0; i < NS; ++i) {
-            for (int h = 0; h < GH; ++h) ptx::mbar_init(&full[i * GH + h], 8);
+            // BPRE: the 4 A warps + the TMA producer's expect_tx for the pre-expanded B tile
+            for (int h = 0; h < GH; ++h) ptx::mbar_init(&full[i * GH + h], BPRE ? 5 : 8);
             ptx::mbar_init(&empty[i], 1);
         }
         for (int i = 0; i < 2; ++i) {
@@ -758,20 +763,38 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         if (lane == 0) {
             int p = 0;
             uint32_t round = 0;
+            int bs = 0;           // BPRE: B slot of the stage and how often it was used
+            uint32_t buse = 0;
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
                 const int64_t t = blockIdx.x + tl * gridDim.x;
                 const uint32_t t32 = (uint32_t)t;
                 uint32_t lbt, cbt;
-                if (TRI) tri_decode(args.nlb, args.tlo + t, lbt, cbt);
+                if (BPRE) decode_sym(t32, lbt, cbt);   // grouped triangle raster (B blocks reused from L2)
+                else if (TRI) tri_decode(args.nlb, args.tlo + t, lbt, cbt);
                 else if (args.sym) decode_sym(t32, lbt, cbt);
                 else { lbt = tile_lb(t32); cbt = tile_cb(t32); }
                 const int32_t rl = (int32_t)(lbt * BM), rc = (int32_t)(cbt * BN);
                 for (int s = 0; s < nst; ++s) {
                     if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);   // lane 0 only
-                    ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
+#ifdef GEMM_DEBUG_SKIP
+                    const bool no_b = BPRE || SNP_PROF(args.debug_skip == 3);
+#else
+                    constexpr bool no_b = BPRE;
+#endif
+                    ptx::mbar_arrive_expect_tx(&pfull[p], no_b ? BM * PROW : PSLOT);
                     ptx::tma_load_2d(ring + p * PSLOT, &tmL, &pfull[p], s * KW, rl);
-                    ptx::tma_load_2d(ring + p * PSLOT + BM * PROW, &tmC, &pfull[p], s * KW, rc);
+                    if (!no_b) ptx::tma_load_2d(ring + p * PSLOT + BM * PROW, &tmC, &pfull[p], s * KW, rc);
                     if (++p == NP) { p = 0; ++round; }
+                    if (BPRE) {
+                        // the stage's B operand arrives pre-expanded (128-byte rows, 128B swizzle)
+                        // straight into its MMA slot once the MMA has released that slot
+                        if (buse > 0) ptx::mbar_wait(&empty[bs], (buse - 1) & 1);
+                        ptx::mbar_arrive_expect_tx(&full[bs * GH], BSLOT);
+                        uint8_t *dst = bexp + (size_t)bs * BSLOT;
+                        ptx::tma_load_2d(dst, &tmC, &full[bs * GH], s * (KW * 4), rc);
+                        ptx::tma_load_2d(dst + BSLOT / 2, &tmC, &full[bs * GH], s * (KW * 4) + KW * 2, rc);
+                        if (++bs == NS) { bs = 0; ++buse; }
+                    }
                 }
             }
         }
@@ -786,6 +809,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         const int row = q * 32 + lane;
         const int sw = (row >> 1) & 3;                  // TMA 64B swizzle of a 64-byte row
         const uint32_t tAq = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)A_COL0;
+        const int64_t my_total_it = (BPRE && !is_a) ? 0 : total_it;   // BPRE: B arrives expanded
         int64_t tl = g / nst;
         int s = g % nst;
         int slot = g % NS;
@@ -793,7 +817,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         static_assert(NP % G == 0, "each packed slot belongs to one expander group");
         int pk = g;                                     // packed slot (group g: g, g + G, ...)
         uint32_t pround = 0;
-        for (int64_t it = g; it < total_it; it += G) {
+        for (int64_t it = g; it < my_total_it; it += G) {
 #ifdef GEMM_TRACE
             const bool tr = SNP_PROF(args.trace) && blockIdx.x == 0 && r8 == 0 && lane == 0 && it < 2048;
 #endif
@@ -810,7 +834,8 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             if (tr) g_gemm_trace[8 * it + 1] = clock64();
 #endif
 #ifdef GEMM_DEBUG_SKIP
-            if (SNP_PROF(args.debug_skip)) {
+            // debug_skip 1: every expander skips; 2: only the A warps on the MMA warp's sub-partition
+            if (SNP_PROF(args.debug_skip == 1 || (args.debug_skip == 2 && is_a && q == (MMA_WARP & 3)))) {
                 __syncwarp();
                 if (lane == 0) {
                     ptx::mbar_arrive(&pempty[pk]);
@@ -827,6 +852,14 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
 #endif
             const uint8_t *src = ring + pk * PSLOT + (is_a ? 0 : BM * PROW) + row * PROW;
             uint32_t w[KW];
+#ifdef GEMM_DEBUG_SKIP
+            // debug_skip 3: the B operand's packed words are not loaded (nor read): the cost of
+            // the B half of the packed ring in shared memory (results invalid)
+            if (SNP_PROF(args.debug_skip == 3 && !is_a)) {
+#pragma unroll
+                for (int i = 0; i < KW; ++i) w[i] = (uint32_t)(lane * 0x9E3779B9u + i + s);
+            } else
+#endif
 #pragma unroll
             for (int c = 0; c < 4; ++c) {
                 const uint4 x = *reinterpret_cast<const uint4 *>(src + ((c ^ sw) << 4));
@@ -898,7 +931,8 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
         constexpr uint32_t IDESC = idesc_mxf4(BM, BN);
         const uint32_t tmu = __reduce_or_sync(0xffffffffu, tmem);
         const uint32_t sfa = tmu + SF_COL, sfb = tmu + SF_COL + 16;
-        const uint64_t bdesc0 = ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(bexp), BN * 16, 128);
+        const uint64_t bdesc0 = BPRE ? ptx::smem_desc_kmajor_sw128(ptx::smem_u32(bexp))
+                                     : ptx::smem_desc_kmajor_noswizzle(ptx::smem_u32(bexp), BN * 16, 128);
         constexpr uint32_t BSTEP = (2 * BN * 16) >> 4;
         int b = 0;
         uint32_t round = 0;
@@ -932,7 +966,11 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                         ptx::mbar_wait_uniform(&full[b * GH + 1], round & 1);
                         ptx::tc_fence_after();
                     }
-                    ptx::mma_mxf4_ts(d, a0 + 8 * k, b0 + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                    // BPRE: K-step k is bytes [32 (k % 4), +32) of the 128-byte rows of half k / 4
+                    // (16 KB each; the descriptor's start address moves inside the swizzle atom)
+                    const uint64_t bk = BPRE ? b0 + (uint64_t)((((k >> 2) * (BSLOT / 2)) + (k & 3) * 32) >> 4)
+                                             : b0 + (uint64_t)(k * BSTEP);
+                    ptx::mma_mxf4_ts(d, a0 + 8 * k, bk, IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
                 }
                 ptx::mma_commit_uniform(&empty[b]);
                 if (++b == NS) { b = 0; ++round; }
@@ -961,9 +999,13 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             const int64_t t = blockIdx.x + tl * gridDim.x;
             const uint32_t t32 = (uint32_t)t;
             uint32_t lbt, cbt;
-            if (TRI) tri_decode(args.nlb, args.tlo + t, lbt, cbt);
+            if (BPRE) decode_sym(t32, lbt, cbt);
+            else if (TRI) tri_decode(args.nlb, args.tlo + t, lbt, cbt);
             else if (args.sym) decode_sym(t32, lbt, cbt);
             else { lbt = tile_lb(t32); cbt = tile_cb(t32); }
+            // BPRE processes the whole triangle in the grouped raster; the tile's packed-triangle
+            // storage slot is its row-major triangle index
+            const int64_t tst = BPRE ? tri_start(args.nlb, lbt) + (int64_t)(cbt - lbt) : t;
             const bool mirror = !TRI && args.sym && lbt != cbt;   // f3: also write the mirror block
             // packed triangle: the epilogue addresses the tile as rows t * 128 .. t * 128 + 127
             // of a [ntri * 128][128] matrix (args.nl / nc / ldo are those virtual sizes), so
@@ -973,7 +1015,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
             const int64_t nlr = TRI ? args.mreal : args.nl, ncr = TRI ? args.mreal : args.nc;
             const int64_t gl = (int64_t)lbt * BM + li;
             const int64_t gc0 = (int64_t)cbt * BN + c0;
-            const int64_t erow0 = TRI ? t * BM + q * 32 : gl - lane;   // epilogue block origin
+            const int64_t erow0 = TRI ? tst * BM + q * 32 : gl - lane;   // epilogue block origin
             const int64_t ecol0 = TRI ? (int64_t)c0 : gc0;
             const bool rows_ok = gl < args.nl && gc0 < args.nc;
             const int ncols = gc0 < ncr ? (int)(ncr - gc0 < 64 ? ncr - gc0 : 64) : 0;
@@ -1133,7 +1175,7 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
 // pipe and the ALU were the binding resources of the 1-CTA kernel.
 // Cross-CTA protocol:
 //   full[s]   (leader)  12 arrivals: the 6 expander warps of the stage's group in BOTH CTAs,
-//                       remote arrive.release.cluster after their TMEM / shared writes;
+//                       remote mbarrier.arrive after their TMEM / shared writes;
 //   empty[s]  (both)    tcgen05.commit multicast from the leader's MMA thread;
 //   accf[a]   (both)    tcgen05.commit multicast at the end of a pair tile;
 //   acce[a]   (leader)  16 arrivals: 8 epilogue warps of each CTA after draining TMEM.
@@ -1187,7 +1229,11 @@ __device__ __forceinline__ void cluster_sync() {
 __device__ __forceinline__ void arrive_remote(uint64_t *bar, uint32_t rank) {
     uint32_t ra;
     asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(ptx::smem_u32(bar)), "r"(rank));
-    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
+    // default semantics (release, CTA scope), as for any producer signalling the pair's MMA: the
+    // data it publishes is this CTA's own shared memory / TMEM, already ordered for the tensor
+    // core by fence.proxy.async / tcgen05.fence::before_thread_sync.  A cluster-scope release
+    // here cost ~1,500 cycles per arrival (measured: scripts/trace_x2.py)
+    asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
 }
 __device__ __forceinline__ bool try_wait_cluster(uint64_t *bar, uint32_t parity) {
     uint32_t ok;
@@ -1237,7 +1283,24 @@ __device__ __forceinline__ void commit_both(uint64_t *bar) {
 }
 }  // namespace x2
 
-template <int EPI>
+// f3 on CTA pairs: pair tile u <-> (P, J), lane blocks 2P and 2P + 1 (one per CTA) x column
+// block J, J = 2P .. T - 1 in row-major order, start(P) = P (T + 1 - P).  The pair's lower
+// tile (2P + 1, 2P) and lane block T (odd T) are computed on zeros / below the diagonal and
+// not stored.
+__host__ __device__ __forceinline__ int64_t pair_start(int64_t T, int64_t P) { return P * (T + 1 - P); }
+__host__ __device__ __forceinline__ void pair_decode(int64_t T, int64_t u, uint32_t &P, uint32_t &J) {
+    const double b = (double)T + 1.0;
+    int64_t p = (int64_t)((b - sqrt(b * b - 4.0 * (double)u)) * 0.5);
+    const int64_t np = (T + 1) / 2;
+    if (p < 0) p = 0;
+    if (p > np - 1) p = np - 1;
+    while (p > 0 && pair_start(T, p) > u) --p;
+    while (p + 1 < np && pair_start(T, p + 1) <= u) ++p;
+    P = (uint32_t)p;
+    J = (uint32_t)(2 * p + (u - pair_start(T, p)));
+}
+
+template <int EPI, bool TRI = false>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(x2::NTHREADS, 1)
 gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmC,
                   const GArgs args) {
@@ -1267,7 +1330,8 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
     const int nst = args.nst;
     // pair tiles: nlb = lane blocks of 256 rows, ncb = column blocks of 128
     const uint32_t nlb32 = (uint32_t)args.nlb, ncb32 = (uint32_t)args.ncb;
-    const uint32_t ntiles = nlb32 * ncb32;
+    // TRI: nlb = T (128-row blocks of the m x m triangle), ntri = pair tiles
+    const uint32_t ntiles = TRI ? (uint32_t)args.ntri : nlb32 * ncb32;
     const uint32_t cid = cluster_id(), ncl = num_clusters();
     const int64_t my_tiles = ntiles > cid ? (int64_t)((ntiles - 1u - cid) / ncl + 1u) : 0;
     const int64_t total_it = my_tiles * nst;
@@ -1331,8 +1395,16 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
             uint32_t round = 0;
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
                 const uint32_t t32 = cid + (uint32_t)tl * ncl;
-                const int32_t rl = (int32_t)(tile_lb(t32) * (2 * BM) + rank * BM);
-                const int32_t rc = (int32_t)(tile_cb(t32) * BNP + rank * BNH);
+                int32_t rl, rc;
+                if (TRI) {
+                    uint32_t P, J;
+                    pair_decode(nlb32, t32, P, J);
+                    rl = (int32_t)((2 * P + rank) * BM);
+                    rc = (int32_t)(J * BNP + rank * BNH);
+                } else {
+                    rl = (int32_t)(tile_lb(t32) * (2 * BM) + rank * BM);
+                    rc = (int32_t)(tile_cb(t32) * BNP + rank * BNH);
+                }
                 for (int s = 0; s < nst; ++s) {
                     if (round > 0) ptx::mbar_wait(&pempty[p], (round - 1) & 1);
                     ptx::mbar_arrive_expect_tx(&pfull[p], PSLOT);
@@ -1360,12 +1432,28 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
         int pk = g;
         uint32_t pround = 0;
         for (int64_t it = g; it < total_it; it += G) {
+#ifdef GEMM_TRACE
+            // warp 0 (group 0, lane quarter 0) of both CTAs of cluster 0: loop start, empty
+            // seen, packed stage seen, arrivals done
+            const bool tr = SNP_PROF(args.trace) && blockIdx.x < 2 && warp == 0 && lane == 0 && it < 4096;
+            long long *tp = g_gemm_trace + 8 * (it >> 1) + 4 * blockIdx.x;
+            if (tr) tp[0] = clock64();
+#endif
             if (use > 0) ptx::mbar_wait_warp(&empty[slot], (use - 1) & 1);
+#ifdef GEMM_TRACE
+            if (tr) tp[1] = clock64();
+#endif
             ptx::mbar_wait_warp(&pfull[pk], pround & 1);
+#ifdef GEMM_TRACE
+            if (tr) tp[2] = clock64();
+#endif
 #ifdef GEMM_DEBUG_SKIP
             if (SNP_PROF(args.debug_skip)) {   // profiling experiment: tokens only (results invalid)
                 __syncwarp();
                 if (lane == 0) { ptx::mbar_arrive(&pempty[pk]); arrive_remote(&full[slot], 0); }
+#ifdef GEMM_TRACE
+                if (tr) tp[3] = clock64();
+#endif
                 s += G;
                 while (s >= nst) s -= nst;
                 slot += G;
@@ -1433,11 +1521,25 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
             uint32_t round = 0;
             for (int64_t tl = 0; tl < my_tiles; ++tl) {
                 const int acc = (int)(tl & 1);
+#ifdef GEMM_TRACE4
+                const bool tr4 = SNP_PROF(args.trace) && blockIdx.x == 0 && lane == 0 && tl < 2048;
+                long long fw = 0;
+                if (tr4) g_gemm_trace[8 * tl + 0] = clock64();
+#endif
                 if (tl >= 2) wait_cluster_uniform(&acce[acc], (uint32_t)(((tl >> 1) - 1) & 1));
+#ifdef GEMM_TRACE4
+                if (tr4) g_gemm_trace[8 * tl + 1] = clock64();
+#endif
                 ptx::tc_fence_after();
                 const uint32_t d = tmu + (uint32_t)(acc * ACC_COLS);
                 for (int s = 0; s < nst; ++s) {
+#ifdef GEMM_TRACE4
+                    const long long w0 = clock64();
+#endif
                     wait_cluster_uniform(&full[b], round & 1);
+#ifdef GEMM_TRACE4
+                    fw += clock64() - w0;
+#endif
                     ptx::tc_fence_after();
                     const uint32_t a0 = tmu + (uint32_t)(A_COL0 + 64 * b);
                     const uint64_t b0 = bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4);
@@ -1448,6 +1550,9 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
                     if (++b == NS) { b = 0; ++round; }
                 }
                 commit_both(&accf[acc]);
+#ifdef GEMM_TRACE4
+                if (tr4) { g_gemm_trace[8 * tl + 2] = clock64(); g_gemm_trace[8 * tl + 5] = fw; }
+#endif
             }
         }
         __syncwarp();
@@ -1466,16 +1571,32 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
             const int acc = (int)(tl & 1);
             const uint32_t ph = (uint32_t)((tl >> 1) & 1);
             const uint32_t t32 = cid + (uint32_t)tl * ncl;
-            const int64_t gl = (int64_t)tile_lb(t32) * (2 * BM) + rank * BM + li;
-            const int64_t gc0 = (int64_t)tile_cb(t32) * BNP + c0;
-            const int ncols = gc0 < args.nc ? (int)(args.nc - gc0 < 64 ? args.nc - gc0 : 64) : 0;
+            int64_t gl, gc0, erow0 = 0;
+            bool store = true;
+            if (TRI) {   // this CTA's tile (I, J) of the pair; virtual [ntri 128][128] output
+                uint32_t P, J;
+                pair_decode(nlb32, t32, P, J);
+                const uint32_t I = 2 * P + rank;
+                store = I <= J && I < nlb32;
+                gl = (int64_t)I * BM + li;
+                gc0 = (int64_t)J * BNP + c0;
+                erow0 = (store ? tri_start(nlb32, I) + (int64_t)(J - I) : 0) * BM + q * 32;
+            } else {
+                gl = (int64_t)tile_lb(t32) * (2 * BM) + rank * BM + li;
+                gc0 = (int64_t)tile_cb(t32) * BNP + c0;
+            }
+            const int64_t nlr = TRI ? args.mreal : args.nl, ncr = TRI ? args.mreal : args.nc;
+            const int ncols = gc0 < ncr ? (int)(ncr - gc0 < 64 ? ncr - gc0 : 64) : 0;
             uint32_t pl = 0, pcol0 = 0, pcol1 = 0;
             if (need_pop) {
-                if (gl < args.nl) pl = __ldg(args.popL + gl);
+                if (gl < nlr) pl = __ldg(args.popL + gl);
                 if (lane < ncols) pcol0 = __ldg(args.popC + gc0 + lane);
                 if (32 + lane < ncols) pcol1 = __ldg(args.popC + gc0 + 32 + lane);
             }
             ptx::mbar_wait_warp(&accf[acc], ph);
+#ifdef GEMM_TRACE4
+            if (SNP_PROF(args.trace) && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 2048) g_gemm_trace[8 * tl + 3] = clock64();
+#endif
             ptx::tc_fence_after();
             const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * ACC_COLS + c0);
             const float ia = EPI == EPI_LD ? inv_exact((int64_t)pl * (n - (int64_t)pl)) : 0.f;
@@ -1489,6 +1610,15 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
                     ptx::tc_fence_before();
                     __syncwarp();
                     if (lane == 0) arrive_remote(&acce[acc], 0);   // drained: the leader may reuse it
+#ifdef GEMM_TRACE4
+                    if (SNP_PROF(args.trace) && blockIdx.x == 0 && e == 0 && lane == 0 && tl < 2048) g_gemm_trace[8 * tl + 4] = clock64();
+#endif
+                }
+                if (TRI) {
+                    if (store)
+                        epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, erow0, (int64_t)c0 + 32 * hh, pl,
+                                            hh ? pcol1 : pcol0, ia, small_n, want_dp, false);
+                    continue;
                 }
                 epi_transposed<EPI>(args, v, trs + e * 32 * 32, lane, gl - lane, gc0 + 32 * hh, pl,
                                     hh ? pcol1 : pcol0, ia, small_n, want_dp, false);
@@ -1509,14 +1639,36 @@ bool make_map(CUtensorMap *tm, const uint32_t *base, int64_t rows, int64_t ld32,
     return make_map_u32_2d(tm, base, rows, ld32, KW, box_rows, CU_TENSOR_MAP_SWIZZLE_64B);
 }
 
-template <int EPI, bool TRI = false>
+// Pre-expanded column operand (BPRE): word w of row r -> the 16 bytes expandB(w) at
+// out[r * wrow + w], zeros for words past nbits (so the row pitch wrow * 16 bytes holds
+// whole 512-bit stages).  Coalesced 4-byte reads, 16-byte writes.
+__global__ void expand_b_kernel(const uint32_t *__restrict__ A, int64_t m, int64_t lda32, int64_t nbits,
+                                int64_t wrow, uint4 *__restrict__ out) {
+    const int64_t total = m * wrow;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = i / wrow, w = i - r * wrow;
+        const uint32_t msk = word_mask(w, nbits);
+        const uint32_t x = msk ? __ldg(A + r * lda32 + w) & msk : 0u;
+        uint4 o;
+        expandB(x, o.x, o.y, o.z, o.w);
+        out[i] = o;
+    }
+}
+
+template <int EPI, bool TRI = false, bool BPRE = false>
 cudaError_t launch_g(const GArgs &g, const uint32_t *L, int64_t ldl32, const uint32_t *Cn, int64_t ldc32,
                      cudaStream_t s) {
     CUtensorMap tmL, tmC;
     // packed-triangle launches keep virtual output sizes in g.nl / g.nc: the operands have m rows
     const int64_t rows_l = TRI ? g.mreal : g.nl, rows_c = TRI ? g.mreal : g.nc;
-    if (!make_map(&tmL, L, rows_l, ldl32) || !make_map(&tmC, Cn, rows_c, ldc32)) return cudaErrorInvalidValue;
-    auto kern = gemm_tc4_kernel<EPI, TRI>;
+    if (!make_map(&tmL, L, rows_l, ldl32)) return cudaErrorInvalidValue;
+    if (BPRE) {   // Cn = the expanded operand, ldc32 its row pitch in 32-bit words; 128-byte boxes
+        if (!make_map_u32_2d(&tmC, Cn, rows_c, ldc32, 32, BN, CU_TENSOR_MAP_SWIZZLE_128B))
+            return cudaErrorInvalidValue;
+    } else if (!make_map(&tmC, Cn, rows_c, ldc32)) {
+        return cudaErrorInvalidValue;
+    }
+    auto kern = gemm_tc4_kernel<EPI, TRI, BPRE>;
     if (cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)SMEM); e != cudaSuccess) return e;
     const int64_t ntiles = TRI ? g.ntri : g.sym ? g.nlb * (g.nlb + 1) / 2 : g.nlb * g.ncb;
     if (ntiles <= 0) return cudaSuccess;
@@ -1537,18 +1689,44 @@ cudaError_t launch_g(const GArgs &g, const uint32_t *L, int64_t ldl32, const uin
     return cudaGetLastError();
 }
 
-template <int EPI>
+template <int EPI, bool TRI = false>
 cudaError_t launch_g2(GArgs g, const uint32_t *L, int64_t ldl32, const uint32_t *Cn, int64_t ldc32, cudaStream_t s) {
     CUtensorMap tmL, tmC;
-    if (!make_map(&tmL, L, g.nl, ldl32, 128) || !make_map(&tmC, Cn, g.nc, ldc32, x2::BNH))
+    const int64_t rows_l = TRI ? g.mreal : g.nl, rows_c = TRI ? g.mreal : g.nc;
+    if (!make_map(&tmL, L, rows_l, ldl32, 128) || !make_map(&tmC, Cn, rows_c, ldc32, x2::BNH))
         return cudaErrorInvalidValue;
-    auto kern = gemm_tc4x2_kernel<EPI>;
+    auto kern = gemm_tc4x2_kernel<EPI, TRI>;
     if (cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)x2::SMEM); e != cudaSuccess)
         return e;
-    g.nlb = (g.nl + 2 * BM - 1) / (2 * BM);
-    g.ncb = (g.nc + x2::BNP - 1) / x2::BNP;
-    const int64_t npairs = g.nlb * g.ncb;
-    const int pairs = device_sms() / 2;
+    int64_t npairs;
+    if (TRI) {   // g.nlb = T; pair tiles over the whole triangle
+        npairs = pair_start(g.nlb, (g.nlb + 1) / 2);
+        g.ntri = npairs;
+    } else {
+        g.nlb = (g.nl + 2 * BM - 1) / (2 * BM);
+        g.ncb = (g.nc + x2::BNP - 1) / x2::BNP;
+        npairs = g.nlb * g.ncb;
+    }
+    // co-resident 2-CTA clusters: a GPC with an odd SM count leaves one SM unpaired, so
+    // SMs / 2 clusters would run a second wave of a few clusters (doubling the time)
+    int pairs = device_sms() / 2;
+    {
+        cudaLaunchConfig_t qc{};
+        qc.gridDim = dim3(2 * (unsigned)pairs);
+        qc.blockDim = dim3((unsigned)x2::NTHREADS);
+        qc.dynamicSmemBytes = x2::SMEM;
+        cudaLaunchAttribute ca[1];
+        ca[0].id = cudaLaunchAttributeClusterDimension;
+        ca[0].val.clusterDim.x = 2; ca[0].val.clusterDim.y = 1; ca[0].val.clusterDim.z = 1;
+        qc.attrs = ca;
+        qc.numAttrs = 1;
+        int nc = 0;
+        if (cudaOccupancyMaxActiveClusters(&nc, reinterpret_cast<const void *>(kern), &qc) == cudaSuccess && nc > 0 &&
+            nc < pairs)
+            pairs = nc;
+        static const bool report = std::getenv("SNP_X2_REPORT") != nullptr;
+        if (report) fprintf(stderr, "x2: %d co-resident clusters (SMs %d)\n", nc, device_sms());
+    }
     const int grid = 2 * (int)(npairs < pairs ? npairs : pairs);
     kern<<<grid, x2::NTHREADS, x2::SMEM, s>>>(tmL, tmC, g);
     count_launches(1);
@@ -1559,15 +1737,38 @@ cudaError_t launch_g2(GArgs g, const uint32_t *L, int64_t ldl32, const uint32_t 
 
 namespace {
 thread_local bool g_last_sym = false;
+thread_local bool g_last_pair = false;
 }
 bool gemm_tc4_last_sym() { return g_last_sym; }
+bool gemm_tc4_last_pair() { return g_last_pair; }
+
+size_t gemm_tc4_bpre_bytes(int64_t m, int64_t nbits) {
+    return (size_t)m * (size_t)((nbits + KBITS - 1) / KBITS) * KW * 16;
+}
 
 bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits) {
     return m >= 1 && n >= 1 && nbits >= 1 && nbits < (1LL << 24) && m < (1LL << 31) && n < (1LL << 31);
 }
 
+// SNP_GEMM_X2: "1" forces the CTA-pair kernel where it applies, "0" the 1-CTA kernel,
+// unset = the shape default
+static int x2_mode() {
+    static const int m = [] {
+        const char *e = std::getenv("SNP_GEMM_X2");
+        return e && e[0] == '1' ? 1 : e && e[0] == '0' ? 0 : -1;
+    }();
+    return m;
+}
+
 cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     GArgs g{};
+    g_last_pair = false;
+#ifdef SNP_PROFILING
+    static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
+    g.trace = trace ? 1 : 0;
+    static const char *skip = std::getenv("SNP_DEBUG_SKIP_EXPAND");
+    g.debug_skip = skip ? skip[0] - '0' : 0;
+#endif
     if (a.tri_n >= 0) {   // f3 packed triangle: self-LD only (A == B), no swap, no mirror
         if (a.m != a.n || a.A != a.B || a.lda32 != a.ldb32 || a.C2) return cudaErrorInvalidValue;
         g.popL = a.popA;
@@ -1591,6 +1792,29 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
         g.v4 = (((uintptr_t)a.r2 & 15u) == 0 && ((uintptr_t)a.C & 15u) == 0) ? 1 : 0;
         g.order = 2;
         g_last_sym = true;
+        const int64_t T = g.nlb;
+        const bool whole = a.tri_lo == 0 && a.tri_n == T * (T + 1) / 2 && a.tri_n < (1LL << 31);
+        const int x2m = x2_mode();
+        if (whole && !a.bpre && (x2m == 1 || (x2m < 0 && pair_start(T, (T + 1) / 2) >= device_sms()))) {
+            // whole triangle on CTA pairs (tcgen05 cta_group::2, M = 256 pair tiles): half of
+            // the B operand's expansion, shared-memory writes and MMA reads per SM (LD-32K
+            // 3.50 -> 2.95 ms).  Default from two waves of pair tiles up (LD-2K, one wave:
+            // equal kernel time, +1 us launch), partial ranges keep the 1-CTA kernel
+            g_last_pair = true;
+            return epi == EPI_LD ? launch_g2<EPI_LD, true>(g, a.A, a.lda32, a.A, a.lda32, s)
+                                 : launch_g2<EPI_COUNTS, true>(g, a.A, a.lda32, a.A, a.lda32, s);
+        }
+        if (a.bpre && whole) {
+            // whole triangle with the pre-expanded column operand (a.bpre: bpre_bytes(m, nbits))
+            const int64_t wrow = (int64_t)g.nst * KW;
+            const int64_t total = a.m * wrow;
+            const int blocks = (int)std::min<int64_t>((total + 255) / 256, (int64_t)device_sms() * 16);
+            expand_b_kernel<<<blocks, 256, 0, s>>>(a.A, a.m, a.lda32, a.nbits, wrow, reinterpret_cast<uint4 *>(a.bpre));
+            count_launches(1);
+            if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) return e;
+            return epi == EPI_LD ? launch_g<EPI_LD, true, true>(g, a.A, a.lda32, a.bpre, wrow * 4, s)
+                                 : launch_g<EPI_COUNTS, true, true>(g, a.A, a.lda32, a.bpre, wrow * 4, s);
+        }
         return epi == EPI_LD ? launch_g<EPI_LD, true>(g, a.A, a.lda32, a.A, a.lda32, s)
                              : launch_g<EPI_COUNTS, true>(g, a.A, a.lda32, a.A, a.lda32, s);
     }
@@ -1615,12 +1839,6 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     g.nlb = (g.nl + BM - 1) / BM;
     g.ncb = (g.nc + BN - 1) / BN;
     g.nst = (int)((a.nbits + KBITS - 1) / KBITS);
-#ifdef SNP_PROFILING
-    static const bool trace = std::getenv("SNP_TRACE") && std::getenv("SNP_TRACE")[0] == '1';
-    g.trace = trace ? 1 : 0;
-    static const bool skip = std::getenv("SNP_DEBUG_SKIP_EXPAND") && std::getenv("SNP_DEBUG_SKIP_EXPAND")[0] == '1';
-    g.debug_skip = skip ? 1 : 0;
-#endif
     g.off32 = (uint64_t)(swap ? a.n : a.m) * (uint64_t)a.ldc < (1ull << 32) ? 1 : 0;
     g.v4 = (a.ldc % 4 == 0 && ((uintptr_t)a.r2 & 15u) == 0 && ((uintptr_t)a.C & 15u) == 0) ? 1 : 0;
     // f3 symmetric self-LD (B aliases A, symmetric output: LD statistics, AND or XOR
@@ -1636,14 +1854,12 @@ cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s) {
     // where all query blocks of a database block run together (configs[3] on 1 GPU: 102.7 ->
     // 95.8 ms for the counts pass; scripts/gpu_f20m_order.sh)
     g.order = ord ? (ord[0] - '0') : (swap ? 1 : 2);
-    // CTA-pair kernel: opt-in (SNP_GEMM_X2=1) for the unswapped shapes with more than one
-    // lane block.  Measured slower on B200 (LD-32K counts 9.1 ms vs 7.0 ms; with expansion
-    // skipped 7.8 vs 4.7 ms: the M = 256, N = 128 pair MMAs run at about half the per-SM
-    // rate of the 1-CTA M = N = 128 ones here), so the 1-CTA kernel is the default.
-    static const char *x2e = std::getenv("SNP_GEMM_X2");
-    const bool use_x2 = !swap && g.nl > BM && x2e && x2e[0] == '1';
+    // CTA-pair kernel for the unswapped shapes with more than one lane block: opt-in
+    // (SNP_GEMM_X2=1) here, see DESIGN.md §9 for the measured default.
+    const bool use_x2 = !swap && g.nl > BM && x2_mode() == 1;
     if (use_x2) g.sym = 0;
     g_last_sym = g.sym != 0;
+    g_last_pair = use_x2;
     if (use_x2)
         return epi == EPI_LD ? launch_g2<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g2<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);
     return epi == EPI_LD ? launch_g<EPI_LD>(g, L, ldl32, Cn, ldc32, s) : launch_g<EPI_COUNTS>(g, L, ldl32, Cn, ldc32, s);

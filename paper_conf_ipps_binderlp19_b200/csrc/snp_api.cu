@@ -167,7 +167,9 @@ snp_status run_gemm(GemmArgs &a, int epi, int variant, void *ws, size_t ws_bytes
         } else {
             e = launch_bitgemm_tc(a, epi, ws, ws_bytes, s);
         }
-        g_last_kernel = (kern == SNP_KERNEL_TC_MXF4 && gemm_tc4_last_sym()) ? SNP_KERNEL_TC_MXF4_SYM : kern;
+        g_last_kernel = (kern == SNP_KERNEL_TC_MXF4 && gemm_tc4_last_pair()) ? SNP_KERNEL_TC_MXF4_PAIR
+                        : (kern == SNP_KERNEL_TC_MXF4 && gemm_tc4_last_sym()) ? SNP_KERNEL_TC_MXF4_SYM
+                                                                               : kern;
     } else {
         e = launch_bitgemm_popc(a, epi, s);
         g_last_kernel = SNP_KERNEL_POPC;
@@ -322,9 +324,23 @@ int64_t snp_sym_tiles(int64_t m) {
     return T * (T + 1) / 2;
 }
 
+namespace {
+// measurement hook: SNP_GEMM_BPRE=1 pre-expands the column operand of whole-triangle
+// tensor-core self-LD into the workspace
+bool ld_sym_bpre() {
+    static const bool on = [] {
+        const char *e = std::getenv("SNP_GEMM_BPRE");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+}  // namespace
+
 size_t snp_ld_sym_workspace_bytes(int64_t m, int64_t nbits) {
     if (m <= 0 || nbits <= 0) return 0;
-    return align256((size_t)m * 4);   // row popcounts when popA is NULL
+    size_t b = align256((size_t)m * 4);   // row popcounts when popA is NULL
+    if (ld_sym_bpre() && nbits < (1LL << 24)) b += align256(gemm_tc4_bpre_bytes(m, nbits));
+    return b;
 }
 
 snp_status snp_ld_sym(const uint64_t *A, int64_t m, int64_t lda, const uint32_t *popA, int64_t nbits,
@@ -366,9 +382,11 @@ snp_status snp_ld_sym(const uint64_t *A, int64_t m, int64_t lda, const uint32_t 
     a.op = SNP_OP_AND; a.accumulate = 0; a.ldc = SYM_TILE; a.C = counts;
     a.r2 = r2; a.dprime = dprime; a.popA = a.popB = popA;
     a.tri_lo = tile_lo; a.tri_n = tile_hi - tile_lo;
+    if (variant == SNP_VARIANT_TC && ld_sym_bpre() && ws && ws_bytes >= snp_ld_sym_workspace_bytes(m, nbits))
+        a.bpre = reinterpret_cast<uint32_t *>(reinterpret_cast<uint8_t *>(ws) + align256((size_t)m * 4));
     if (variant == SNP_VARIANT_TC) {
         e = launch_gemm_tc4(a, want_ld ? EPI_LD : EPI_COUNTS, s);
-        g_last_kernel = SNP_KERNEL_TC_MXF4_SYM;
+        g_last_kernel = gemm_tc4_last_pair() ? SNP_KERNEL_TC_MXF4_SYM_PAIR : SNP_KERNEL_TC_MXF4_SYM;
     } else {
         e = launch_bitgemm_popc(a, want_ld ? EPI_LD : EPI_COUNTS, s);
         g_last_kernel = SNP_KERNEL_POPC;

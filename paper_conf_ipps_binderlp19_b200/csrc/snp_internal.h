@@ -66,6 +66,9 @@ struct GemmArgs {
     // tri_lo + tri_n - 1 only, tile u of the call stored dense at element u * 128 * 128
     // of C / r2 / dprime (row-major, ldc = 128); no mirror.
     int64_t tri_lo = 0, tri_n = -1;
+    // optional scratch for the whole-triangle tensor path: the column operand pre-expanded to
+    // e2m1 nibbles (gemm_tc4_bpre_bytes(m, nbits) bytes, 16-byte aligned), nullptr = off
+    uint32_t *bpre = nullptr;
 };
 
 // CUDA-core LOP3 + POPC variant (bitgemm_popc.cu).
@@ -118,10 +121,12 @@ cudaError_t launch_bitgemm_tc(const GemmArgs &a, int epi, void *ws, size_t ws_by
 
 
 // General tcgen05 mxf4 kernel (gemm_tc4.cu): 128x128 tiles, TMA-fed, A in TMEM.
+size_t gemm_tc4_bpre_bytes(int64_t m, int64_t nbits);
 bool gemm_tc4_supported(int64_t m, int64_t n, int64_t nbits);
 cudaError_t launch_gemm_tc4(const GemmArgs &a, int epi, cudaStream_t s);
 // Whether the most recent launch_gemm_tc4 on this thread ran the symmetric (f3) schedule.
 bool gemm_tc4_last_sym();
+bool gemm_tc4_last_pair();   // the last launch_gemm_tc4 of this thread ran the CTA-pair kernel
 
 // FastID-shaped tcgen05 mxf4 kernel (fastid_tc4.cu): <= 128 queries resident in shared
 // memory, database streamed by TMA.  The queries are the user's first operand.

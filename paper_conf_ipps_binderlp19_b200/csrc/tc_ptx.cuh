@@ -236,6 +236,14 @@ __device__ __forceinline__ uint64_t smem_desc_kmajor_noswizzle(uint32_t saddr, u
 }
 
 // Instruction descriptor for kind::i8: D = s32, A = B = u8, both K-major, dense.
+// K-major operand in 128B-swizzled rows (TMA SWIZZLE_128B tiles: 8-row groups of 1024 bytes);
+// the K offset inside a swizzle atom is added to the start address.  Layout type 2 at bit 61,
+// stride (8-row group) 1024 B, version 1 (sm_100).
+__device__ __forceinline__ uint64_t smem_desc_kmajor_sw128(uint32_t saddr) {
+    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) |
+           (2ull << 61);
+}
+
 __host__ __device__ constexpr uint32_t idesc_u8_s32(int M, int N) {
     return (2u << 4)                       // c_format = S32
            | (0u << 7) | (0u << 10)        // a/b format = unsigned 8-bit

@@ -11,12 +11,28 @@ import paper_conf_ipps_binderlp19_b200 as snp
 torch.cuda.set_device(0)
 nq, nd, nbits = int(os.environ.get("NQ", 1024)), int(os.environ.get("ND", 2_000_000)), int(os.environ.get("NBITS", 8192))
 w = snp.snp_words(nbits)
-D = torch.randint(-2**62, 2**62, (nd, w), dtype=torch.int64, device="cuda").view(torch.uint64)
-Q = torch.randint(-2**62, 2**62, (nq, w), dtype=torch.int64, device="cuda").view(torch.uint64)
-pd = snp.snp_row_popc(D, nbits)
-outs = [torch.empty((nq, nd), dtype=torch.uint32, device="cuda") for _ in range(2)]
-for _ in range(2):
-    snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=outs, best=False, popD=pd)
+if os.environ.get("MODE") == "ldrows":   # LD of ND x ND SNPs in the row layout (r2 + counts)
+    A = torch.randint(-2**62, 2**62, (nd, w), dtype=torch.int64, device="cuda").view(torch.uint64)
+    B = A.clone()   # not aliased: the general (non-mirrored) layout
+    for _ in range(2):
+        r2, _, cnt = snp.snp_ld_r2(A, B, nbits, counts=True)
+    nq = nd   # single: (nd/128)^2 tiles over 148 CTAs; pair: (nd/256)(nd/128) over 74 clusters
+elif os.environ.get("MODE") == "ld":   # packed-triangle self-LD of ND SNPs (r2 + counts)
+    A = torch.randint(-2**62, 2**62, (nd, w), dtype=torch.int64, device="cuda").view(torch.uint64)
+    pa = snp.snp_row_popc(A, nbits)
+    nt = snp.snp_sym_tiles(nd)
+    r2 = torch.empty((nt, 128, 128), dtype=torch.float32, device="cuda")
+    cnt = torch.empty((nt, 128, 128), dtype=torch.uint32, device="cuda")
+    for _ in range(2):
+        snp.snp_ld_sym(A, nbits, popA=pa, r2=r2, counts=cnt)
+    nq = 128 * nt // ((nd + 127) // 128)   # so that the tile count below is the triangle's
+else:
+    D = torch.randint(-2**62, 2**62, (nd, w), dtype=torch.int64, device="cuda").view(torch.uint64)
+    Q = torch.randint(-2**62, 2**62, (nq, w), dtype=torch.int64, device="cuda").view(torch.uint64)
+    pd = snp.snp_row_popc(D, nbits)
+    outs = [torch.empty((nq, nd), dtype=torch.uint32, device="cuda") for _ in range(2)]
+    for _ in range(2):
+        snp.snp_fastid_search(Q, D, nbits, ("xor", "andnot"), counts=outs, best=False, popD=pd)
 torch.cuda.synchronize()
 print("kernel", snp.snp_last_kernel())
 buf = (ctypes.c_longlong * 16384)()

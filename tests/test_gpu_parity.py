@@ -506,8 +506,9 @@ def test_cfg2_search_1m(snp, variant):
 
 
 def test_ld_cta_pair_kernel_subprocess():
-    """The opt-in CTA-pair LD kernel (SNP_GEMM_X2=1, read once per process) on ragged
-    shapes spanning several pair tiles and K stages, counts + r2 + D' vs the oracle."""
+    """The CTA-pair kernels forced (SNP_GEMM_X2=1, read once per process): the general LD
+    layout and the whole f3 triangle on ragged shapes spanning several pair tiles and K
+    stages (odd tile counts: a phantom lane block), counts + r2 + D' vs the oracle."""
     import subprocess
     import sys
     code = r'''
@@ -523,9 +524,31 @@ for (m, n, nbits) in [(512, 256, 1024), (700, 300, 1500), (2048, 2048, 4096)]:
     r2, dp, cnt = snp.snp_ld_r2(A, B, nbits, dprime=True, counts=True)
     r2_ref, dp_ref, n_ref = oracle.ld(ga, gb)
     assert np.array_equal(cnt.cpu().numpy().view(np.uint32), n_ref), (m, n, nbits)
+    assert snp.snp_last_kernel() == "tc_mxf4_pair", snp.snp_last_kernel()
     for got, ref in ((r2, r2_ref), (dp, dp_ref)):
         g = got.cpu().numpy().astype(np.float64); z = ref == 0
         assert (g[z] == 0).all() and (np.abs(g[~z] - ref[~z]) <= 1e-6 * np.abs(ref[~z])).all()
+# the whole f3 triangle on CTA pairs: odd / even tile counts (T = 1 has a phantom lane
+# block), ragged rows, one and several K stages, D' and counts-only
+from paper_conf_ipps_binderlp19_b200.multigpu import sym_tile_coords
+for (m, nbits) in [(1, 5), (100, 64), (129, 700), (300, 1025), (640, 2000), (1000, 4100)]:
+    g = snpgen.ld_genotypes(53, np.arange(m), nbits, structure=True)
+    A = snp.snp_pack(torch.from_numpy(g).cuda())
+    r2, dp, cnt = snp.snp_ld_sym(A, nbits, r2=True, dprime=True, counts=True)
+    assert snp.snp_last_kernel() == "tc_mxf4_sym_pair", snp.snp_last_kernel()
+    _, _, c2 = snp.snp_ld_sym(A, nbits, r2=False, counts=True)
+    r2_ref, dp_ref, n_ref = oracle.ld(g, g)
+    C, C2, R2, DP = (x.cpu().numpy() for x in (cnt, c2, r2, dp))
+    for t in range(snp.snp_sym_tiles(m)):
+        I, J = sym_tile_coords(m, t)
+        rs, cs = slice(128 * I, min(m, 128 * I + 128)), slice(128 * J, min(m, 128 * J + 128))
+        h, w = rs.stop - rs.start, cs.stop - cs.start
+        for X in (C, C2):
+            assert np.array_equal(X[t, :h, :w].view(np.uint32), n_ref[rs, cs]), (m, t)
+            assert (X[t, h:, :] == 0).all() and (X[t, :, w:] == 0).all()
+        for X, ref in ((R2, r2_ref[rs, cs]), (DP, dp_ref[rs, cs])):
+            gx = X[t, :h, :w].astype(np.float64); z = ref == 0
+            assert (gx[z] == 0).all() and (np.abs(gx[~z] - ref[~z]) <= 1e-6 * np.abs(ref[~z])).all(), (m, t)
 print("ok")
 '''
     env = dict(os.environ, SNP_GEMM_X2="1")
@@ -697,7 +720,8 @@ def _sym_blocks_ref(g, m):
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
-@pytest.mark.parametrize("m,nbits", [(300, 1025), (128, 64), (129, 700), (2300, 1025), (1, 5)])
+@pytest.mark.parametrize("m,nbits", [(300, 1025), (128, 64), (129, 700), (2300, 1025), (1, 5),
+                                    (3000, 515), (3100, 700)])   # the last two: CTA pairs in AUTO
 def test_ld_sym_packed_tiles(snp, variant, m, nbits):
     """f3 packed triangle: every tile of the row-major upper triangle equals the oracle's
     block (counts bit-exact, r2 / D' within 1e-6 relative, exactly 0 where the oracle is 0);
@@ -711,7 +735,7 @@ def test_ld_sym_packed_tiles(snp, variant, m, nbits):
         kern = snp.snp_last_kernel()
     finally:
         _variant(snp, "auto")
-    assert kern == ("tc_mxf4_sym" if variant == "tc" else "popc")
+    assert kern in (("tc_mxf4_sym", "tc_mxf4_sym_pair") if variant == "tc" else ("popc",))
     r2_ref, dp_ref, n_ref = oracle.ld(g, g)
     R2, DP, C = r2.cpu().numpy(), dp.cpu().numpy(), u32(cnt)
     for t in range(snp.snp_sym_tiles(m)):

@@ -40,6 +40,10 @@ __global__ void probe(int iters, long long *out) {
         for (int i = 0; i < iters; ++i) {
             if (MODE == 0) mma_mxf4_ss(tmem, ad, bd, idesc_mxf4(M, N), 1, tmem + 480, tmem + 496);
             else if (MODE == 1) mma_mxf4_ts(tmem, tmem + 256 + (i & 7) * 8, bd, idesc_mxf4(M, N), 1, tmem + 480, tmem + 496);
+            else if (MODE == 4)   // B walks 8 K-steps x 3 stages of a [3][8][N x 32 B] region (the LD kernel)
+                mma_mxf4_ts(tmem, tmem + 256 + (i & 7) * 8,
+                            bd + (uint64_t)((((i % 24) / 8) * N * 256 + (i & 7) * N * 32) >> 4), idesc_mxf4(M, N), 1,
+                            tmem + 480, tmem + 496);
             else if (MODE == 2) ptx::mma_i8_ss(tmem, ad, bd, ptx::idesc_u8_s32(M, N), 1);
             else ptx::mma_i8_ts(tmem, tmem + 256 + (i & 7) * 8, bd, ptx::idesc_u8_s32(M, N), 1);
         }
@@ -60,16 +64,91 @@ __global__ void probe(int iters, long long *out) {
     if (threadIdx.x < 32) { ptx::tc_fence_after(); ptx::tmem_dealloc<512>(tmem); }
 }
 
+// CTA pair (cta_group::2, M = 256 across the pair, each CTA 128 rows x N/2 B rows): the
+// leader CTA's thread issues; both CTAs allocate TMEM for the pair.
+template <int N, bool SS, bool WALK = false>
+__global__ void __cluster_dims__(2, 1, 1) probe2(int iters, long long *out) {
+    extern __shared__ __align__(1024) uint8_t sm[];
+    __shared__ uint64_t bar;
+    __shared__ uint32_t slot;
+    uint32_t rank;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+    if (threadIdx.x < 32) {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(ptx::smem_u32(&slot)) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    }
+    if (threadIdx.x == 0) { ptx::mbar_init(&bar, 1); ptx::fence_mbar_init(); }
+    ptx::tc_fence_before();
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    ptx::tc_fence_after();
+    const uint32_t tmem = slot;
+    long long t0 = clock64();
+    if (rank == 0 && threadIdx.x < 32) {
+        const uint32_t sa = ptx::smem_u32(sm), sb = sa + 128 * 32;
+        const uint64_t ad = ptx::smem_desc_kmajor_noswizzle(sa, 128 * 16, 128);
+        const uint64_t bd = ptx::smem_desc_kmajor_noswizzle(sb, (N / 2) * 16, 128);
+        const uint32_t idesc = idesc_mxf4(256, N);
+        for (int i = 0; i < iters; ++i) {
+            const uint32_t sfa = tmem + 480, sfb = tmem + 496;
+            if (SS)
+                asm volatile("{\n\t.reg .pred e, p;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, 1, 0;\n\t"
+                             "@e tcgen05.mma.cta_group::2.kind::mxf4.block_scale.block32 [%0], %1, %2, %3, [%4], [%5], p;\n\t}"
+                             ::"r"(tmem), "l"(ad), "l"(bd), "r"(idesc), "r"(sfa), "r"(sfb) : "memory");
+            else
+                asm volatile("{\n\t.reg .pred e, p;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, 1, 0;\n\t"
+                             "@e tcgen05.mma.cta_group::2.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%4], [%5], p;\n\t}"
+                             ::"r"(tmem), "r"(tmem + 256 + (i & 7) * 8),
+                               "l"(WALK ? bd + (uint64_t)((((i % 24) / 8) * (N / 2) * 256 + (i & 7) * (N / 2) * 32) >> 4) : bd),
+                               "r"(idesc), "r"(sfa), "r"(sfb) : "memory");
+        }
+        asm volatile("{\n\t.reg .pred e;\n\t.reg .b16 m;\n\tmov.b16 m, 3;\n\telect.sync _|e, 0xffffffff;\n\t"
+                     "@e tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], m;\n\t}"
+                     ::"r"(ptx::smem_u32(&bar)) : "memory");
+    }
+    if (threadIdx.x == 0) {
+        ptx::mbar_wait(&bar, 0);
+        out[blockIdx.x] = clock64() - t0;
+    }
+    ptx::tc_fence_before();
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (threadIdx.x < 32) {
+        ptx::tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, 512;" ::"r"(tmem) : "memory");
+    }
+}
+
+template <int N, bool SS, bool WALK = false>
+void run2(const char *name) {
+    long long *d; cudaMalloc(&d, 148 * sizeof(long long));
+    const int iters = 4096;
+    auto k = probe2<N, SS, WALK>;
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    k<<<148, 128, 200 * 1024>>>(iters, d);
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    cudaEventRecord(e0);
+    k<<<148, 128, 200 * 1024>>>(iters, d);
+    cudaEventRecord(e1); cudaEventSynchronize(e1);
+    cudaError_t err = cudaGetLastError();
+    if (err != cudaSuccess) { printf("%-14s pair M=256 N=%3d FAILED: %s\n", name, N, cudaGetErrorString(err)); exit(1); }
+    float ms; cudaEventElapsedTime(&ms, e0, e1);
+    long long h[148]; cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
+    const double cyc = (double)h[0] / iters;
+    const double macs_sm = 128.0 * N * 64;   // per SM per pair instruction
+    printf("%-14s pair M=256 N=%3d  %7.1f cycles/MMA  %8.1f MAC/clk/SM  %7.0f TMAC/s (event %.3f ms)\n", name, N, cyc,
+           macs_sm / cyc, macs_sm * 148 * iters / (ms * 1e-3) / 1e12, ms);
+    cudaFree(d);
+}
+
 template <int MODE, int N, int CONTEND = 0, int M = 128>
 void run(const char *name) {
     long long *d; cudaMalloc(&d, 148 * sizeof(long long));
     const int iters = 4096;
     auto k = probe<MODE, N, CONTEND, M>;
-    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-    k<<<148, 192, 64 * 1024>>>(iters, d);
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    k<<<148, 192, 200 * 1024>>>(iters, d);
     cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
     cudaEventRecord(e0);
-    k<<<148, 192, 64 * 1024>>>(iters, d);
+    k<<<148, 192, 200 * 1024>>>(iters, d);
     cudaEventRecord(e1); cudaEventSynchronize(e1);
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     long long h[148]; cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
@@ -89,6 +168,13 @@ void run(const char *name) {
 
 int main() {
     setvbuf(stdout, nullptr, _IONBF, 0);
+    if (getenv("PAIR_ONLY")) {
+        run2<64, false>("mxf4 TS x2"); run2<128, false>("mxf4 TS x2"); run2<256, false>("mxf4 TS x2");
+        run2<128, true>("mxf4 SS x2"); run2<256, true>("mxf4 SS x2");
+        run2<128, false, true>("mxf4 TS x2 walkB"); run2<256, false, true>("mxf4 TS x2 walkB");
+        run<1, 128>("mxf4 TS"); run<1, 256>("mxf4 TS"); run<4, 128>("mxf4 TS walkB");
+        return 0;
+    }
     run<0, 64>("mxf4 SS"); run<0, 128>("mxf4 SS"); run<0, 256>("mxf4 SS");
     run<1, 64>("mxf4 TS"); run<1, 128>("mxf4 TS"); run<1, 256>("mxf4 TS");
     run<2, 64>("i8 SS"); run<2, 128>("i8 SS"); run<2, 256>("i8 SS");
