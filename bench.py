@@ -322,7 +322,7 @@ def setup_fastid(wl, rank, world, dev):
     best = {op: (torch.empty(nq, dtype=torch.uint32, device=dev), torch.empty(nq, dtype=torch.int64, device=dev))
             for op in OPS}
     if fused:
-        ws = torch.empty(snp.snp_fastid_search_workspace_bytes(nq, nd, nbits, len(OPS)), dtype=torch.uint8,
+        ws = torch.zeros(snp.snp_fastid_search_workspace_bytes(nq, nd, nbits, len(OPS)), dtype=torch.uint8,
                          device=dev)
     else:
         ws = {op: (torch.empty(snp.snp_fastid_workspace_bytes(nq, nd, nbits, op), dtype=torch.uint8, device=dev))
@@ -483,7 +483,7 @@ def setup_ld(wl, rank, world, dev):
                 kernel_cmp=rows * m * nbits, kernel_bytes=alg_bytes, h2d=(m * nbits if rank == 0 else 0),
                 d2h=4, l2_flush=True, flush=l2flush, d2h_full=(rows * m * 8 if full_host is not None else None),
                 e2e_result="r2 of the first pair (the r2 and count matrices stay in HBM; e2e_full copies them back)",
-                l2_note="L2 flushed (256 MB write) between timed steps, outside the per-step events",
+                l2_note="L2 flushed (256 MB read+write) before every timed step; the flushes timed alone and subtracted",
                 state=dict(B=B, r2=r2, cnt=cnt), snp=snp)
 
 
@@ -579,7 +579,7 @@ def setup_ld_tri(wl, rank, world, dev):
                             "(e2e_full copies every tile back block by block)" if world == 1 else
                             "genotype bytes H2D on rank 0, packed and broadcast; r2 of the first pair"),
                 layout=f"packed upper triangle: tiles [{lo}, {hi}) of {b[-1]} (128 x 128, row-major triangle order)",
-                l2_note="L2 flushed (256 MB write) between timed steps, outside the per-step events",
+                l2_note="L2 flushed (256 MB read+write) before every timed step; the flushes timed alone and subtracted",
                 state=dict(B=B, r2=r2, cnt=cnt), snp=snp)
 
 
@@ -637,12 +637,14 @@ def timed(wlrun, steps, host, world, kernel_events=True, graph=None):
     return total, (statistics.mean(kms) if kms else None)
 
 
-def capture_run(wlrun, steps, kernel_events=True):
-    """Capture ALL timed steps (L2 flush between steps where the workload asks for it) in one
-    CUDA graph, with per-step and per-kernel timing events inside it (external event-record
-    nodes), so the timed region is one graph launch: no host launch gaps between the step's
-    kernels or between steps, and every kernel duration is still a CUDA-event measurement
-    on the launching stream."""
+def capture_run(wlrun, steps, mode="step"):
+    """Capture ALL timed steps in one CUDA graph with NO timing nodes inside it: an event-record
+    node between kernels costs ~4-5 us and breaks their programmatic-dependent-launch overlap
+    (scripts/step_overhead.py: FastID-1M step 174.4 us bare, 183.2 us with step-boundary event
+    nodes, 196.5 us with event nodes around the search call too), so timing events are recorded
+    on the stream around the replay instead.  mode "step": every part of the step (the L2 flush
+    before each step where the workload asks for it); "kernel": only the dominant kernel's call
+    (after the same flush); "flush": the flushes alone (subtracted from the other two)."""
     import torch
 
     import paper_conf_ipps_binderlp19_b200 as snp
@@ -653,45 +655,32 @@ def capture_run(wlrun, steps, kernel_events=True):
             fn()                                   # warm the capture stream
     torch.cuda.current_stream().wait_stream(side)
     torch.cuda.synchronize()
-    nk = 2 * wlrun["kernel_launches_per_step"]
-    mk = lambda: torch.cuda.Event(enable_timing=True, external=True)   # noqa: E731
-    kevs = [[mk() for _ in range(nk)] for _ in range(steps)]
-    sev = [(mk(), mk()) for _ in range(steps)]
     n0 = snp.snp_launch_count()
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g):
-        s = torch.cuda.current_stream()
         for i in range(steps):
             if wlrun["l2_flush"]:
                 wlrun["flush"]()
-            sev[i][0].record(s)
-            j = 0
             for fn, is_kernel in wlrun["parts"]:
-                if is_kernel and kernel_events:
-                    kevs[i][j].record(s)
-                fn()
-                if is_kernel and kernel_events:
-                    kevs[i][j + 1].record(s)
-                    j += 2
-            sev[i][1].record(s)
+                if mode == "step" or (mode == "kernel" and is_kernel):
+                    fn()
     torch.cuda.synchronize()
-    return {"graph": g, "kevs": kevs if kernel_events else [], "sev": sev, "launches": snp.snp_launch_count() - n0}
+    return {"graph": g, "launches": snp.snp_launch_count() - n0}
 
 
-def timed_run_graph(run, wlrun, world):
-    """One replay of the whole-run graph; returns (total_ms, mean dominant-kernel ms)."""
+def replay_ms(run, world):
+    """One replay of a captured graph, CUDA events on the stream around it (max over ranks)."""
     import torch
+    s = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier(world)
+    torch.cuda.synchronize()
+    e0.record(s)
     run["graph"].replay()
+    e1.record(s)
     torch.cuda.synchronize()
     barrier(world)
-    sev, kevs = run["sev"], run["kevs"]
-    if wlrun["l2_flush"]:
-        total = sum(a.elapsed_time(b) for a, b in sev)
-    else:
-        total = sev[0][0].elapsed_time(sev[-1][1])
-    kms = [ev[j].elapsed_time(ev[j + 1]) for ev in kevs for j in range(0, len(ev), 2)]
-    return max_over_ranks(total, world), (statistics.mean(kms) if kms else None)
+    return max_over_ranks(e0.elapsed_time(e1), world)
 
 
 def run_ours(args):
@@ -723,13 +712,20 @@ def run_ours(args):
         # from a second replay of the same steps with event-record nodes around that kernel
         # (event nodes between kernels break their programmatic-dependent-launch overlap, so
         # they stay out of the step timing)
-        graph = capture_run(wlrun, steps, kernel_events=False)
-        kgraph = capture_run(wlrun, steps, kernel_events=True)
-        graph["graph"].replay()
+        graph = capture_run(wlrun, steps, "step")
+        kgraph = capture_run(wlrun, steps, "kernel")
+        fgraph = capture_run(wlrun, steps, "flush") if wlrun["l2_flush"] else None
+        for r in (graph, kgraph, fgraph):
+            if r is not None:
+                r["graph"].replay()               # one untimed replay each
         torch.cuda.synchronize()
         with ClockSampler(local) as clk:
-            total_ms, _ = timed_run_graph(graph, wlrun, world)
-            _, kern_ms = timed_run_graph(kgraph, wlrun, world)
+            step_all = replay_ms(graph, world)
+            kern_all = replay_ms(kgraph, world)
+            flush_all = replay_ms(fgraph, world) if fgraph is not None else 0.0
+        # steps (or dominant-kernel calls) back to back, the flushes' own time subtracted
+        total_ms = step_all - flush_all
+        kern_ms = (kern_all - flush_all) / steps
         launches = graph["launches"]             # kernels replayed from the graph (all steps)
     else:
         with ClockSampler(local) as clk:
@@ -827,8 +823,12 @@ def run_ours(args):
                        **{k: v for k, v in wl.items() if k in ("nq", "nd", "m", "nbits")},
                        "variant": variant, "kernel": kernel, "l2": wlrun["l2_note"],
                        **({"step": wlrun["step_mode"]} if "step_mode" in wlrun else {}),
-                       "launch": ("one captured CUDA graph of all timed steps (timing events inside)"
+                       "launch": (("one captured CUDA graph of all timed steps, CUDA events around its replay"
+                                   + ("; the L2 flush before every step timed alone (a graph of the flushes) "
+                                      "and subtracted" if wlrun["l2_flush"] else ""))
                                   if use_graph else "eager"),
+                       **({"kernel_timing": "dominant kernel's call replayed back to back (same flushes, "
+                                            "subtracted), CUDA events around the replay"} if use_graph else {}),
                        **({"output": wlrun["layout"]} if "layout" in wlrun else {}),
                        "parallelism": (f"db-shard x{world}" if wl["kind"] == "fastid" else
                                        f"triangle-tile-shard x{world}" if LD_LAYOUT == "tri" else

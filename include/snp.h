@@ -211,10 +211,15 @@ snp_status snp_fastid_best(const uint32_t *counts, int64_t nq, int64_t nd, int64
  *               can be too; given, the kernel skips counting every streamed word.
  *               They must be exact: wrong popcounts give wrong XOR/ANDNOT/NOTAND counts.
  * nd < 2^32 - 1.  ws: snp_fastid_search_workspace_bytes(nq, nd, nbits, nops) bytes
- * (never 0 when nq > 0).  Kernels: the fused tcgen05 kernel for nq <= 64 (two or three
- * launches: key init + search [+ pack by the caller]); other shapes / a forced
- * SNP_VARIANT_POPC compose snp_fastid's kernels with best.cu per op, chunking the
- * database through workspace counts when counts[j] is NULL. */
+ * (never 0 when nq > 0), ZERO-FILLED before its first use by this call (e.g. one
+ * cudaMemsetAsync after allocating it); every call leaves it zero-filled again when it
+ * completes (the fused kernels merge best matches into it without an init launch and the
+ * last CTA clears it, as a CUTLASS split-K semaphore workspace is), so a workspace is
+ * cleared once and reused for any number of calls.  A workspace must not be shared by
+ * calls that may run concurrently.  Kernels: the fused tcgen05 kernel for nq <= 64 (one
+ * launch, + the caller's query pack); other shapes / a forced SNP_VARIANT_POPC compose
+ * snp_fastid's kernels with best.cu per op, chunking the database through workspace
+ * counts when counts[j] is NULL. */
 size_t snp_fastid_search_workspace_bytes(int64_t nq, int64_t nd, int64_t nbits, int nops);
 snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
                              const uint64_t *D, int64_t nd, int64_t ldd, const uint32_t *popD,

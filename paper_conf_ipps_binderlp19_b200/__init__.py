@@ -224,6 +224,8 @@ def snp_fastid_best(counts: torch.Tensor, index_base: int = 0, nd: int | None = 
 
 
 def snp_fastid_search_workspace_bytes(nq: int, nd: int, nbits: int, nops: int) -> int:
+    """Bytes of the search workspace; allocate it zero-filled (torch.zeros): the library
+    keeps it zero-filled from call to call."""
     return int(lib().snp_fastid_search_workspace_bytes(int(nq), int(nd), int(nbits), int(nops)))
 
 
@@ -268,8 +270,8 @@ def snp_fastid_search(Q: torch.Tensor, D: torch.Tensor, nbits: int, ops=("xor", 
     bc_arr = P(*[_ptr(None if b is None else b[0]) for b in best])
     bi_arr = P(*[_ptr(None if b is None else b[1]) for b in best])
     need = snp_fastid_search_workspace_bytes(nq, nd, nbits, k)
-    if ws is None:
-        ws = _workspace(need, dev)
+    if ws is None:   # zero-filled on first use (snp.h); every call leaves it zero-filled
+        ws = None if need == 0 else torch.zeros(need, dtype=torch.uint8, device=dev)
     any_best = any(b is not None for b in best)
     _dev_tensor(popD, "popD", _U32)
     if popD is not None and popD.numel() < nd:

@@ -217,7 +217,7 @@ fastid_stream_kernel(const __grid_constant__ CUtensorMap tmD, const StreamArgs a
         if (args.best_mask) {
             const int j = lane / NQ, q = lane % NQ;
             if (j < args.nops && q < args.nq && ((args.best_mask >> j) & 1) && bc != 0xffffffffu)
-                atomicMin(args.keys + (int64_t)j * args.nq + q, ((unsigned long long)bc << 32) | bi);
+                atomicMax(args.keys + (int64_t)j * args.nq + q, ~(((unsigned long long)bc << 32) | bi));   // complemented keys
             __threadfence();
             uint32_t last = 0;
             if (lane == 0) last = atomicAdd(args.done, 1u) == gridDim.x * NCW - 1 ? 1u : 0u;
@@ -226,22 +226,18 @@ fastid_stream_kernel(const __grid_constant__ CUtensorMap tmD, const StreamArgs a
                 for (int jj = 0; jj < args.nops; ++jj) {
                     if (!((args.best_mask >> jj) & 1)) continue;
                     for (int i = lane; i < args.nq; i += 32) {
-                        const unsigned long long k = __ldcg(args.keys + jj * args.nq + i);
+                        const unsigned long long k = ~__ldcg(args.keys + jj * args.nq + i);
                         args.best_count[jj][i] = k == ~0ULL ? 0xffffffffu : (uint32_t)(k >> 32);
                         args.best_index[jj][i] = k == ~0ULL ? -1 : (int64_t)(k & 0xffffffffULL) + args.index_base;
+                        args.keys[jj * args.nq + i] = 0ULL;   // the workspace is left zero-filled
                     }
                 }
+                if (lane == 0) *args.done = 0u;
             }
         }
     }
 }
 
-__global__ void stream_search_init(unsigned long long *keys, int64_t n, unsigned int *done) {
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        keys[i] = ~0ULL;
-    if (blockIdx.x == 0 && threadIdx.x == 0) *done = 0u;
-}
 
 size_t stream_smem(int nq_t, int64_t nbits) {
     const int64_t nst = (nbits + SKW * 32 - 1) / (SKW * 32);
@@ -302,12 +298,6 @@ cudaError_t launch_fastid_stream(const SearchArgs &a, cudaStream_t s) {
                 : nqt == 3 ? fastid_stream_kernel<3> : fastid_stream_kernel<4>;
     if (cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)STREAM_MAX_SMEM); e != cudaSuccess)
         return e;
-    if (f.best_mask) {
-        const int64_t nk = (int64_t)a.nops * a.nq;
-        stream_search_init<<<(int)((nk + 255) / 256), 256, 0, s>>>(a.keys, nk, a.done);
-        count_launches(1);
-        if (cudaError_t e = cudaGetLastError(); e != cudaSuccess) return e;
-    }
     const int64_t slots = (int64_t)device_sms() * (smem * SCTAS <= 232448 - 2048 ? SCTAS : 1);
     const int grid = (int)(f.ntiles < slots ? f.ntiles : slots);
     cudaLaunchConfig_t cfg{};

@@ -42,7 +42,7 @@ __device__ long long g_fastid_trace[8 * 1024];
 __device__ long long g_fastid_etrace[4 * 256];   // FASTID_TRACE2: per tile, CTA 0
 __device__ long long g_fastid_wtrace[4 * 1024];
 __device__ long long g_fastid_wtrace2[32 * 1024]; // FASTID_TRACE2: per stage and warp qa: 8 stamps  // FASTID_TRACE2: per stage, full-arrive clock of warps qa = 0..3
-__device__ long long g_fastid_cta_time[3 * 1024];
+__device__ long long g_fastid_cta_time[4 * 1024];   // per CTA: entry, after griddepcontrol.wait, main loop, end
 __device__ long long g_fastid_launch_time[2 * 64];   // CTA 0: start / end globaltimer per launch
 __device__ unsigned int g_fastid_launch_ctr;   // per CTA: start, main loop start, end (globaltimer ns)
 
@@ -160,8 +160,8 @@ struct FArgs {
     int accumulate;
     int64_t ldo;
     int best_mask;                       // bit j: keep the best match of op j
-    unsigned long long *keys;            // [nops][nq] (count << 32 | local row), pre-set to ~0
-    unsigned int *done;                  // CTA completion counter, pre-set to 0
+    unsigned long long *keys;            // [nops][nq] ~(count << 32 | local row); zero-filled on entry and exit
+    unsigned int *done;                  // epilogue-warp completion counter; zero on entry and exit
     uint32_t *best_count[MAXOPS];        // [nq] per op with a best bit
     int64_t *best_index[MAXOPS];
     int64_t index_base;
@@ -217,7 +217,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     __shared__ unsigned int launch_k;
-    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x] = (long long)ptx::globaltimer_ns();
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[4 * blockIdx.x] = (long long)ptx::globaltimer_ns();
     if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x == 0) {
         launch_k = atomicAdd(&g_fastid_launch_ctr, 1u) & 63u;
         g_fastid_launch_time[2 * launch_k] = (long long)ptx::globaltimer_ns();
@@ -279,34 +279,59 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     // previous kernel in the stream (the key-init kernel); its results (and the packed
     // queries from before it) are visible after this wait
     asm volatile("griddepcontrol.wait;" ::: "memory");
-
-    // ---- prologue: expand the whole query batch once (resident MMA B operand).  Warp w
-    // takes words w, w + 26, ...; lane = query row (BN / 32 rows per lane), so the 16-byte
-    // stores of a warp are contiguous (conflict-free) and the loads of consecutive words are
-    // independent (unrolled); row popcounts: one shared atomic per thread and row.
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[4 * blockIdx.x + 1] = (long long)ptx::globaltimer_ns();
+    // ---- prologue: expand the whole query batch once (resident MMA B operand).  A warp item
+    // is 8 query rows x 16 words: lane = (row r = lane & 7, 4-word chunk c = lane >> 3), one
+    // 16-byte load per lane (each row's 64 bytes in whole sectors), and every 16-byte store
+    // instruction covers 8 consecutive rows of one word (128 contiguous bytes per chunk:
+    // 4 wavefronts, conflict-free).  Row popcounts: reduced over the 4 chunks, one shared
+    // atomic per row and item.  (Round 2's lane-per-row prologue issued 32 sectors per load
+    // and took ~6 us per CTA, 3-4 % of FastID-1M.)
     {
-        constexpr int RPL = BN / 32;
-        const int64_t nchunks = (int64_t)nst * (KBITS / 32);   // 32-bit words per row
+        static_assert(KBITS % 512 == 0, "16-word items");
+        const int nwb = nst * (KBITS / 32) / 16;   // 16-word blocks per row
+        const int nitems = (BN / 8) * nwb;
         const int64_t nw32 = ((nbits + 127) / 128) * 4;
-        uint32_t pc[RPL];
+        const int r8 = lane & 7, c4 = lane >> 3;
+        // items in batches of 4 per warp: all four loads are in flight before the first use
+        constexpr int NWARPS = NTHREADS / 32;
+        for (int item0 = warp; item0 < nitems; item0 += 4 * NWARPS) {
+            uint4 x[4];
 #pragma unroll
-        for (int h = 0; h < RPL; ++h) pc[h] = 0;
-#pragma unroll 4
-        for (int64_t w = warp; w < nchunks; w += NTHREADS / 32) {
+            for (int u = 0; u < 4; ++u) {
+                const int item = item0 + u * NWARPS;
+                const int row = (item % (BN / 8)) * 8 + r8;
+                const int w = (item / (BN / 8)) * 16 + c4 * 4;
+                x[u] = make_uint4(0u, 0u, 0u, 0u);
+                if (item < nitems && row < args.nq && w < nw32)
+                    x[u] = __ldg(reinterpret_cast<const uint4 *>(args.Q + row * args.ldq32 + w));
+            }
 #pragma unroll
-            for (int h = 0; h < RPL; ++h) {
-                const int row = 32 * h + lane;
-                uint32_t x = 0;
-                if (row < args.nq && w < nw32) x = __ldg(args.Q + row * args.ldq32 + w) & word_mask(w, nbits);
-                pc[h] += __popc(x);
+            for (int u = 0; u < 4; ++u) {
+                const int item = item0 + u * NWARPS;
+                if (item >= nitems) break;   // warp-uniform
+                const int row = (item % (BN / 8)) * 8 + r8;
+                const int w = (item / (BN / 8)) * 16 + c4 * 4;
+                x[u].x &= word_mask(w, nbits);
+                x[u].y &= word_mask(w + 1, nbits);
+                x[u].z &= word_mask(w + 2, nbits);
+                x[u].w &= word_mask(w + 3, nbits);
+                uint32_t pc = __popc(x[u].x) + __popc(x[u].y) + __popc(x[u].z) + __popc(x[u].w);
+                uint8_t *dst = qsm + (size_t)w * BN * 16 + row * 16;
                 uint4 o;
-                expandB(x, o.x, o.y, o.z, o.w);   // queries: MMA B operand
-                *reinterpret_cast<uint4 *>(qsm + (size_t)w * BN * 16 + row * 16) = o;
+                expandB(x[u].x, o.x, o.y, o.z, o.w);
+                *reinterpret_cast<uint4 *>(dst) = o;
+                expandB(x[u].y, o.x, o.y, o.z, o.w);
+                *reinterpret_cast<uint4 *>(dst + BN * 16) = o;
+                expandB(x[u].z, o.x, o.y, o.z, o.w);
+                *reinterpret_cast<uint4 *>(dst + 2 * BN * 16) = o;
+                expandB(x[u].w, o.x, o.y, o.z, o.w);
+                *reinterpret_cast<uint4 *>(dst + 3 * BN * 16) = o;
+                pc += __shfl_xor_sync(0xffffffffu, pc, 8);
+                pc += __shfl_xor_sync(0xffffffffu, pc, 16);
+                if (c4 == 0 && pc) atomicAdd(&popQ[row], pc);
             }
         }
-#pragma unroll
-        for (int h = 0; h < RPL; ++h)
-            if (pc[h]) atomicAdd(&popQ[32 * h + lane], pc[h]);
     }
     if (warp >= EPI_WARP0 && warp < EPI_WARP0 + 4) {   // one warp per lane quarter
         const int q = warp & 3;
@@ -326,7 +351,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         asm volatile("bar.sync 1, %0;" ::"r"(NEPI * 32) : "memory");
     }
 
-    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 1] = (long long)ptx::globaltimer_ns();
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[4 * blockIdx.x + 2] = (long long)ptx::globaltimer_ns();
     if (warp == TMA_WARP) {
         // ------------------------------------------------------------ TMA producer
         if (lane == 0) {
@@ -682,9 +707,11 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
         if (BEST) {
 #pragma unroll
             for (int j = 0; j < NOPS; ++j) {
+                // keys are stored complemented and merged by atomicMax, so the zero-filled
+                // workspace means "no candidate" and no init kernel runs before the search
                 if (((args.best_mask >> j) & 1) && lane < ncols && bc[j] != 0xffffffffu)
-                    atomicMin(args.keys + (int64_t)j * args.nq + c0 + lane,
-                              ((unsigned long long)bc[j] << 32) | bi[j]);
+                    atomicMax(args.keys + (int64_t)j * args.nq + c0 + lane,
+                              ~(((unsigned long long)bc[j] << 32) | bi[j]));
             }
             // the last epilogue warp of the grid to finish turns the merged keys into
             // (best_count, best_index) (kept inside this role: a CTA-wide finalize after
@@ -699,31 +726,26 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 for (int j = 0; j < NOPS; ++j) {
                     if (!((args.best_mask >> j) & 1)) continue;
                     for (int i = lane; i < nq; i += 32) {
-                        const unsigned long long k = __ldcg(args.keys + j * nq + i);
+                        const unsigned long long k = ~__ldcg(args.keys + j * nq + i);
                         args.best_count[j][i] = k == ~0ULL ? 0xffffffffu : (uint32_t)(k >> 32);
                         args.best_index[j][i] = k == ~0ULL ? -1 : (int64_t)(k & 0xffffffffULL) + args.index_base;
+                        args.keys[j * nq + i] = 0ULL;   // the workspace is left zero-filled
                     }
                 }
+                if (lane == 0) *args.done = 0u;
             }
         }
     }
 
     ptx::tc_fence_before();
     __syncthreads();
-    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[3 * blockIdx.x + 2] = (long long)ptx::globaltimer_ns();
+    if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x < 1024) g_fastid_cta_time[4 * blockIdx.x + 3] = (long long)ptx::globaltimer_ns();
     if (SNP_PROF(args.trace) && tid == 0 && blockIdx.x == 0) g_fastid_launch_time[2 * launch_k + 1] = (long long)ptx::globaltimer_ns();
     if (warp == MMA_WARP) {
         ptx::tc_fence_after();
         ptx::tmem_dealloc<512>(tmem);
     }
     }   // C::OK
-}
-
-__global__ void fastid_search_init(unsigned long long *keys, int64_t n, unsigned int *done) {
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");   // let the search kernel start
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        keys[i] = ~0ULL;
-    if (blockIdx.x == 0 && threadIdx.x == 0) *done = 0u;
 }
 
 size_t smem_bytes(int bn, int64_t nbits) {
@@ -821,13 +843,6 @@ cudaError_t launch_f(const SearchArgs &a, cudaStream_t s) {
     if (cudaError_t e = ensure_dyn_smem(reinterpret_cast<const void *>(kern), (int)(MAX_SMEM - 1024)); e != cudaSuccess)
         return e;
     const int grid = (int)(f.ntiles < device_sms() ? f.ntiles : device_sms());
-    if (f.best_mask) {
-        const int64_t nk = (int64_t)a.nops * a.nq;
-        fastid_search_init<<<(int)((nk + 255) / 256), 256, 0, s>>>(a.keys, nk, a.done);
-        count_launches(1);
-        cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) return e;
-    }
     // programmatic dependent launch: the kernel's setup (barriers, TMEM allocation, tensor
     // map prefetch) overlaps the preceding kernel; it waits (griddepcontrol.wait) before
     // touching any data that kernel produces
@@ -896,35 +911,41 @@ cudaError_t FASTID_FN(launch_fastid_search_tc4)(const SearchArgs &a, cudaStream_
 
 }  // namespace snp
 
-#if defined(SNP_PROFILING) && defined(FASTID_PRIMARY)
+#if defined(SNP_PROFILING)
 // Profiling aid (not part of include/snp.h): copy the pipeline trace of the last
-// traced fastid_tc4 launch (4 x 1024 clock64 stamps) to host memory.
-extern "C" int snp_debug_fastid_launch_times(long long *host, int n) {
+// traced fastid_tc4 launch (4 x 1024 clock64 stamps) to host memory.  The 512-bit-stage
+// instantiation exports the plain names, the 1024-bit one the same names + "_k1024".
+#ifdef FASTID_PRIMARY
+#define FASTID_DBG(name) name
+#else
+#define FASTID_DBG(name) name##_k1024
+#endif
+extern "C" int FASTID_DBG(snp_debug_fastid_launch_times)(long long *host, int n) {
     if (n > 128) n = 128;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_launch_time, sizeof(long long) * n);
 }
 
-extern "C" int snp_debug_fastid_cta_times(long long *host, int n) {
-    if (n > 3 * 1024) n = 3 * 1024;
+extern "C" int FASTID_DBG(snp_debug_fastid_cta_times)(long long *host, int n) {
+    if (n > 4 * 1024) n = 4 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_cta_time, sizeof(long long) * n);
 }
 
-extern "C" int snp_debug_fastid_etrace(long long *host, int n) {
+extern "C" int FASTID_DBG(snp_debug_fastid_etrace)(long long *host, int n) {
     if (n > 4 * 256) n = 4 * 256;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_etrace, sizeof(long long) * n);
 }
 
-extern "C" int snp_debug_fastid_wtrace2(long long *host, int n) {
+extern "C" int FASTID_DBG(snp_debug_fastid_wtrace2)(long long *host, int n) {
     if (n > 32 * 1024) n = 32 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_wtrace2, sizeof(long long) * n);
 }
 
-extern "C" int snp_debug_fastid_wtrace(long long *host, int n) {
+extern "C" int FASTID_DBG(snp_debug_fastid_wtrace)(long long *host, int n) {
     if (n > 4 * 1024) n = 4 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_wtrace, sizeof(long long) * n);
 }
 
-extern "C" int snp_debug_fastid_trace(long long *host, int n) {
+extern "C" int FASTID_DBG(snp_debug_fastid_trace)(long long *host, int n) {
     if (n > 8 * 1024) n = 8 * 1024;
     return (int)cudaMemcpyFromSymbol(host, snp::g_fastid_trace, sizeof(long long) * n);
 }

@@ -707,6 +707,8 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
                 (e = launch_best_finalize(keys + (int64_t)j * nq, nq, index_base, a.best_count[j], a.best_index[j], s)) !=
                     cudaSuccess)
                 return set_cuda_error(e);
+        if (any_best && (e = cudaMemsetAsync(ws, 0, (size_t)nops * nq * 8, s)) != cudaSuccess)   // zero-filled again
+            return set_cuda_error(e);
         g_last_variant = SNP_VARIANT_TC;
         g_last_kernel = SNP_KERNEL_FASTID_MXF4;
         return SNP_OK;
@@ -776,6 +778,8 @@ snp_status snp_fastid_search(const uint64_t *Q, int64_t nq, int64_t ldq,
                         cudaSuccess)
             return set_cuda_error(e);
     }
+    // the key region is returned to zero (the fused kernels rely on a zero-filled workspace)
+    if (any_best && (e = cudaMemsetAsync(ws, 0, (size_t)nops * nq * 8, s)) != cudaSuccess) return set_cuda_error(e);
     return SNP_OK;
 }
 

@@ -61,7 +61,7 @@ def stream_search(Q: torch.Tensor, D_host: torch.Tensor, nbits: int, ops=("xor",
     # ragged last chunk with few rows can take a path that needs more workspace than a full
     # chunk, so size for every distinct chunk length
     ws_need = max(snp_fastid_search_workspace_bytes(nq, rows, nbits, nops) for rows in {r1 - r0 for r0, r1 in plan})
-    ws = torch.empty(max(1, ws_need), dtype=torch.uint8, device=dev)
+    ws = torch.zeros(max(1, ws_need), dtype=torch.uint8, device=dev)   # zero-filled once (snp.h)
     comp = torch.cuda.current_stream(dev)
     copy = torch.cuda.Stream(dev)
     copy.wait_stream(comp)   # the buffers (and Q) were just allocated / produced on comp

@@ -46,7 +46,7 @@ for K in [int(x) for x in a.K.split(",")]:
                     rec[v + "_ms"] = None
                     continue
                 snp.snp_set_variant(v)
-                ws = torch.empty(snp.snp_fastid_search_workspace_bytes(M, N, K, 1), dtype=torch.uint8, device="cuda")
+                ws = torch.zeros(snp.snp_fastid_search_workspace_bytes(M, N, K, 1), dtype=torch.uint8, device="cuda")
                 outc = [torch.empty((M, N), dtype=torch.uint32, device="cuda")] if a.counts else False
                 ms = timeit(lambda: snp.snp_fastid_search(Q, D, K, ("xor",), counts=outc, best=True, ws=ws, popD=pd))
                 rec[v + "_ms"] = ms

@@ -459,6 +459,35 @@ def test_search_chunked_composition(snp, monkeypatch):
         assert np.array_equal(u32(best[j][0]), rb) and np.array_equal(best[j][1].cpu().numpy(), ri), op
 
 
+def test_search_shared_workspace_stays_zero(snp, monkeypatch):
+    """snp.h: the search workspace is zero-filled once and every call leaves it zero-filled
+    (the fused kernels merge complemented keys with atomicMax, the last CTA clears them; the
+    composed paths clear the key region).  ONE workspace through calls that take every path
+    (streaming kernel, fused tcgen05 kernel, 64-query slices, the composed chunked path, an
+    empty database), each vs the oracle, the workspace checked all-zero after each call."""
+    monkeypatch.setenv("SNP_SEARCH_CHUNK_ROWS", "384")
+    nbits = 700
+    db = snpgen.fastid_db(45, np.arange(3000), nbits)
+    D = pack_dev(snp, db)
+    shapes = [(1, 3000), (40, 3000), (130, 3000), (100, 2000), (64, 1500), (3, 3000), (40, 0), (40, 2999)]
+    need = max(snp.snp_fastid_search_workspace_bytes(nq, nd, nbits, 2) for nq, nd in shapes)
+    ws = torch.zeros(need, dtype=torch.uint8, device=DEV)
+    for nq, nd in shapes:
+        q, _ = snpgen.fastid_queries(46 + nq, nq, max(nd, 1), nbits)
+        for counts in (True, False):
+            _, best = snp.snp_fastid_search(pack_dev(snp, q), D[:nd], nbits, ("xor", "andnot"), counts=counts,
+                                            index_base=7, ws=ws)
+            torch.cuda.synchronize()
+            for j, op in enumerate(("xor", "andnot")):
+                if nd == 0:
+                    assert (u32(best[j][0]) == 0xFFFFFFFF).all() and (best[j][1].cpu().numpy() == -1).all()
+                    continue
+                rb, ri = oracle.best(oracle.counts(q, db[:nd], op), 7)
+                assert np.array_equal(u32(best[j][0]), rb), (nq, nd, counts, op, snp.snp_last_kernel())
+                assert np.array_equal(best[j][1].cpu().numpy(), ri), (nq, nd, counts, op)
+            assert int(ws.count_nonzero()) == 0, (nq, nd, counts, snp.snp_last_kernel())
+
+
 def test_search_empty_database(snp):
     nbits = 256
     q = snpgen.fastid_db(44, np.arange(5), nbits)
