@@ -7,7 +7,7 @@ import paper_conf_ipps_binderlp19_b200 as snp
 torch.cuda.set_device(0)
 nq = int(os.environ.get("NQ", 64)); nd = int(os.environ.get("ND", 1_000_000)); nbits = int(os.environ.get("K", 4096))
 counts = os.environ.get("COUNTS", "1") == "1"; nops = int(os.environ.get("NOPS", 2))
-w = snp.snp_words(nbits)
+w = snp.snp_words(nbits) if os.environ.get("TIGHT") != "1" else (int(os.environ["LDW"]) if os.environ.get("LDW") else 2 * ((nbits + 127) // 128))   # TIGHT: 16-byte-granular rows
 if os.environ.get("DATA", "random") == "snpgen":   # the bench's seeded genotype recipe
     import numpy as np
     import snpgen
@@ -40,6 +40,14 @@ for _ in range(5):
     res.append(e0.elapsed_time(e1) / 20 * 1e3)
 byt = (nd + nq) * w * 8 + (len(ops) * nq * nd * 4 if counts else 0)
 lib = os.path.basename(os.environ.get("SNP_LIB_PATH", "libsnp.so"))
-print(json.dumps({"lib": lib, "data": os.environ.get("DATA", "random"), "nq": nq, "nd": nd, "nbits": nbits, "counts": counts, "best": best is not None, "kernel": snp.snp_last_kernel(),
+print(json.dumps({"lib": lib, "data": os.environ.get("DATA", "random"), "nq": nq, "nd": nd, "nbits": nbits, "ldw": w, "counts": counts, "best": best is not None, "kernel": snp.snp_last_kernel(),
                   "us_best": round(min(res), 2), "us_all": [round(x, 2) for x in res],
                   "hbm_frac": round(byt / (min(res) * 1e-6) / 6548.2e9, 4)}), flush=True)
+if os.environ.get("CHECK") == "1" and best is not None:   # vs the CUDA-core variant of the same library
+    ref = [(torch.empty(nq, dtype=torch.uint32, device="cuda"), torch.empty(nq, dtype=torch.int64, device="cuda")) for _ in ops]
+    snp.snp_set_variant("popc")
+    snp.snp_fastid_search(Q, D, nbits, ops, counts=False, best=ref, popD=pd)
+    snp.snp_set_variant("auto")
+    call(); torch.cuda.synchronize()
+    ok = all(torch.equal(a[0], b[0]) and torch.equal(a[1], b[1]) for a, b in zip(best, ref))
+    print(json.dumps({"lib": lib, "check_vs_popc": ok}), flush=True)

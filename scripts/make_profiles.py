@@ -11,7 +11,7 @@ DST = os.path.join(ROOT, "profiles", ROUND)
 os.makedirs(DST, exist_ok=True)
 
 def short(name):
-    for key in ("fastid_tc4_kernel", "fastid_stream_kernel", "gemm_tc4_kernel", "bitgemm_popc_kernel", "bitgemm_tc_kernel",
+    for key in ("gemm_tc4x2_kernel", "fastid_tc4_kernel", "fastid_stream_kernel", "gemm_tc4_kernel", "bitgemm_popc_kernel", "bitgemm_tc_kernel",
                 "pack_popc_kernel", "pack_vec_kernel", "pack_byte_kernel", "row_popc_kernel", "sym_unpack_kernel",
                 "fastid_search_init", "stream_search_init", "best_init", "best_reduce", "best_finalize"):
         if key in name:
@@ -60,7 +60,7 @@ for wl, per_step in (("fastid1m", 3), ("ld32k", 2), ("ld2k", 2), ("fastid20m", 7
         summary.append(f"## launch list {wl} (ncu gpu__time_duration.sum, cold-cache serialised; last 2 steps, {len(ks)} launches)")
         for k, (n, v) in sorted(agg.items(), key=lambda x: -x[1][1]):
             summary.append(f"  {k:24s} launches {n:3d}  total {v / 1e3:10.1f} us  share {100 * v / tot:5.1f} %")
-for name, wl, kern in (("full_fastid1m", "fastid1m", "fastid_mxf4"), ("full_ld32k", "ld32k", "tc_mxf4_sym"),
+for name, wl, kern in (("full_fastid1m", "fastid1m", "fastid_mxf4"), ("full_ld32k", "ld32k", "tc_mxf4_sym_pair"),
                        ("full_ld2k", "ld2k", "tc_mxf4_sym"), ("full_fastid20m", "fastid20m", "tc_mxf4"),
                        ("full_fastid1m_popc", "fastid1m", "popc"), ("full_stream1", "skinny1x20Mx4096", "popc_stream"),
                        ("full_skinny8", "skinny8x20Mx4096", "fastid_mxf4")):

@@ -8,7 +8,7 @@ import numpy as np, torch
 import paper_conf_ipps_binderlp19_b200 as snp
 torch.cuda.set_device(0)
 nq, nd, nbits = int(os.environ.get("NQ", 64)), int(os.environ.get("ND", 1_000_000)), int(os.environ.get("NBITS", 4096))
-w = snp.snp_words(nbits)
+w = snp.snp_words(nbits) if os.environ.get("TIGHT") != "1" else (int(os.environ["LDW"]) if os.environ.get("LDW") else 2 * ((nbits + 127) // 128))
 D = torch.randint(-2**62, 2**62, (nd, w), dtype=torch.int64, device="cuda").view(torch.uint64)
 Q = torch.randint(-2**62, 2**62, (nq, w), dtype=torch.int64, device="cuda").view(torch.uint64)
 pd = snp.snp_row_popc(D, nbits)
@@ -23,9 +23,10 @@ for _ in range(3):
         snp.snp_fastid(Q, D, nbits, "xor", out=outs[0])
 torch.cuda.synchronize()
 buf = (ctypes.c_longlong * 8192)()
-snp.lib().snp_debug_fastid_trace(buf, 8192)
+SUF = "" if os.environ.get("SNP_FASTID_KBITS") == "512" else "_k1024"
+getattr(snp.lib(), "snp_debug_fastid_trace" + SUF)(buf, 8192)
 t = np.array(buf, dtype=np.int64).reshape(1024, 8)
-nst = (nbits + 511) // 512
+nst = (nbits + (511 if SUF == "" else 1023)) // (512 if SUF == "" else 1024)
 ntile = (nd + 127) // 128 // 148
 nit = min(1024, ntile * nst)
 t = t[:nit]
@@ -44,8 +45,11 @@ for it in range(40, 56):
     print(it, r[0], r[4], r[1], r[2], "| mma", r[3], r[5])
 
 eb = (ctypes.c_longlong * 1024)()
-snp.lib().snp_debug_fastid_etrace(eb, 1024)
+getattr(snp.lib(), "snp_debug_fastid_etrace" + SUF)(eb, 1024)
 e = np.array(eb, dtype=np.int64).reshape(256, 4)[:min(ntile, 256)]
+print("per tile (rel. cycles): MMA before acce wait | after | epilogue got accf | epilogue done")
+for k in range(20, 30):
+    print(k, *(e[k] - e[20, 0]))
 print("tile: MMA acce wait", med(e[2:50, 1] - e[2:50, 0]), "mean", float((e[2:50, 1] - e[2:50, 0]).mean()),
       " epilogue busy (accf->done)", med(e[2:50, 3] - e[2:50, 2]), " tile interval (MMA)", med(np.diff(e[2:50, 1])))
 for k in range(10, 16):
