@@ -130,8 +130,17 @@ struct FCfg {
     // frees accumulator columns for more stages with 2 groups: the lane quarter that shares
     // the MMA warp's sub-partition runs ~3.5 stages behind the others (its TMEM stores queue
     // behind the issued MMAs, scripts/trace_fastid2.py), and deeper staging keeps the MMA fed.
+#if defined(FASTID_NS32_K1024)   // experiment: TMEM A stages of the 32-wide 1024-bit-stage kernels
+    static constexpr int NS_PREF = (KBITS == 1024 && BN == 32) ? FASTID_NS32_K1024
+                                 : FASTID_NS != 4 ? FASTID_NS : (BN == 32 ? FASTID_NS32 : 4);
+#else
     static constexpr int NS_PREF = FASTID_NS != 4 ? FASTID_NS : (BN == 32 ? FASTID_NS32 : 4);
+#endif
+#ifdef FASTID_NS_ANY   // experiment: slot count not a multiple of the group count
+    static constexpr int NS_FIT = NS_PREF;
+#else
     static constexpr int NS_FIT = NS_PREF / GG * GG;
+#endif
     static constexpr bool OK = NS_FIT >= GG;   // else this (BN, GG) is not instantiated for launch
     static constexpr int NS = OK ? NS_FIT : GG;
     static_assert(NP % 4 == 0, "the packed ring is shared round-robin by up to 4 groups");

@@ -445,6 +445,33 @@ def test_search_ties_lowest_index_across_ctas(snp, nq):
             _variant(snp, "auto")
 
 
+@pytest.mark.parametrize("counts", ["both", "first"])
+def test_search_general_kernel_best(snp, counts):
+    """Many-query search on the general tcgen05 kernel (swapped layout: > 64 queries above
+    4096 bits; both ops' counts from one pass, best matches by best.cu).  Exact ties spread
+    over every CTA / lane quarter / ragged last tile must give the lowest index; counts and
+    bests vs the oracle.  counts="first": op 0 stored, op 1 best-only (chunked path)."""
+    nbits, nd, nq = 4500, 20_000, 100
+    base = snpgen.fastid_db(47, np.arange(29), nbits)
+    idx = (np.arange(nd) * 11 + 5) % 29
+    db = base[idx]
+    q = base[np.arange(nq) % 29].copy()
+    q[::7, :5] ^= 1
+    D = pack_dev(snp, db)
+    Q = pack_dev(snp, q)
+    ops = ("xor", "andnot")
+    c = True if counts == "both" else [torch.empty((nq, nd), dtype=torch.uint32, device=DEV), None]
+    got, best = snp.snp_fastid_search(Q, D, nbits, ops, counts=c, index_base=3)
+    assert snp.snp_last_kernel() in ("tc_mxf4", "popc"), snp.snp_last_kernel()
+    for j, op in enumerate(ops):
+        ref = oracle.counts(q, base, op)[:, idx]
+        if got[j] is not None:
+            assert np.array_equal(u32(got[j]), ref), op
+        rb, ri = oracle.best(ref, 3)
+        assert np.array_equal(u32(best[j][0]), rb), op
+        assert np.array_equal(best[j][1].cpu().numpy(), ri), op
+
+
 def test_search_chunked_composition(snp, monkeypatch):
     """Best-only search for shapes the fused kernel does not take runs in database
     chunks through workspace counts; force small ragged chunks."""
