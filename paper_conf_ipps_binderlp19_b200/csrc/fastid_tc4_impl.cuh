@@ -454,9 +454,14 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 wv[4 * c] = x.x; wv[4 * c + 1] = x.y; wv[4 * c + 2] = x.z; wv[4 * c + 3] = x.w;
             }
             const int64_t w0 = (int64_t)s * KW;
-            if (w0 + KW > full32) {
+            if (w0 + KW > full32) {   // the profile's last stage: bits past nbits are zeroed
+                // 32-bit arithmetic on the bits left in this stage (0 < rem < KBITS)
+                const int rem = (int)(nbits - w0 * 32);
 #pragma unroll
-                for (int i = 0; i < KW; ++i) wv[i] &= word_mask(w0 + i, nbits);
+                for (int i = 0; i < KW; ++i) {
+                    const int r = rem - 32 * i;
+                    wv[i] &= r >= 32 ? 0xffffffffu : r <= 0 ? 0u : (1u << r) - 1u;
+                }
             }
             if (!pre) {
 #pragma unroll
