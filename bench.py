@@ -378,7 +378,8 @@ def setup_fastid(wl, rank, world, dev):
             # global best per query and op, lowest global index on ties: both
             # ops' (count, index) packed into int64 keys, ONE all-gather, ONE min
             from paper_conf_ipps_binderlp19_b200 import multigpu
-            keys = torch.stack([multigpu.pack_best(*best[op]) for op in OPS])
+            # bounds checked on the host from the shape (no device sync inside the timed step)
+            keys = torch.stack([multigpu.pack_best(*best[op], nbits=nbits, rows=nd_total) for op in OPS])
             merged["keys"] = multigpu.gather_best(keys)
             if host:   # e2e: D2H of the step's result, the GLOBAL best (count << 40 | index keys)
                 keys_host.copy_(merged["keys"], non_blocking=True)

@@ -50,18 +50,27 @@ KEY_IDX_BITS = 40                     # global database index < 2^40; count < 2^
 KEY_NONE = (1 << 63) - 1              # an empty shard: larger than every real key
 
 
-def pack_best(bc: torch.Tensor, bi: torch.Tensor) -> torch.Tensor:
+def pack_best(bc: torch.Tensor, bi: torch.Tensor, nbits: int | None = None, rows: int | None = None) -> torch.Tensor:
     """(best count, global best index) -> one int64 key ``count << 40 | index`` whose
     minimum over shards is the global best with the lowest-index tie-break (reading R4):
-    ONE all-gather and ONE min replace two gathers and an argmin merge."""
+    ONE all-gather and ONE min replace two gathers and an argmin merge.
+
+    A real count must stay below 2^23 (so count << 40 keeps the sign bit clear) and an index
+    below 2^40.  Given the shape (nbits bounds every count, rows every global index) the
+    bounds are checked on the host; otherwise the values are checked on the device, which
+    synchronises the stream (keep that off a timed multi-GPU step)."""
     c = (bc.view(torch.int32) if bc.dtype == torch.uint32 else bc).to(torch.int64) & 0xFFFFFFFF
-    # a real count must stay below 2^23 so count << 40 keeps the sign bit clear; counts of
-    # longer profiles go through merge_best (two-tensor gather) instead
-    real = bi >= 0
-    if bool(((c >= (1 << (63 - KEY_IDX_BITS))) & real).any()):
-        raise ValueError("pack_best: count >= 2^23 does not fit the packed key; use merge_best")
-    if bool((bi >= (1 << KEY_IDX_BITS)).any()):
-        raise ValueError("pack_best: index >= 2^40 does not fit the packed key")
+    if nbits is not None and rows is not None:
+        if nbits >= (1 << (63 - KEY_IDX_BITS)):
+            raise ValueError("pack_best: nbits >= 2^23: counts do not fit the packed key; use merge_best")
+        if rows > (1 << KEY_IDX_BITS):
+            raise ValueError("pack_best: more than 2^40 rows do not fit the packed key")
+    else:
+        real = bi >= 0
+        if bool(((c >= (1 << (63 - KEY_IDX_BITS))) & real).any()):
+            raise ValueError("pack_best: count >= 2^23 does not fit the packed key; use merge_best")
+        if bool((bi >= (1 << KEY_IDX_BITS)).any()):
+            raise ValueError("pack_best: index >= 2^40 does not fit the packed key")
     key = (c << KEY_IDX_BITS) | bi.to(torch.int64)
     return torch.where(bi < 0, torch.full_like(key, KEY_NONE), key)
 
@@ -99,8 +108,8 @@ def fastid_step(Q: torch.Tensor, D_shard: torch.Tensor, nbits: int, op: str, ind
     bc, bi = best(counts, index_base)
     if world == 1:
         return counts, bc.to(torch.int64), bi
-    nq = bc.numel()
-    c, i = unpack_best(gather_best(pack_best(bc, bi), group=group))
+    c, i = unpack_best(gather_best(pack_best(bc, bi, nbits=nbits, rows=index_base + D_shard.shape[0]),
+                                   group=group))
     return counts, c, i
 
 

@@ -153,6 +153,13 @@ def test_pack_best_rejects_counts_that_overflow_the_key():
         pack_best(torch.tensor([1 << 23]), torch.tensor([0]))
     with pytest.raises(ValueError):
         pack_best(torch.tensor([1]), torch.tensor([1 << 40]))
+    # shape-bounded form (no device sync): the host check rejects the shape instead
+    with pytest.raises(ValueError):
+        pack_best(torch.tensor([1]), torch.tensor([0]), nbits=1 << 23, rows=10)
+    with pytest.raises(ValueError):
+        pack_best(torch.tensor([1]), torch.tensor([0]), nbits=100, rows=(1 << 40) + 1)
+    k = pack_best(torch.tensor([5, 0xFFFFFFFF]), torch.tensor([7, -1]), nbits=100, rows=10)
+    assert k.tolist() == [(5 << 40) | 7, (1 << 63) - 1]
     pack_best(torch.tensor([(1 << 23) - 1, 0xFFFFFFFF]), torch.tensor([0, -1]))   # empty shard is fine
 
 
