@@ -1,1 +1,2 @@
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_exactness.py -q -x -k "fastid or search or stream or best or exact" 2>&1 | tail -2
+bash scripts/gpu_ab.sh dyn4 libsnp_headA.so libsnp.so libsnp_nodyn.so | cut -c1-170
+SNP_LIB_PATH=$PWD/paper_conf_ipps_binderlp19_b200/libsnp_prof.so timeout 300 python scripts/trace_cta.py
