@@ -82,6 +82,9 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 #ifndef FASTID_ISSUE_AHEAD
 #define FASTID_ISSUE_AHEAD 0
 #endif
+#ifndef FASTID_ELECT_STAGE
+#define FASTID_ELECT_STAGE 1   // one elect.sync per stage's block of MMAs
+#endif
 #ifndef FASTID_NACC
 #define FASTID_NACC 2   // TMEM accumulators (the MMA may run NACC - 1 tiles ahead of the epilogue)
 #endif
@@ -575,21 +578,73 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 // K-steps of this stage that hold bits < nbits (the rest would multiply zeros:
                 // a 128-SNP profile issues 2 MMAs per tile instead of KBITS / 64)
                 const int kmax = s == nst - 1 ? kmax_last : KBITS / 64;
+                if (NHALF == 1 && FASTID_ELECT_STAGE) {
+                    // one elected lane issues the stage's MMAs back to back and commits them (one
+                    // elect.sync per stage, not per MMA: the MMA issue is on the pipeline's
+                    // critical path — FastID-1M 171.5 -> 169.0 us, 8 x 20M x 4096 best-only
+                    // 2.34 -> 2.13 ms); a full stage has no per-MMA bound test
+                    if (ptx::elect_one()) {
+                        if (kmax == KBITS / 64) {
 #pragma unroll
-                for (int k = 0; k < KBITS / 64; ++k) {
-                    if (NHALF == 2 && k == KBITS / 128) {   // second half of the stage
-                        ptx::mbar_wait_uniform(&full[b * NHALF + 1], bround & 1);
-                        ptx::tc_fence_after();
+                            for (int k = 0; k < KBITS / 64; ++k)
+                                ptx::mma_mxf4_ts_one(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC,
+                                                     (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                        } else {
+#pragma unroll
+                            for (int k = 0; k < KBITS / 64; ++k) {
+                                if (k >= kmax) break;
+                                ptx::mma_mxf4_ts_one(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC,
+                                                     (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                            }
+                        }
+                        ptx::mma_commit_one(&empty[b]);
+                        if (s == nst - 1) ptx::mma_commit_one(&accf[acc]);
                     }
-                    if (NHALF == 1 && k >= kmax) break;
-                    ptx::mma_mxf4_ts(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa,
-                                     sfb);
+                    __syncwarp();
+                    bd += SSTEP;
+                    if (++b == NS) { b = 0; ++bround; }
+                    continue;
+                } else if (NHALF == 2 && FASTID_ELECT_STAGE) {
+                    // half-stage barriers: the same per-half elected issue (elect.sync picks the
+                    // same lane both times, so the commits track both halves' MMAs)
+                    constexpr int KH = KBITS / 128;
+                    if (ptx::elect_one()) {
+#pragma unroll
+                        for (int k = 0; k < KH; ++k)
+                            ptx::mma_mxf4_ts_one(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC,
+                                                 (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                    }
+                    __syncwarp();
+                    ptx::mbar_wait_uniform(&full[b * NHALF + 1], bround & 1);
+                    ptx::tc_fence_after();
+                    if (ptx::elect_one()) {
+#pragma unroll
+                        for (int k = KH; k < 2 * KH; ++k)
+                            ptx::mma_mxf4_ts_one(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC, 1u, sfa, sfb);
+                        ptx::mma_commit_one(&empty[b]);
+                        if (s == nst - 1) ptx::mma_commit_one(&accf[acc]);
+                    }
+                    __syncwarp();
+                    bd += SSTEP;
+                    if (++b == NS) { b = 0; ++bround; }
+                    continue;
+                } else {
+#pragma unroll
+                    for (int k = 0; k < KBITS / 64; ++k) {
+                        if (NHALF == 2 && k == KBITS / 128) {   // second half of the stage
+                            ptx::mbar_wait_uniform(&full[b * NHALF + 1], bround & 1);
+                            ptx::tc_fence_after();
+                        }
+                        if (NHALF == 1 && k >= kmax) break;
+                        ptx::mma_mxf4_ts(d, a0 + 8 * k, bd + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u,
+                                         sfa, sfb);
+                    }
                 }
                 ptx::mma_commit_uniform(&empty[b]);
                 bd += SSTEP;
                 if (++b == NS) { b = 0; ++bround; }
             }
-            ptx::mma_commit_uniform(&accf[acc]);
+            if (!FASTID_ELECT_STAGE) ptx::mma_commit_uniform(&accf[acc]);
         }
         __syncwarp();
     } else {

@@ -960,22 +960,40 @@ gemm_tc4_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__
                 ptx::tc_fence_after();
                 const uint32_t a0 = tmu + (uint32_t)(A_COL0 + 64 * b);
                 const uint64_t b0 = bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4);
+                if (GH == 1) {
+                    // one elected lane issues the stage's MMAs back to back and commits them
+                    // (one elect.sync per stage, not per MMA; the FastID kernel measured this
+                    // on its critical path)
+                    if (ptx::elect_one()) {
 #pragma unroll
-                for (int k = 0; k < KBITS / 64; ++k) {
-                    if (GH == 2 && k == KBITS / 128) {
-                        ptx::mbar_wait_uniform(&full[b * GH + 1], round & 1);
-                        ptx::tc_fence_after();
+                        for (int k = 0; k < KBITS / 64; ++k) {
+                            // BPRE: K-step k is bytes [32 (k % 4), +32) of the 128-byte rows of half
+                            // k / 4 (16 KB each; the descriptor's start address moves inside the
+                            // swizzle atom)
+                            const uint64_t bk = BPRE ? b0 + (uint64_t)((((k >> 2) * (BSLOT / 2)) + (k & 3) * 32) >> 4)
+                                                     : b0 + (uint64_t)(k * BSTEP);
+                            ptx::mma_mxf4_ts_one(d, a0 + 8 * k, bk, IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                        }
+                        ptx::mma_commit_one(&empty[b]);
+                        if (s == nst - 1) ptx::mma_commit_one(&accf[acc]);
                     }
-                    // BPRE: K-step k is bytes [32 (k % 4), +32) of the 128-byte rows of half k / 4
-                    // (16 KB each; the descriptor's start address moves inside the swizzle atom)
-                    const uint64_t bk = BPRE ? b0 + (uint64_t)((((k >> 2) * (BSLOT / 2)) + (k & 3) * 32) >> 4)
-                                             : b0 + (uint64_t)(k * BSTEP);
-                    ptx::mma_mxf4_ts(d, a0 + 8 * k, bk, IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                    __syncwarp();
+                } else {
+#pragma unroll
+                    for (int k = 0; k < KBITS / 64; ++k) {
+                        if (GH == 2 && k == KBITS / 128) {
+                            ptx::mbar_wait_uniform(&full[b * GH + 1], round & 1);
+                            ptx::tc_fence_after();
+                        }
+                        const uint64_t bk = BPRE ? b0 + (uint64_t)((((k >> 2) * (BSLOT / 2)) + (k & 3) * 32) >> 4)
+                                                 : b0 + (uint64_t)(k * BSTEP);
+                        ptx::mma_mxf4_ts(d, a0 + 8 * k, bk, IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                    }
+                    ptx::mma_commit_uniform(&empty[b]);
                 }
-                ptx::mma_commit_uniform(&empty[b]);
                 if (++b == NS) { b = 0; ++round; }
             }
-            ptx::mma_commit_uniform(&accf[acc]);
+            if (GH != 1) ptx::mma_commit_uniform(&accf[acc]);
 #ifdef GEMM_TRACE4
             if (tr4) { g_gemm_trace[8 * tl + 2] = clock64(); g_gemm_trace[8 * tl + 5] = fw; }
 #endif
@@ -1273,6 +1291,21 @@ __device__ __forceinline__ void mma_mxf4_ts2(uint32_t d, uint32_t a, uint64_t b,
         "r"(a), "l"(b), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb)
         : "memory");
 }
+__device__ __forceinline__ void mma_mxf4_ts2_one(uint32_t d, uint32_t a, uint64_t b, uint32_t idesc, uint32_t accumulate,
+                                                 uint32_t sfa, uint32_t sfb) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}" ::"r"(d),
+        "r"(a), "l"(b), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb)
+        : "memory");
+}
+__device__ __forceinline__ void commit_both_one(uint64_t *bar) {   // by the issuing thread alone
+    asm volatile(
+        "{\n\t.reg .b16 m;\n\tmov.b16 m, 3;\n\t"
+        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], m;\n\t}" ::"r"(
+            ptx::smem_u32(bar))
+        : "memory");
+}
 // commit the leader's outstanding MMAs to the barrier at this offset in BOTH CTAs
 __device__ __forceinline__ void commit_both(uint64_t *bar) {
     asm volatile(
@@ -1310,6 +1343,7 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
     constexpr int SF_COL = x2::SF_COL, BNP = x2::BNP, BNH = x2::BNH;
     using x2::cta_rank; using x2::cluster_id; using x2::num_clusters; using x2::cluster_sync;
     using x2::arrive_remote; using x2::wait_cluster_uniform; using x2::mma_mxf4_ts2; using x2::commit_both;
+    using x2::mma_mxf4_ts2_one; using x2::commit_both_one;
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t *ring = smem;                                        // [NP][PSLOT]
     uint8_t *bexp = smem + (size_t)NP * PSLOT;                   // [NS][BSLOT]
@@ -1543,13 +1577,29 @@ gemm_tc4x2_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant
                     ptx::tc_fence_after();
                     const uint32_t a0 = tmu + (uint32_t)(A_COL0 + 64 * b);
                     const uint64_t b0 = bdesc0 + (uint64_t)(((uint32_t)b * BSLOT) >> 4);
+#ifndef GEMM_X2_ELECT_STAGE
+#define GEMM_X2_ELECT_STAGE 0   // one elect per stage: measured LD-32K 2.91 -> 3.00 ms, off
+#endif
+                    if (GEMM_X2_ELECT_STAGE) {
+                        if (ptx::elect_one()) {
 #pragma unroll
-                    for (int k = 0; k < KBITS / 64; ++k)
-                        mma_mxf4_ts2(d, a0 + 8 * k, b0 + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u, sfa, sfb);
-                    commit_both(&empty[b]);
+                            for (int k = 0; k < KBITS / 64; ++k)
+                                mma_mxf4_ts2_one(d, a0 + 8 * k, b0 + (uint64_t)(k * BSTEP), IDESC,
+                                                 (s | k) != 0 ? 1u : 0u, sfa, sfb);
+                            commit_both_one(&empty[b]);
+                            if (s == nst - 1) commit_both_one(&accf[acc]);
+                        }
+                        __syncwarp();
+                    } else {
+#pragma unroll
+                        for (int k = 0; k < KBITS / 64; ++k)
+                            mma_mxf4_ts2(d, a0 + 8 * k, b0 + (uint64_t)(k * BSTEP), IDESC, (s | k) != 0 ? 1u : 0u,
+                                         sfa, sfb);
+                        commit_both(&empty[b]);
+                        if (s == nst - 1) commit_both(&accf[acc]);
+                    }
                     if (++b == NS) { b = 0; ++round; }
                 }
-                commit_both(&accf[acc]);
 #ifdef GEMM_TRACE4
                 if (tr4) { g_gemm_trace[8 * tl + 2] = clock64(); g_gemm_trace[8 * tl + 5] = fw; }
 #endif

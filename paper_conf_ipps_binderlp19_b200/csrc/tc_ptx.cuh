@@ -357,6 +357,27 @@ __device__ __forceinline__ void mma_mxf4_ts(uint32_t d, uint32_t a, uint64_t b, 
         "r"(a), "l"(b), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb)
         : "memory");
 }
+// The same MMA without its own elect.sync: for a block of MMAs issued by one already-elected
+// lane (one elect per stage instead of one per instruction).
+__device__ __forceinline__ void mma_mxf4_ts_one(uint32_t d, uint32_t a, uint64_t b, uint32_t idesc, uint32_t accumulate,
+                                                uint32_t sfa, uint32_t sfb) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::mxf4.block_scale.block32 [%0], [%1], %2, %3, [%5], [%6], p;\n\t}" ::"r"(d),
+        "r"(a), "l"(b), "r"(idesc), "r"(accumulate), "r"(sfa), "r"(sfb)
+        : "memory");
+}
+// tcgen05.commit by the calling thread alone (the thread that issued the MMAs it tracks).
+__device__ __forceinline__ void mma_commit_one(uint64_t *bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+                 : "memory");
+}
+// elect.sync: true in exactly one lane of the (converged) warp.
+__device__ __forceinline__ bool elect_one() {
+    uint32_t r;
+    asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\tselp.u32 %0, 1, 0, e;\n\t}" : "=r"(r));
+    return r != 0;
+}
 // tcgen05.commit to an mbarrier by the elect.sync leader (uniform UTCBAR).
 __device__ __forceinline__ void mma_commit_uniform(uint64_t *bar) {
     asm volatile(
