@@ -105,9 +105,11 @@ int choose_variant(int64_t m, int64_t n, int64_t nbits) {
     return tc_any_supported(m, n, nbits) ? SNP_VARIANT_TC : SNP_VARIANT_POPC;
 }
 
-// a7: the CUDA-core streaming kernel serves the few-query FastID shapes (nq <= STREAM_NQ in
-// AUTO, from the measured configs[4] sweep; any nq <= 4 when the CUDA-core variant is forced)
-constexpr int64_t STREAM_NQ = 3;   // profiles/round2/sweep_stream2.txt: 1-3 queries win everywhere
+// a7: the CUDA-core streaming kernel serves the few-query FastID shapes in AUTO from the
+// measured configs[4] sweep (profiles/round2/head/sweep/sweep_few.txt, after the tensor kernel's
+// per-stage MMA issue): 1-2 queries everywhere; 3 queries only for profiles above 12,288 SNPs
+// (3 x 20M x 16384: 8.2 vs 11.3 ms; 3 x 20M x 4096: tensor 2.14 vs 2.25 ms).  Any nq <= 4
+// when the CUDA-core variant is forced.
 bool use_stream(int64_t nq, int64_t nd, int64_t nbits) {
     const char *e = std::getenv("SNP_FASTID_STREAM");   // "0": never (A/B measurement hook)
     if (e && e[0] == '0') return false;
@@ -115,7 +117,7 @@ bool use_stream(int64_t nq, int64_t nd, int64_t nbits) {
     const int v = current_variant();
     if (v == SNP_VARIANT_POPC) return true;
     if (v == SNP_VARIANT_TC) return false;
-    return nq <= STREAM_NQ;
+    return nq <= 2 || (nq == 3 && nbits > 12288);
 }
 
 size_t pops_bytes(int64_t m, int64_t n) { return align256((size_t)m * 4) + align256((size_t)n * 4); }

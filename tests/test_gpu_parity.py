@@ -404,6 +404,19 @@ def test_search_all_ops_counts_and_best(snp, variant, nq, nd, nbits, pre):
         _variant(snp, "auto")
 
 
+def test_search_stream_dispatch(snp):
+    """a7 (profiles/round2/head/sweep/sweep_few.txt): AUTO streams 1-2 queries on the CUDA
+    cores, 3 queries only above 12,288 SNPs; the tensor kernel takes 3+ queries otherwise."""
+    for nq, nbits, want in ((1, 4096, "popc_stream"), (2, 2048, "popc_stream"), (3, 4096, "fastid_mxf4"),
+                            (3, 16384, "popc_stream"), (4, 16384, "fastid_mxf4")):
+        db = snpgen.fastid_db(5, np.arange(1000), nbits)
+        q, _ = snpgen.fastid_queries(5, nq, 1000, nbits)
+        _, best = snp.snp_fastid_search(pack_dev(snp, q), pack_dev(snp, db), nbits, ("xor",), counts=False)
+        assert snp.snp_last_kernel() == want, (nq, nbits, snp.snp_last_kernel())
+        rb, ri = oracle.best(oracle.counts(q, db, "xor"))
+        assert np.array_equal(u32(best[0][0]), rb) and np.array_equal(best[0][1].cpu().numpy(), ri)
+
+
 def test_search_kernel_choice(snp):
     for nq, nbits in ((32, 8192), (20, 9000)):   # the 32-wide resident-query kernel
         db = snpgen.fastid_db(4, np.arange(2048), nbits)
@@ -849,8 +862,8 @@ def test_fastid_stream_all_ops_counts_and_best(snp, nq, nd, nbits, pre):
     Q = pack_dev(snp, q, garbage_seed=4)
     pd = snp.snp_row_popc(D, nbits) if pre else None
     ops = ("and", "xor", "andnot", "notand")
-    # AUTO takes the streaming kernel for <= 3 queries (a7); the forced CUDA-core variant for <= 4
-    _variant(snp, "auto" if nq <= 3 else "popc")
+    # AUTO takes the streaming kernel for <= 2 queries (a7); the forced CUDA-core variant for <= 4
+    _variant(snp, "auto" if nq <= 2 else "popc")
     try:
         counts, best = snp.snp_fastid_search(Q, D, nbits, ops, index_base=7, popD=pd)
         assert snp.snp_last_kernel() == "popc_stream"
