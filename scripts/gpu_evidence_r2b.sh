@@ -3,6 +3,7 @@
 # reference arm), ncu launch lists and --set full captures of the dominant kernels.
 set -x
 mkdir -p gpurun_out/prof
+bash scripts/gpu_mg.sh > gpurun_out/prof/multirank_gloo_1gpu.txt 2>&1; echo mg=$?
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv
 timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/prof/pytest_gpu.log 2>&1; echo pytest=$?
 tail -3 gpurun_out/prof/pytest_gpu.log
