@@ -85,6 +85,9 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 #ifndef FASTID_ELECT_STAGE
 #define FASTID_ELECT_STAGE 1   // one elect.sync per stage's block of MMAs
 #endif
+#ifndef FASTID_ELECT_HALF
+#define FASTID_ELECT_HALF 1   // the same for the half-stage (GG = 4) instantiations
+#endif
 #ifndef FASTID_NACC
 #define FASTID_NACC 2   // TMEM accumulators (the MMA may run NACC - 1 tiles ahead of the epilogue)
 #endif
@@ -298,8 +301,11 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     // queries): FastID-1M 169.6 -> 168.9 us.  (With the per-MMA elect issue loop this ordering
     // measured 30 % slower; that loop was later found to be sensitive to code generation —
     // the cause was not isolated further.)
-    const int64_t n_early = FASTID_EARLY_TMA ? (total_it < NP ? total_it : (int64_t)NP) : 0;
-    if (FASTID_EARLY_TMA && warp == TMA_WARP && lane == 0) {
+    // Only for the 2-group (database popcounts given) kernels: with 4 expander groups and
+    // half-stage barriers it measured ~10 % slower (FastID-1M without popD 182 -> 200 us).
+    constexpr bool EARLY = FASTID_EARLY_TMA && GG == 2;
+    const int64_t n_early = EARLY ? (total_it < NP ? total_it : (int64_t)NP) : 0;
+    if (EARLY && warp == TMA_WARP && lane == 0) {
         for (int64_t it = 0; it < n_early; ++it) {
             const int64_t t = FASTID_TILE(it / nst);
             const int s = (int)(it % nst);
@@ -393,7 +399,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 const int64_t t = FASTID_TILE(tl);
                 const int32_t row0 = (int32_t)(t * BM);
                 for (int s = 0; s < nst; ++s, ++itp) {
-                    if (FASTID_EARLY_TMA && itp < n_early) {   // issued before the prologue
+                    if (EARLY && itp < n_early) {   // issued before the prologue
                         if (++p == NP) { p = 0; ++round; }
                         continue;
                     }
@@ -625,7 +631,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                     bd += SSTEP;
                     if (++b == NS) { b = 0; ++bround; }
                     continue;
-                } else if (NHALF == 2 && FASTID_ELECT_STAGE) {
+                } else if (NHALF == 2 && FASTID_ELECT_HALF) {
                     // half-stage barriers: the same per-half elected issue (elect.sync picks the
                     // same lane both times, so the commits track both halves' MMAs)
                     constexpr int KH = KBITS / 128;
@@ -665,7 +671,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 bd += SSTEP;
                 if (++b == NS) { b = 0; ++bround; }
             }
-            if (!FASTID_ELECT_STAGE) ptx::mma_commit_uniform(&accf[acc]);
+            if (!(NHALF == 1 ? FASTID_ELECT_STAGE : FASTID_ELECT_HALF)) ptx::mma_commit_uniform(&accf[acc]);
         }
         __syncwarp();
     } else {
