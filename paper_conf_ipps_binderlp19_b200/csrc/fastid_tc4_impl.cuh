@@ -85,6 +85,9 @@ constexpr int ACOLS = KW * 4;           // TMEM columns of an expanded A stage
 #ifndef FASTID_ELECT_STAGE
 #define FASTID_ELECT_STAGE 1   // one elect.sync per stage's block of MMAs
 #endif
+#ifndef FASTID_COUNT_GG2
+#define FASTID_COUNT_GG2 0   // experiment: 1024-bit stages with 2 groups also counting popcounts
+#endif
 #ifndef FASTID_ELECT_HALF
 #define FASTID_ELECT_HALF 1   // the same for the half-stage (GG = 4) instantiations
 #endif
@@ -992,8 +995,9 @@ cudaError_t FASTID_FN(launch_fastid_tc4)(const GemmArgs &a, int epi, cudaStream_
     sa.nops = 1; sa.ops[0] = a.op; sa.counts[0] = a.C;
     sa.ldo = a.ldc; sa.accumulate = a.accumulate;
     // queries <= 64 (fastid_tc4_supported)
-    if (FASTID_FN(fastid_bn)(sa.nq, sa.nbits) == 32) return sa.popD ? launch_f<32, 2>(sa, s) : launch_f<32, 4>(sa, s);
-    return sa.popD ? launch_f<64, 2>(sa, s) : launch_f<64, 4>(sa, s);
+    const bool two = sa.popD || (FASTID_COUNT_GG2 && KBITS == 1024);
+    if (FASTID_FN(fastid_bn)(sa.nq, sa.nbits) == 32) return two ? launch_f<32, 2>(sa, s) : launch_f<32, 4>(sa, s);
+    return two ? launch_f<64, 2>(sa, s) : launch_f<64, 4>(sa, s);
 }
 
 size_t FASTID_FN(fastid_search_tc4_ws_bytes)(int64_t nq, int nops) {
@@ -1001,8 +1005,9 @@ size_t FASTID_FN(fastid_search_tc4_ws_bytes)(int64_t nq, int nops) {
 }
 
 cudaError_t FASTID_FN(launch_fastid_search_tc4)(const SearchArgs &a, cudaStream_t s) {
-    if (FASTID_FN(fastid_bn)(a.nq, a.nbits) == 32) return a.popD ? launch_f<32, 2>(a, s) : launch_f<32, 4>(a, s);
-    return a.popD ? launch_f<64, 2>(a, s) : launch_f<64, 4>(a, s);
+    const bool two = a.popD || (FASTID_COUNT_GG2 && KBITS == 1024);
+    if (FASTID_FN(fastid_bn)(a.nq, a.nbits) == 32) return two ? launch_f<32, 2>(a, s) : launch_f<32, 4>(a, s);
+    return two ? launch_f<64, 2>(a, s) : launch_f<64, 4>(a, s);
 }
 
 }  // namespace snp
