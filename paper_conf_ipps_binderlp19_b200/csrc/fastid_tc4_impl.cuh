@@ -210,7 +210,10 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
     constexpr int G = GG, NEXP = Roles<GG>::NEXP, EPI_WARP0 = Roles<GG>::EPI_WARP0;
     constexpr int TMA_WARP = Roles<GG>::TMA_WARP, MMA_WARP = Roles<GG>::MMA_WARP;
     constexpr int NTHREADS = Roles<GG>::NTHREADS, NEPI = Roles<GG>::NEPI;
-    constexpr int NHALF = (GG == FASTID_HALF && KBITS == 512) ? 2 : 1;
+#ifndef FASTID_HALF1024
+#define FASTID_HALF1024 0   // experiment: half-stage barriers for the 2-group 1024-bit kernels
+#endif
+    constexpr int NHALF = ((GG == FASTID_HALF && KBITS == 512) || (FASTID_HALF1024 && GG == 2 && KBITS == 1024)) ? 2 : 1;
     using C = FCfg<BN, GG>;
     if constexpr (!C::OK) {
         return;   // never launched (launch_f refuses this configuration)
@@ -520,7 +523,7 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 for (int i = 0; i < 8; ++i)
                     expandA(wv[8 * h + i], v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
                 ptx::tmem_st32(tbase + 32 * h, v);
-                if (NHALF == 2 && h == 0) {   // publish the first half: the MMA may start on it
+                if (NHALF == 2 && h == KW / 16 - 1) {   // publish the first half: the MMA may start on it
                     ptx::tmem_st_wait();
                     ptx::tc_fence_before();
                     __syncwarp();
