@@ -28,18 +28,19 @@
 #include <cstdio>
 #include <cstdlib>
 
-// Output stores: ordinary write-back stores by default — measured equal or faster than
-// evict-first streaming stores on every workload (FastID-20M 125.1 -> 121.1 ms, LD-32K
-// 3.10 -> 3.05 ms, LD-2K step 17.4 -> 16.8 us, one box); -DGEMM_STORE_CS
-// selects st.global.cs (the output is written once and could push the packed operands out
-// of L2; not observed).
-#ifndef GEMM_STORE_CS
+// LD output stores: evict-first streaming stores (st.global.cs) by default — an LD output is
+// written once and must not push the packed operands out of L2 (with write-back stores LD-32K
+// re-read 2.2 instead of 1.6 GB from DRAM and ran ~2 % slower under the power cap);
+// -DGEMM_STORE_WB makes them write-back.  The swapped FastID count stores are write-back
+// (SWAP_STG_FN: FastID-20M 125.1 -> 121.1 ms).
+#ifdef GEMM_STORE_WB
 #define STG_OUT "st.global"
 #define STG_OUT_FN(p, v) (void)(*(p) = (v))
 #else
 #define STG_OUT "st.global.cs"
 #define STG_OUT_FN(p, v) __stcs((p), (v))
 #endif
+#define SWAP_STG_FN(p, v) (void)(*(p) = (v))
 
 namespace snp {
 
@@ -623,12 +624,12 @@ __device__ __forceinline__ void epi_swapped_counts(const GArgs &args, uint32_t (
 #endif
         if (ok) {
             if (acc) *o1 += x1;
-            else STG_OUT_FN(o1, x1);
+            else SWAP_STG_FN(o1, x1);
         }
         o1 += ldo;
         if (two) {
             const uint32_t x2 = cc2 * c + (cq2 * pq + b2);
-            if (ok) STG_OUT_FN(o2, x2);
+            if (ok) SWAP_STG_FN(o2, x2);
             o2 += ldo;
         }
     }
