@@ -119,7 +119,11 @@ struct Roles {
     static constexpr int NEPI = GG == 2 ? FASTID_NEPI2 : FASTID_NEPI;
     static constexpr int G = GG;
     static constexpr int NEXP = 4 * GG;
-    static constexpr int EPI_WARP0 = NEXP;
+#ifndef FASTID_EXP_HIGH
+#define FASTID_EXP_HIGH 0   // experiment: expanders above the epilogue warps (scheduler priority)
+#endif
+    static constexpr int EPI_WARP0 = FASTID_EXP_HIGH ? 0 : NEXP;
+    static constexpr int EXP_WARP0 = FASTID_EXP_HIGH ? NEPI : 0;
 #ifndef FASTID_MMA_FIRST
     static constexpr int TMA_WARP = NEXP + NEPI;
     static constexpr int MMA_WARP = NEXP + NEPI + 1;
@@ -207,7 +211,7 @@ __host__ __device__ constexpr uint32_t op_cc(int op) { return op == 0 ? 1u : op 
 template <int BN, int NOPS, bool BEST, bool ACC, int OPS, int GG>
 __global__ void __launch_bounds__(Roles<GG>::NTHREADS, 1)
 fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
-    constexpr int G = GG, NEXP = Roles<GG>::NEXP, EPI_WARP0 = Roles<GG>::EPI_WARP0;
+    constexpr int G = GG, NEXP = Roles<GG>::NEXP, EPI_WARP0 = Roles<GG>::EPI_WARP0, EXP_WARP0 = Roles<GG>::EXP_WARP0;
     constexpr int TMA_WARP = Roles<GG>::TMA_WARP, MMA_WARP = Roles<GG>::MMA_WARP;
     constexpr int NTHREADS = Roles<GG>::NTHREADS, NEPI = Roles<GG>::NEPI;
 #ifndef FASTID_HALF1024
@@ -420,11 +424,11 @@ fastid_tc4_kernel(const __grid_constant__ CUtensorMap tmD, const FArgs args) {
                 }
             }
         }
-    } else if (warp < NEXP) {
+    } else if (warp >= EXP_WARP0 && warp < EXP_WARP0 + NEXP) {
         // ------------------------------------------------------------ expanders
         // group g = warp / 4 handles iterations it = g, g+G, ...; warp (g, q) handles the
         // 32 database rows of lane quarter q for all 256 bits of the stage.
-        const int g = warp >> 2, qa = warp & 3;
+        const int g = (warp - EXP_WARP0) >> 2, qa = warp & 3;   // EXP_WARP0 is a multiple of 4
         const int arow = qa * 32 + lane;
         uint32_t popa = 0;
         int cur_tl = 0;       // tile whose popcount partial is being accumulated
