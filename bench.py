@@ -16,9 +16,12 @@ A *step* is one pass of the whole hot path over one batch:
            (counts and r2 written) for this rank's row block.
 value = SNP comparisons (bit pairs, M*N*nbits per op) of all ranks / max-over-ranks
 device time.  Inputs live in HBM before the timed region (the database is larger
-than L2; for the LD workloads L2 is flushed between timed steps, outside the
-per-step events).  `e2e` repeats the measurement through the public API with
-pinned host inputs (H2D of the genotype bytes) and a D2H of each step's result.
+than L2; for the LD workloads L2 is flushed before every timed step and the flushes'
+own time, measured by a graph of the flushes alone, is subtracted).  At N = 1 the
+timed steps are one CUDA-graph replay with events on the stream around it (no event
+nodes inside the graph).  `e2e` repeats the measurement through the public API with
+pinned host inputs (H2D of the genotype bytes) and a D2H of each step's result
+(FastID at N = 1: double-buffered on a copy stream, overlapped with the next step).
 """
 from __future__ import annotations
 
