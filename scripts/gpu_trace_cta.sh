@@ -1,5 +1,7 @@
-timeout 1200 python -m pytest tests/test_gpu_parity.py -q -x -k "ld or sym or general or ties or search_chunked" 2>&1 | tail -1
-for w in ld32k ld2k fastid20m; do st=20; [ $w = fastid20m ] && st=5
-  timeout 600 python bench.py --workload $w --steps $st --no-cpu-baseline --no-e2e 2>/dev/null | python -c "
-import sys, json; d = json.loads(sys.stdin.readline()); print('$w', round(d['ms_per_step'], 5), round(d['roofline']['kernel_ms'], 5), round(d['roofline']['frac'], 4), d['clocks']['reasons'])"
-done
+for r in 1 2; do for l in libsnp.so libsnp_ns2.so libsnp_ns4.so; do
+  SNP_LIB_PATH=$PWD/paper_conf_ipps_binderlp19_b200/$l timeout 600 python bench.py --workload ld32k --steps 10 --no-cpu-baseline --no-e2e 2>/dev/null | python -c "
+import sys, json
+try:
+    d = json.loads(sys.stdin.readline()); print('ld32k', '$l', round(d['ms_per_step'], 4), round(d['roofline']['kernel_ms'], 4), d['clocks']['sm_mhz'], d['clocks']['reasons'])
+except Exception as e: print('$l failed')"
+done; done
